@@ -1,0 +1,173 @@
+/*
+ * tid_oracle.c — CPU ORACLE for the texture-identification hot path.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and
+ * bench.py's cpu_baseline / --impl reference legs may load this library.  The
+ * product path (paper_conf_icpp_wangzll21_b200/) never links, imports or calls
+ * it, and shares no code, header, table or helper with it.
+ *
+ * What it computes is the PLAIN DEFINITION of the method, written out slowly
+ * and directly (no Eq. 1 expansion, no GEMM, no blocking, no fusion):
+ *
+ *   Wang et al., "Exploring HW/SW Co-Optimizations for Accelerating Large-scale
+ *   Texture Identification on Distributed GPUs", ICPP'21.  PAPER.md lines:
+ *   - squared Euclidean distance between two 128-d local features,
+ *     §3.3 P:327-333 and Eq. 1 left side rho^2(R,Q) P:353-354;
+ *   - 2-nearest neighbours of each QUERY feature over one reference image,
+ *     P:117, §3.1, Alg. 1 step 5 P:377, top-2 scan P:420-425;
+ *   - Lowe ratio test "below ... a predefined threshold", §3.1 P:280-284;
+ *   - good-match count per (query, reference), §3.1 P:284-288;
+ *   - one-to-many search: match the query against every reference one by one,
+ *     then rank (top-1 accuracy P:307-308), generalised to top-k.
+ *
+ * Readings where the paper is silent:
+ *   R1 ratio threshold = num/den (0.8 = 4/5), compared on SQUARED distances:
+ *      pass  <=>  den^2 * d1 < num^2 * d2   (strict "<", int64).
+ *   R2 ties: (d1,i1) = lexicographic min of (d_i, i); (d2,i2) = lexicographic
+ *      min over i != i1 (so duplicated nearest gives d2 == d1 -> fail).
+ *   R3 a reference with fewer than 2 keypoints gives no match (pass = 0).
+ *   R4 top-k order: (count desc, global reference id asc).
+ *   R5 padded / absent keypoints never participate (callers pass n_q, m_r).
+ *
+ * Arithmetic: every distance is an exact int64 sum of int64 squared
+ * differences (max 128*255^2 = 8,323,200).  No floating point anywhere.
+ */
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+#define DIM 128
+
+/* d(q, r) = sum_t (q_t - r_t)^2  — P:327-333, Eq. 1 LHS P:353-354 */
+int64_t oracle_sqdist(const uint8_t* q, const uint8_t* r) {
+  int64_t s = 0;
+  for (int t = 0; t < DIM; ++t) {
+    int64_t df = (int64_t)q[t] - (int64_t)r[t];
+    s += df * df;
+  }
+  return s;
+}
+
+/* Full distance matrix D[j][i] = d(Q_j, R_i) (used only by the oracle's own pins). */
+void oracle_dist_matrix(const uint8_t* Q, int32_t n, const uint8_t* R, int32_t m, int64_t* D) {
+  for (int32_t j = 0; j < n; ++j)
+    for (int32_t i = 0; i < m; ++i)
+      D[(size_t)j * m + i] = oracle_sqdist(Q + (size_t)j * DIM, R + (size_t)i * DIM);
+}
+
+/*
+ * 2-NN of one query feature over the m_r features of ONE reference image
+ * ("each query feature's nearest and second-nearest"; Alg. 1 step 5
+ * P:377; scan once keeping two candidates).  Reading R2 for ties.
+ * out = {d1, i1, d2, i2}; for m_r == 1 the second is {INT64_MAX, -1}; for
+ * m_r == 0 both are.
+ */
+void oracle_two_nn(const uint8_t* q, const uint8_t* R, int32_t m_r, int64_t out[4]) {
+  int64_t d1 = INT64_MAX, d2 = INT64_MAX;
+  int64_t i1 = -1, i2 = -1;
+  for (int32_t i = 0; i < m_r; ++i) {
+    int64_t d = oracle_sqdist(q, R + (size_t)i * DIM);
+    /* scanning i in increasing order: strict "<" keeps the lowest index on ties */
+    if (d < d1) {
+      d2 = d1; i2 = i1;
+      d1 = d;  i1 = i;
+    } else if (d < d2) {
+      d2 = d;  i2 = i;
+    }
+  }
+  out[0] = d1; out[1] = i1; out[2] = d2; out[3] = i2;
+}
+
+/* Ratio test, P:280-284 with readings R1 and R3. */
+int oracle_ratio_pass(int64_t d1, int64_t d2, int32_t m_r, uint32_t num, uint32_t den) {
+  if (m_r < 2) return 0;
+  int64_t lhs = (int64_t)den * (int64_t)den * d1;
+  int64_t rhs = (int64_t)num * (int64_t)num * d2;
+  return lhs < rhs;
+}
+
+/* Good-match count of one (query, reference) pair.  nn (nullable) gets [n_q][4]. */
+int32_t oracle_match_count(const uint8_t* Q, int32_t n_q, const uint8_t* R, int32_t m_r,
+                           uint32_t num, uint32_t den, int64_t* nn) {
+  int32_t count = 0;
+  for (int32_t j = 0; j < n_q; ++j) {
+    int64_t o[4];
+    oracle_two_nn(Q + (size_t)j * DIM, R, m_r, o);
+    if (nn) memcpy(nn + (size_t)j * 4, o, sizeof(o));
+    count += oracle_ratio_pass(o[0], o[2], m_r, num, den);
+  }
+  return count;
+}
+
+/*
+ * One-to-one verification over P pairs:
+ * pair p = (Q[p] with n_q[p] of n stored rows, R[p] with m_r[p] of m stored rows).
+ * counts[p]; nn (nullable) = [P][n][4] (rows j >= n_q[p] are left untouched).
+ */
+void oracle_verify(const uint8_t* Q, int32_t n, const uint8_t* R, int32_t m, int64_t P,
+                   const int32_t* n_q, const int32_t* m_r, uint32_t num, uint32_t den,
+                   int32_t* counts, int64_t* nn) {
+#pragma omp parallel for schedule(dynamic, 1)
+  for (int64_t p = 0; p < P; ++p) {
+    int32_t nq = n_q ? n_q[p] : n;
+    int32_t mr = m_r ? m_r[p] : m;
+    counts[p] = oracle_match_count(Q + (size_t)p * n * DIM, nq, R + (size_t)p * m * DIM, mr,
+                                   num, den, nn ? nn + (size_t)p * n * 4 : NULL);
+  }
+}
+
+/*
+ * One-to-many search counts ("calculating the similarity of query
+ * image and every reference image one by one"): counts[b][r] for B queries
+ * (n stored rows, n_q[b] valid) against R references (m stored rows, kp[r] valid).
+ */
+void oracle_search_counts(const uint8_t* Qs, const int32_t* n_q, int32_t n, int64_t B,
+                          const uint8_t* Rs, const int32_t* kp, int32_t m, int64_t R,
+                          uint32_t num, uint32_t den, int32_t* counts) {
+#pragma omp parallel for collapse(2) schedule(dynamic, 16)
+  for (int64_t b = 0; b < B; ++b)
+    for (int64_t r = 0; r < R; ++r)
+      counts[b * R + r] = oracle_match_count(Qs + (size_t)b * n * DIM, n_q ? n_q[b] : n,
+                                             Rs + (size_t)r * m * DIM, kp ? kp[r] : m,
+                                             num, den, NULL);
+}
+
+/* Ranking, reading R4: sort (count desc, id asc), take the first k. */
+typedef struct { int32_t count; int64_t id; } cand_t;
+
+static int cand_cmp(const void* a, const void* b) {
+  const cand_t* x = (const cand_t*)a;
+  const cand_t* y = (const cand_t*)b;
+  if (x->count != y->count) return x->count > y->count ? -1 : 1;
+  return (x->id > y->id) - (x->id < y->id);
+}
+
+/* counts [B][R] for reference ids id_base + r; k <= R. ids/cnts are [B][k]. */
+void oracle_topk(const int32_t* counts, int64_t B, int64_t R, int64_t id_base, int32_t k,
+                 int64_t* ids, int32_t* cnts) {
+  cand_t* c = (cand_t*)malloc(sizeof(cand_t) * (size_t)R);
+  for (int64_t b = 0; b < B; ++b) {
+    for (int64_t r = 0; r < R; ++r) { c[r].count = counts[b * R + r]; c[r].id = id_base + r; }
+    qsort(c, (size_t)R, sizeof(cand_t), cand_cmp);
+    for (int32_t t = 0; t < k; ++t) { ids[b * k + t] = c[t].id; cnts[b * k + t] = c[t].count; }
+  }
+  free(c);
+}
+
+/* Merge G ranked lists per query (each [G][B][k]) into one [B][k] by reading R4.
+ * Used by the oracle's own shard-merge pin. */
+void oracle_merge_topk(const int64_t* ids, const int32_t* cnts, int32_t G, int64_t B, int32_t k,
+                       int64_t* ids_out, int32_t* cnts_out) {
+  cand_t* c = (cand_t*)malloc(sizeof(cand_t) * (size_t)G * k);
+  for (int64_t b = 0; b < B; ++b) {
+    for (int32_t g = 0; g < G; ++g)
+      for (int32_t t = 0; t < k; ++t) {
+        size_t src = ((size_t)g * B + b) * k + t;
+        c[g * k + t].count = cnts[src];
+        c[g * k + t].id = ids[src];
+      }
+    qsort(c, (size_t)G * k, sizeof(cand_t), cand_cmp);
+    for (int32_t t = 0; t < k; ++t) { ids_out[b * k + t] = c[t].id; cnts_out[b * k + t] = c[t].count; }
+  }
+  free(c);
+}
