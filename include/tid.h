@@ -1,0 +1,189 @@
+/*
+ * tid.h — C ABI of the B200-native texture-identification hot path.
+ *
+ * Method: Wang, Zhang, Li, Lin, "Exploring HW/SW Co-Optimizations for
+ * Accelerating Large-scale Texture Identification on Distributed GPUs",
+ * ICPP'21.  Citations are PAPER.md line numbers (P:a-b).
+ *
+ * What the library computes (exact integer arithmetic, bit-identical to the
+ * definition):
+ *   d(q_j, r_i)  = sum_t (q_jt - r_it)^2 over d = 128 u8 dims     (Eq. 1)
+ *   2-NN of every QUERY keypoint over ONE reference image           (Alg. 1 step 5 P:377)
+ *   ratio test   den^2 * d1 < num^2 * d2  (strict)
+ *   count(q, r)  = number of query keypoints passing the ratio test
+ *   search       = count against every reference, rank by (count desc, global id asc),
+ *                  return the first k
+ * Ties in the 2-NN go to the lowest reference-keypoint index; a reference with
+ * fewer than 2 keypoints never matches.  Readings are listed in DESIGN.md.
+ *
+ * Conventions (every entry point):
+ *   - Status codes only; nothing throws across the ABI.  On failure the
+ *     thread-local message is available from tid_last_error().
+ *   - The caller owns every input and output buffer.  Buffers may be HOST
+ *     (pageable or pinned) or DEVICE memory of the index's device; the library
+ *     classifies each pointer (cudaPointerGetAttributes) and copies as needed.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *     Device outputs are valid once `stream` completes; host outputs are valid
+ *     when the call returns (the call synchronises the stream).
+ *   - One index per host thread; an index is not thread-safe.
+ *   - The library requires an sm_100a device (B200): TID_EUNSUPPORTED otherwise.
+ *     There is no CPU fallback.
+ */
+#ifndef TID_H_
+#define TID_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct tid_index tid_index; /* opaque; owns all device + pinned memory it allocates */
+
+typedef enum {
+  TID_OK = 0,
+  TID_EINVAL = -1,        /* bad argument (message says which)                       */
+  TID_ENOMEM = -2,        /* device / pinned allocation failed or capacity exceeded  */
+  TID_ECUDA = -3,         /* CUDA runtime / driver error                             */
+  TID_ENCCL = -4,         /* NCCL error                                              */
+  TID_EUNSUPPORTED = -5,  /* device is not sm_100 (tcgen05 kind::i8 needs sm_100a)   */
+  TID_ESTATE = -6         /* call not valid in the index's current state            */
+} tid_status;
+
+typedef struct {
+  int32_t  device;             /* CUDA device ordinal                                             */
+  int32_t  dim;                /* descriptor length d; must be 128 (SIFT)              */
+  int32_t  ref_kp;             /* m: stored keypoints per reference, 2..1024 (asymmetric budgets,
+                                  §7); rows beyond a reference's own count are padding */
+  int32_t  query_kp_max;       /* largest n a search/verify call may pass, 1..8192                */
+  uint32_t ratio_num;          /* ratio threshold num/den, each 1..65535 (0.8 = 4/5)   */
+  uint32_t ratio_den;
+  uint64_t hbm_budget_bytes;   /* reference descriptor bytes kept resident in HBM (level-1 cache,
+                                  §6.1); 0 = auto (free HBM minus 8 GiB workspace)      */
+  uint64_t host_budget_bytes;  /* pinned host tier capacity in bytes (level-2 cache); 0 = none    */
+  int64_t  id_base;            /* global id of this rank's first reference (shard offset)         */
+  int32_t  rank;               /* this process's rank; 0 when world_size == 1                     */
+  int32_t  world_size;         /* number of shards (GPUs); 1 = single GPU                         */
+  const void* nccl_unique_id;  /* 128-byte ncclUniqueId (same on all ranks) when world_size > 1   */
+} tid_config;
+
+/* Create an index on cfg->device.  Allocates the HBM arena lazily (on first add).
+ * With world_size > 1 this is collective: every rank must call it (NCCL init). */
+tid_status tid_index_create(const tid_config* cfg, tid_index** out);
+
+/* Release every device / pinned buffer and the NCCL communicator.  NULL is a no-op. */
+tid_status tid_index_destroy(tid_index* idx);
+
+/*
+ * Append `count` references (offline ingest, Alg. 1 step 1 P:372).
+ *   desc       : u8 [count][ref_kp][128], host or device.  Row i of reference r is
+ *                keypoint i; rows >= kp_counts[r] are ignored (zeroed in the arena).
+ *   kp_counts  : int32 [count] keypoints per reference (0..ref_kp), host or device;
+ *                NULL = every reference has ref_kp keypoints.  A reference with < 2
+ *                keypoints is stored but can never match (count 0).
+ *   first_local_id (out, nullable): local index of the first appended reference;
+ *                its global id is cfg.id_base + local index.
+ * References go to HBM until hbm_budget_bytes, then to the pinned host tier until
+ * host_budget_bytes (FIFO order preserved).  All-or-nothing: TID_ENOMEM adds nothing.
+ * The squared norms N_R are computed here and kept in HBM.
+ */
+tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t* kp_counts,
+                              int64_t count, int64_t* first_local_id);
+
+/*
+ * One-to-many search, batched over B queries.
+ *   queries          : u8 [B][n][128], host or device; n <= query_kp_max.
+ *   n_q              : int32 [B] valid keypoints per query (<= n), host or device; NULL = all n.
+ *   k                : 1..64 and k <= total references over all ranks.
+ *   ref_ids_out      : int64 [B][k]  global reference ids, rank order (count desc, id asc).
+ *   match_counts_out : int32 [B][k]  their good-match counts.
+ * With world_size > 1 the call is collective: every rank passes the same queries
+ * and receives the same merged result (one NCCL all-gather of B*k candidates).
+ */
+tid_status tid_search(tid_index* idx, const uint8_t* queries, const int32_t* n_q, int32_t n,
+                      int64_t B, int32_t k, int64_t* ref_ids_out, int32_t* match_counts_out,
+                      void* stream);
+
+/*
+ * Parity/debug entry: the full local count matrix of a search (this rank's references only).
+ *   counts_out : uint32 [B][num_local_references], host or device.
+ */
+tid_status tid_search_counts(tid_index* idx, const uint8_t* queries, const int32_t* n_q, int32_t n,
+                             int64_t B, uint32_t* counts_out, void* stream);
+
+/*
+ * One-to-one verification of P independent pairs.
+ * Does not touch the index's references (uses its ratio, device and workspace).
+ *   q      : u8 [P][n][128], r : u8 [P][m][128] (host or device); n <= query_kp_max, 2 <= m <= 1024.
+ *   n_q    : int32 [P] valid query rows per pair (nullable = n);
+ *   m_r    : int32 [P] valid reference rows per pair (nullable = m).
+ *   counts_out : uint32 [P] good-match counts.
+ *   nn_out : nullable int32 [P][n][4] = (d1, i1, d2, i2) per query row, the exact
+ *            squared distances and reference-keypoint indices of the two nearest
+ *            neighbours (Alg. 1 step 8's 2 x n output); a missing
+ *            neighbour (m_r < 2) is (-1, -1).  Rows >= n_q[p] are not written.
+ */
+tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t* r, int32_t m,
+                      int64_t P, const int32_t* n_q, const int32_t* m_r,
+                      uint32_t* counts_out, int32_t* nn_out, void* stream);
+
+/*
+ * Shard merge: merge G ranked lists per query into one.
+ *   ids_in/counts_in : [G][B][k] (int64 / int32), host or device, each list in rank order.
+ *   ids_out/counts_out : [B][k] in (count desc, id asc) order.
+ * Used internally after the NCCL all-gather; exported so a single GPU can run G
+ * virtual shards and prove merge == single-GPU.
+ */
+tid_status tid_merge_topk(tid_index* idx, const int64_t* ids_in, const int32_t* counts_in,
+                          int32_t G, int64_t B, int32_t k, int64_t* ids_out, int32_t* counts_out,
+                          void* stream);
+
+/* 128-byte ncclUniqueId for rank 0 to broadcast before tid_index_create. */
+tid_status tid_nccl_unique_id(void* out128);
+
+typedef struct {
+  int64_t num_references;      /* local references (HBM + host tier)                 */
+  int64_t hbm_references;      /* resident in the HBM arena                          */
+  int64_t host_references;     /* in the pinned host tier (streamed per search)      */
+  int64_t hbm_bytes;           /* device bytes allocated by the index                */
+  int64_t host_bytes;          /* pinned host bytes allocated by the index           */
+  int32_t num_sms;
+  int32_t world_size;
+} tid_info;
+
+tid_status tid_get_info(const tid_index* idx, tid_info* out);
+
+/*
+ * Kernel timing (CUDA events recorded on the stream each kernel is launched on).
+ * enable != 0 starts recording and clears the accumulators.
+ */
+typedef struct {
+  int64_t match_launches;      /* fused TMA->tcgen05->top-2->ratio->count kernel launches */
+  double  match_ms;            /* summed device time of those launches                    */
+  int64_t kernel_launches;     /* all kernels of this library launched while enabled      */
+  int64_t h2d_bytes;           /* host->device bytes copied by the library                */
+  int64_t d2h_bytes;           /* device->host bytes copied by the library                */
+} tid_stats;
+
+tid_status tid_profile(tid_index* idx, int32_t enable);
+tid_status tid_get_stats(tid_index* idx, tid_stats* out); /* synchronises recorded events */
+
+/* Tuning knobs (0 = automatic).  refs_per_job: references resident per CTA job (1..4);
+ * grid: persistent CTAs for the match kernel; host_chunk_refs: references per
+ * host-tier staging buffer. */
+typedef struct {
+  int32_t refs_per_job;
+  int32_t grid;
+  int64_t host_chunk_refs;
+} tid_tuning;
+
+tid_status tid_set_tuning(tid_index* idx, const tid_tuning* t);
+
+/* Thread-local message describing the last non-OK status of this thread ("" if none). */
+const char* tid_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* TID_H_ */

@@ -1,0 +1,885 @@
+// tid_api.cu — C-ABI implementation (include/tid.h): index lifecycle, reference arena
+// (HBM level-1 + pinned-host level-2, §6.1), host-tier streaming with a
+// double-buffered copy stream (§6.2), query batching, shard merge over NCCL.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/tid.h"
+#include "tid_kernels.cuh"
+
+using namespace tid;
+
+namespace {
+
+thread_local std::string g_err;
+
+tid_status fail(tid_status st, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return st;
+}
+
+#define CU(call)                                                                                  \
+  do {                                                                                            \
+    cudaError_t e__ = (call);                                                                     \
+    if (e__ != cudaSuccess)                                                                       \
+      return fail(TID_ECUDA, "%s:%d %s: %s", __FILE__, __LINE__, #call, cudaGetErrorString(e__)); \
+  } while (0)
+
+// NCCL is resolved at run time (dlopen) so that the library never forces its own NCCL
+// build into a process that already loaded another one (e.g. PyTorch's): an already
+// loaded libnccl.so.2 is preferred, then $TID_NCCL_LIBRARY, then the system library.
+struct NcclApi {
+  bool ok = false;
+  std::string err;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+  const char* (*GetErrorString)(ncclResult_t) = nullptr;
+};
+
+const NcclApi& nccl() {
+  static NcclApi api;
+  static bool tried = false;
+  if (tried) return api;
+  tried = true;
+  void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+  if (!h) {
+    const char* env = getenv("TID_NCCL_LIBRARY");
+    if (env && *env) h = dlopen(env, RTLD_NOW | RTLD_LOCAL);
+  }
+  if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_LOCAL);
+  if (!h) {
+    api.err = std::string("cannot load libnccl.so.2: ") + dlerror();
+    return api;
+  }
+  api.GetUniqueId = reinterpret_cast<decltype(api.GetUniqueId)>(dlsym(h, "ncclGetUniqueId"));
+  api.CommInitRank = reinterpret_cast<decltype(api.CommInitRank)>(dlsym(h, "ncclCommInitRank"));
+  api.CommDestroy = reinterpret_cast<decltype(api.CommDestroy)>(dlsym(h, "ncclCommDestroy"));
+  api.AllGather = reinterpret_cast<decltype(api.AllGather)>(dlsym(h, "ncclAllGather"));
+  api.GetErrorString = reinterpret_cast<decltype(api.GetErrorString)>(dlsym(h, "ncclGetErrorString"));
+  api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.AllGather && api.GetErrorString;
+  if (!api.ok) api.err = "libnccl.so.2 lacks a required symbol";
+  return api;
+}
+
+#define NC(call)                                                                                          \
+  do {                                                                                                    \
+    if (!nccl().ok) return fail(TID_ENCCL, "%s", nccl().err.c_str());                                    \
+    ncclResult_t r__ = (call);                                                                            \
+    if (r__ != ncclSuccess)                                                                               \
+      return fail(TID_ENCCL, "%s:%d %s: %s", __FILE__, __LINE__, #call, nccl().GetErrorString(r__));     \
+  } while (0)
+
+#define TRY(x)                    \
+  do {                            \
+    tid_status s__ = (x);         \
+    if (s__ != TID_OK) return s__; \
+  } while (0)
+
+// ---------------------------------------------------------------- growable device buffer
+struct DevBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+  tid_status ensure(size_t need, const char* what) {
+    if (need <= bytes) return TID_OK;
+    if (p) cudaFree(p);
+    p = nullptr;
+    bytes = 0;
+    size_t want = std::max(need, static_cast<size_t>(1) << 20);
+    cudaError_t e = cudaMalloc(&p, want);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      p = nullptr;
+      return fail(TID_ENOMEM, "cudaMalloc(%zu) for %s: %s", want, what, cudaGetErrorString(e));
+    }
+    bytes = want;
+    return TID_OK;
+  }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    bytes = 0;
+  }
+  template <class T> T* as() const { return static_cast<T*>(p); }
+};
+
+// ---------------------------------------------------------------- tensor maps (driver entry point)
+typedef CUresult (*PFN_encodeTiled_t)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                      const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                      CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+PFN_encodeTiled_t encode_fn() {
+  static PFN_encodeTiled_t fn = nullptr;
+  if (!fn) {
+    void* ptr = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &ptr, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_encodeTiled_t>(ptr);
+  }
+  return fn;
+}
+
+// u8 tensor [count][rows][128] -> 3-D map with box {128 B, box_rows, 1}, SWIZZLE_128B,
+// out-of-bounds rows zero-filled (this is how ragged n / m are padded to the tile).
+tid_status make_map(CUtensorMap* map, const void* base, int64_t count, int64_t rows, int box_rows) {
+  PFN_encodeTiled_t fn = encode_fn();
+  if (!fn) return fail(TID_ECUDA, "cuTensorMapEncodeTiled entry point unavailable");
+  if (reinterpret_cast<uintptr_t>(base) % 16) return fail(TID_EINVAL, "descriptor buffer must be 16-byte aligned");
+  cuuint64_t dims[3] = {static_cast<cuuint64_t>(kDim), static_cast<cuuint64_t>(rows),
+                        static_cast<cuuint64_t>(std::max<int64_t>(count, 1))};
+  cuuint64_t strides[2] = {static_cast<cuuint64_t>(kDim), static_cast<cuuint64_t>(rows * kDim)};
+  cuuint32_t box[3] = {static_cast<cuuint32_t>(kDim), static_cast<cuuint32_t>(box_rows), 1};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, 3, const_cast<void*>(base), dims, strides, box, estr,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(TID_ECUDA, "cuTensorMapEncodeTiled failed (%d)", static_cast<int>(r));
+  return TID_OK;
+}
+
+bool is_device_ptr(const void* p) {
+  if (!p) return false;
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+struct Segment {          // one cudaMalloc'd piece of the HBM arena
+  uint8_t* desc = nullptr;   // [cap][m][128]
+  int32_t* colkey = nullptr; // [cap][cpr*256]
+  int64_t cap = 0, count = 0, first = 0;  // first = local index of its first reference
+};
+
+struct HostSegment {      // one cudaHostAlloc'd piece of the pinned host tier
+  uint8_t* desc = nullptr;   // [cap][m][128] raw (as added)
+  int64_t cap = 0, count = 0, first = 0;
+};
+
+}  // namespace
+
+struct tid_index {
+  tid_config cfg{};
+  int device = 0;
+  int num_sms = 148;
+  int cpr = 1;                    // chunks per reference = ceil(ref_kp / 256)
+  int64_t ref_bytes = 0;          // bytes per stored reference
+  uint64_t hbm_budget = 0, host_budget = 0;
+  std::vector<Segment> segs;
+  std::vector<HostSegment> hsegs;
+  std::vector<int32_t> host_kp;   // keypoint counts of host-tier references
+  int64_t n_hbm = 0, n_host = 0;
+  int64_t hbm_alloc = 0, host_alloc = 0;
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t ev_h2d[2] = {nullptr, nullptr}, ev_free[2] = {nullptr, nullptr};
+  // workspaces
+  DevBuf ws_q, ws_nq, ws_nvalid, ws_counts, ws_cand, ws_keys, ws_gather, ws_ids, ws_cnts, ws_r, ws_colkey, ws_nn,
+      ws_kp, ws_mr;
+  DevBuf stage_desc[2], stage_colkey[2], stage_kp[2];
+  int64_t host_chunk = 0;
+  tid_tuning tune{};
+  ncclComm_t comm = nullptr;
+  // profiling
+  bool prof = false;
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> prof_ev;
+  size_t prof_used = 0;
+  tid_stats stats{};
+};
+
+namespace {
+
+tid_status set_device(tid_index* idx) {
+  CU(cudaSetDevice(idx->device));
+  return TID_OK;
+}
+
+void count_kernel(tid_index* idx, int n = 1) {
+  if (idx->prof) idx->stats.kernel_launches += n;
+}
+
+tid_status copy_in(tid_index* idx, void* dst, const void* src, size_t bytes, cudaStream_t s) {
+  if (bytes == 0) return TID_OK;
+  const bool dev = is_device_ptr(src);
+  CU(cudaMemcpyAsync(dst, src, bytes, dev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, s));
+  if (!dev && idx->prof) idx->stats.h2d_bytes += static_cast<int64_t>(bytes);
+  return TID_OK;
+}
+
+tid_status copy_out(tid_index* idx, void* dst, const void* src, size_t bytes, cudaStream_t s, bool* host_out) {
+  if (bytes == 0) return TID_OK;
+  const bool dev = is_device_ptr(dst);
+  CU(cudaMemcpyAsync(dst, src, bytes, dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, s));
+  if (!dev) {
+    *host_out = true;
+    if (idx->prof) idx->stats.d2h_bytes += static_cast<int64_t>(bytes);
+  }
+  return TID_OK;
+}
+
+// Choose job decomposition of a search launch: refs per job G and queries per job.
+void plan_search(const tid_index* idx, int64_t n_refs, int64_t B, int T, int* G_out, int* qpj_out) {
+  const int max_g = kMaxSlots / idx->cpr;
+  int G = idx->tune.refs_per_job > 0 ? std::min(idx->tune.refs_per_job, max_g) : max_g;
+  const int64_t target_jobs = 2LL * idx->num_sms;
+  // spread small reference sets over more CTAs (fewer resident refs per job)
+  while (G > 1 && ceil_div(n_refs, G) < target_jobs) --G;
+  int64_t groups = ceil_div(n_refs, G);
+  int qpj = static_cast<int>(B);
+  // still too few jobs: split the query batch too (each job then re-reads its refs)
+  while (groups * ceil_div(B, qpj) < target_jobs && qpj > 1) qpj = (qpj + 1) / 2;
+  (void)T;
+  *G_out = G;
+  *qpj_out = qpj;
+}
+
+tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const uint8_t* rbase, int64_t map_count,
+                               int64_t ref_map_base, const int32_t* colkey, int64_t n_refs, int64_t B, int32_t n,
+                               int T, const int32_t* nvalid, uint32_t* counts, int64_t ldc, int64_t col0,
+                               cudaStream_t s) {
+  if (n_refs <= 0) return TID_OK;
+  CUtensorMap rmap;
+  TRY(make_map(&rmap, rbase, map_count, idx->cfg.ref_kp, kBN));
+  MatchParams p{};
+  p.mode = kModeSearch;
+  int G, qpj;
+  plan_search(idx, n_refs, B, T, &G, &qpj);
+  p.refs_per_job = G;
+  p.cpr = idx->cpr;
+  p.tiles_per_q = T;
+  p.num_q = static_cast<int32_t>(B);
+  p.q_per_job = qpj;
+  p.n_qchunks = static_cast<int32_t>(ceil_div(B, qpj));
+  p.n_jobs = static_cast<int32_t>(ceil_div(n_refs, G) * p.n_qchunks);
+  p.n_refs = n_refs;
+  p.ref_map_base = ref_map_base;
+  p.colkey = colkey;
+  p.nq = idx->ws_nq.as<int32_t>();
+  p.n_valid = nvalid;
+  p.n_rows = n;
+  p.counts = counts;
+  p.ldc = ldc;
+  p.col0 = col0;
+  p.nn_out = nullptr;
+  p.num2 = idx->cfg.ratio_num * idx->cfg.ratio_num;
+  p.den2 = idx->cfg.ratio_den * idx->cfg.ratio_den;
+  int grid = idx->tune.grid > 0 ? idx->tune.grid : idx->num_sms;
+  grid = static_cast<int>(std::min<int64_t>(grid, p.n_jobs));
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  if (idx->prof) {
+    if (idx->prof_used == idx->prof_ev.size()) {
+      cudaEvent_t a, b;
+      CU(cudaEventCreate(&a));
+      CU(cudaEventCreate(&b));
+      idx->prof_ev.push_back({a, b});
+    }
+    e0 = idx->prof_ev[idx->prof_used].first;
+    e1 = idx->prof_ev[idx->prof_used].second;
+    ++idx->prof_used;
+    CU(cudaEventRecord(e0, s));
+  }
+  cudaError_t e = launch_match(p, qmap, rmap, grid, s);
+  if (e != cudaSuccess) return fail(TID_ECUDA, "match kernel launch: %s", cudaGetErrorString(e));
+  if (idx->prof) {
+    CU(cudaEventRecord(e1, s));
+    idx->stats.match_launches++;
+    count_kernel(idx);
+  }
+  return TID_OK;
+}
+
+// Full local count matrix counts[B][R_local] for queries already resident in ws_q.
+tid_status run_counts(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, int32_t n, int64_t B,
+                      uint32_t* counts, cudaStream_t s) {
+  const int T = static_cast<int>(ceil_div(n, kBM));
+  const int64_t R = idx->n_hbm + idx->n_host;
+  TRY(idx->ws_nq.ensure(static_cast<size_t>(B) * T * kBM * 4, "query norms"));
+  launch_query_prep(dq, B, n, T, idx->ws_nq.as<int32_t>(), s);
+  count_kernel(idx);
+  CU(cudaMemsetAsync(counts, 0, static_cast<size_t>(B) * R * 4, s));
+  CUtensorMap qmap;
+  TRY(make_map(&qmap, dq, B, n, kBM));
+  // level 1: HBM-resident segments
+  for (const Segment& sg : idx->segs)
+    TRY(launch_search_range(idx, qmap, sg.desc, sg.cap, 0, sg.colkey, sg.count, B, n, T, nvalid, counts, R, sg.first, s));
+  // level 2: pinned host tier, streamed through two HBM staging buffers on the copy stream
+  if (idx->n_host > 0) {
+    const int64_t chunk = idx->host_chunk;
+    const int64_t rb = idx->ref_bytes;
+    for (int b = 0; b < 2; ++b) {
+      TRY(idx->stage_desc[b].ensure(static_cast<size_t>(chunk * rb), "host-tier staging"));
+      TRY(idx->stage_colkey[b].ensure(static_cast<size_t>(chunk) * idx->cpr * kBN * 4, "staging keys"));
+      TRY(idx->stage_kp[b].ensure(static_cast<size_t>(chunk) * 4, "staging kp"));
+    }
+    // the copy stream must not overwrite staging buffers still read by a previous call
+    CU(cudaEventRecord(idx->ev_free[0], s));
+    CU(cudaEventRecord(idx->ev_free[1], s));
+    struct Piece { const HostSegment* hs; int64_t off, cnt; };
+    std::vector<Piece> pieces;
+    for (const HostSegment& hs : idx->hsegs)
+      for (int64_t off = 0; off < hs.count; off += chunk) pieces.push_back({&hs, off, std::min(chunk, hs.count - off)});
+    auto issue_copy = [&](size_t i) -> tid_status {
+      const int b = static_cast<int>(i & 1);
+      const Piece& pc = pieces[i];
+      CU(cudaStreamWaitEvent(idx->copy_stream, idx->ev_free[b], 0));
+      CU(cudaMemcpyAsync(idx->stage_desc[b].p, pc.hs->desc + pc.off * rb, static_cast<size_t>(pc.cnt * rb),
+                         cudaMemcpyHostToDevice, idx->copy_stream));
+      CU(cudaMemcpyAsync(idx->stage_kp[b].p, idx->host_kp.data() + (pc.hs->first - idx->n_hbm) + pc.off,
+                         static_cast<size_t>(pc.cnt) * 4, cudaMemcpyHostToDevice, idx->copy_stream));
+      CU(cudaEventRecord(idx->ev_h2d[b], idx->copy_stream));
+      if (idx->prof) idx->stats.h2d_bytes += pc.cnt * rb + pc.cnt * 4;
+      return TID_OK;
+    };
+    if (!pieces.empty()) TRY(issue_copy(0));
+    for (size_t i = 0; i < pieces.size(); ++i) {
+      const int b = static_cast<int>(i & 1);
+      if (i + 1 < pieces.size()) TRY(issue_copy(i + 1));  // prefetch the next chunk while this one computes
+      CU(cudaStreamWaitEvent(s, idx->ev_h2d[b], 0));
+      const Piece& pc = pieces[i];
+      RefPrepParams rp{};
+      rp.desc = idx->stage_desc[b].as<uint8_t>();
+      rp.src = nullptr;
+      rp.kp = idx->stage_kp[b].as<int32_t>();
+      rp.colkey = idx->stage_colkey[b].as<int32_t>();
+      rp.count = pc.cnt;
+      rp.m = idx->cfg.ref_kp;
+      rp.cpr = idx->cpr;
+      launch_ref_prep(rp, s);
+      count_kernel(idx);
+      TRY(launch_search_range(idx, qmap, idx->stage_desc[b].as<uint8_t>(), chunk, 0, rp.colkey, pc.cnt, B, n, T,
+                              nvalid, counts, R, pc.hs->first + pc.off, s));
+      CU(cudaEventRecord(idx->ev_free[b], s));
+    }
+  }
+  return TID_OK;
+}
+
+// Stage queries / n_q on the device.
+tid_status stage_queries(tid_index* idx, const uint8_t* queries, const int32_t* n_q, int32_t n, int64_t B,
+                         const uint8_t** dq, const int32_t** dnv, cudaStream_t s) {
+  if (is_device_ptr(queries)) {
+    if (reinterpret_cast<uintptr_t>(queries) % 16) return fail(TID_EINVAL, "queries must be 16-byte aligned");
+    *dq = queries;
+  } else {
+    TRY(idx->ws_q.ensure(static_cast<size_t>(B) * n * kDim, "query staging"));
+    TRY(copy_in(idx, idx->ws_q.p, queries, static_cast<size_t>(B) * n * kDim, s));
+    *dq = idx->ws_q.as<uint8_t>();
+  }
+  *dnv = nullptr;
+  if (n_q) {
+    TRY(idx->ws_nvalid.ensure(static_cast<size_t>(B) * 4, "n_q"));
+    TRY(copy_in(idx, idx->ws_nvalid.p, n_q, static_cast<size_t>(B) * 4, s));
+    *dnv = idx->ws_nvalid.as<int32_t>();
+  }
+  return TID_OK;
+}
+
+tid_status check_search_args(tid_index* idx, const uint8_t* queries, int32_t n, int64_t B) {
+  if (!idx) return fail(TID_EINVAL, "null index");
+  if (!queries) return fail(TID_EINVAL, "null queries");
+  if (n < 1 || n > idx->cfg.query_kp_max) return fail(TID_EINVAL, "n=%d outside 1..query_kp_max=%d", n, idx->cfg.query_kp_max);
+  if (B < 1) return fail(TID_EINVAL, "B=%lld must be >= 1", static_cast<long long>(B));
+  if (B > (1LL << 31) / 2) return fail(TID_EINVAL, "B too large");
+  if (idx->n_hbm + idx->n_host == 0) return fail(TID_ESTATE, "index holds no references");
+  return TID_OK;
+}
+
+}  // namespace
+
+// =====================================================================================
+extern "C" {
+
+const char* tid_last_error(void) { return g_err.c_str(); }
+
+tid_status tid_nccl_unique_id(void* out128) {
+  if (!out128) return fail(TID_EINVAL, "null output");
+  ncclUniqueId id;
+  NC(nccl().GetUniqueId(&id));
+  static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+  memcpy(out128, &id, sizeof(id));
+  return TID_OK;
+}
+
+tid_status tid_index_create(const tid_config* cfg, tid_index** out) {
+  if (!cfg || !out) return fail(TID_EINVAL, "null argument");
+  *out = nullptr;
+  if (cfg->dim != kDim) return fail(TID_EINVAL, "dim=%d: only 128-d SIFT descriptors are supported", cfg->dim);
+  if (cfg->ref_kp < 2 || cfg->ref_kp > kMaxSlots * kBN)
+    return fail(TID_EINVAL, "ref_kp=%d outside 2..%d", cfg->ref_kp, kMaxSlots * kBN);
+  if (cfg->query_kp_max < 1 || cfg->query_kp_max > 8192)
+    return fail(TID_EINVAL, "query_kp_max=%d outside 1..8192", cfg->query_kp_max);
+  if (cfg->ratio_num < 1 || cfg->ratio_num > 65535 || cfg->ratio_den < 1 || cfg->ratio_den > 65535)
+    return fail(TID_EINVAL, "ratio %u/%u: num and den must be in 1..65535", cfg->ratio_num, cfg->ratio_den);
+  if (cfg->world_size < 1 || cfg->rank < 0 || cfg->rank >= cfg->world_size)
+    return fail(TID_EINVAL, "rank %d / world_size %d invalid", cfg->rank, cfg->world_size);
+  if (cfg->world_size > 1 && !cfg->nccl_unique_id) return fail(TID_EINVAL, "world_size > 1 needs nccl_unique_id");
+  if (cfg->id_base < 0) return fail(TID_EINVAL, "id_base must be >= 0");
+
+  int ndev = 0;
+  CU(cudaGetDeviceCount(&ndev));
+  if (cfg->device < 0 || cfg->device >= ndev) return fail(TID_EINVAL, "device %d not present (%d devices)", cfg->device, ndev);
+  cudaDeviceProp prop;
+  CU(cudaGetDeviceProperties(&prop, cfg->device));
+  if (prop.major != 10 || prop.minor != 0)
+    return fail(TID_EUNSUPPORTED, "device %d is sm_%d%d; this library is built for sm_100a (B200)", cfg->device,
+                prop.major, prop.minor);
+  CU(cudaSetDevice(cfg->device));
+
+  tid_index* idx = new tid_index();
+  idx->cfg = *cfg;
+  idx->cfg.nccl_unique_id = nullptr;
+  idx->device = cfg->device;
+  idx->num_sms = prop.multiProcessorCount;
+  idx->cpr = static_cast<int>(ceil_div(cfg->ref_kp, kBN));
+  idx->ref_bytes = static_cast<int64_t>(cfg->ref_kp) * kDim;
+  size_t free_b = 0, total_b = 0;
+  cudaMemGetInfo(&free_b, &total_b);
+  const uint64_t reserve = 8ull << 30;
+  idx->hbm_budget = cfg->hbm_budget_bytes ? cfg->hbm_budget_bytes : (free_b > reserve ? free_b - reserve : free_b / 2);
+  idx->host_budget = cfg->host_budget_bytes;
+  idx->host_chunk = 16384;
+  cudaError_t e = cudaStreamCreateWithFlags(&idx->copy_stream, cudaStreamNonBlocking);
+  for (int b = 0; b < 2 && e == cudaSuccess; ++b) {
+    e = cudaEventCreateWithFlags(&idx->ev_h2d[b], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&idx->ev_free[b], cudaEventDisableTiming);
+  }
+  if (e != cudaSuccess) {
+    tid_index_destroy(idx);
+    return fail(TID_ECUDA, "stream/event creation: %s", cudaGetErrorString(e));
+  }
+  if (cfg->world_size > 1) {
+    ncclUniqueId id;
+    memcpy(&id, cfg->nccl_unique_id, sizeof(id));
+    if (!nccl().ok) {
+      tid_index_destroy(idx);
+      return fail(TID_ENCCL, "%s", nccl().err.c_str());
+    }
+    ncclResult_t r = nccl().CommInitRank(&idx->comm, cfg->world_size, id, cfg->rank);
+    if (r != ncclSuccess) {
+      idx->comm = nullptr;
+      tid_index_destroy(idx);
+      return fail(TID_ENCCL, "ncclCommInitRank: %s", nccl().GetErrorString(r));
+    }
+  }
+  *out = idx;
+  return TID_OK;
+}
+
+tid_status tid_index_destroy(tid_index* idx) {
+  if (!idx) return TID_OK;
+  cudaSetDevice(idx->device);
+  cudaDeviceSynchronize();
+  for (Segment& s : idx->segs) { cudaFree(s.desc); cudaFree(s.colkey); }
+  for (HostSegment& h : idx->hsegs) cudaFreeHost(h.desc);
+  DevBuf* bufs[] = {&idx->ws_q, &idx->ws_nq, &idx->ws_nvalid, &idx->ws_counts, &idx->ws_cand, &idx->ws_keys,
+                    &idx->ws_gather, &idx->ws_ids, &idx->ws_cnts, &idx->ws_r, &idx->ws_colkey, &idx->ws_nn,
+                    &idx->ws_kp, &idx->ws_mr, &idx->stage_desc[0], &idx->stage_desc[1], &idx->stage_colkey[0],
+                    &idx->stage_colkey[1], &idx->stage_kp[0], &idx->stage_kp[1]};
+  for (DevBuf* b : bufs) b->release();
+  for (auto& pr : idx->prof_ev) { cudaEventDestroy(pr.first); cudaEventDestroy(pr.second); }
+  for (int b = 0; b < 2; ++b) {
+    if (idx->ev_h2d[b]) cudaEventDestroy(idx->ev_h2d[b]);
+    if (idx->ev_free[b]) cudaEventDestroy(idx->ev_free[b]);
+  }
+  if (idx->copy_stream) cudaStreamDestroy(idx->copy_stream);
+  if (idx->comm) nccl().CommDestroy(idx->comm);
+  delete idx;
+  return TID_OK;
+}
+
+tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t* kp_counts, int64_t count,
+                              int64_t* first_local_id) {
+  if (!idx) return fail(TID_EINVAL, "null index");
+  if (count < 0) return fail(TID_EINVAL, "count < 0");
+  if (count > 0 && !desc) return fail(TID_EINVAL, "null descriptors");
+  TRY(set_device(idx));
+  const int64_t first = idx->n_hbm + idx->n_host;
+  if (first_local_id) *first_local_id = first;
+  if (count == 0) return TID_OK;
+  const int64_t rb = idx->ref_bytes;
+  const bool dev_in = is_device_ptr(desc);
+  // how many go to HBM (FIFO: HBM fills first, then the host tier; §6.1)
+  int64_t hbm_room = idx->n_host > 0 ? 0 : static_cast<int64_t>(idx->hbm_budget / rb) - idx->n_hbm;
+  hbm_room = std::max<int64_t>(hbm_room, 0);
+  const int64_t to_hbm = std::min(count, hbm_room);
+  const int64_t to_host = count - to_hbm;
+  if (to_host > 0) {
+    const int64_t host_room = static_cast<int64_t>(idx->host_budget / rb) - idx->n_host;
+    if (to_host > host_room)
+      return fail(TID_ENOMEM, "capacity exceeded: %lld references do not fit (HBM room %lld, host room %lld)",
+                  static_cast<long long>(count), static_cast<long long>(hbm_room), static_cast<long long>(host_room));
+  }
+  // kp counts -> host copy (validated) and device copy
+  std::vector<int32_t> kp_host;
+  if (kp_counts) {
+    kp_host.resize(count);
+    CU(cudaMemcpy(kp_host.data(), kp_counts, static_cast<size_t>(count) * 4, cudaMemcpyDefault));
+    for (int64_t i = 0; i < count; ++i)
+      if (kp_host[i] < 0 || kp_host[i] > idx->cfg.ref_kp)
+        return fail(TID_EINVAL, "kp_counts[%lld]=%d outside 0..ref_kp", static_cast<long long>(i), kp_host[i]);
+  }
+  cudaStream_t s = nullptr;  // ingest is synchronous on the legacy stream
+  // ---- HBM part
+  int64_t done = 0;
+  while (done < to_hbm) {
+    Segment* sg = idx->segs.empty() ? nullptr : &idx->segs.back();
+    if (!sg || sg->count == sg->cap) {
+      const int64_t remaining_budget = static_cast<int64_t>(idx->hbm_budget / rb) - idx->n_hbm;
+      int64_t cap = std::max<int64_t>(to_hbm - done, std::min<int64_t>(idx->n_hbm, remaining_budget));
+      cap = std::min(cap, remaining_budget);
+      Segment ns;
+      ns.first = idx->n_hbm;
+      cudaError_t e1 = cudaMalloc(&ns.desc, static_cast<size_t>(cap * rb));
+      cudaError_t e2 = e1 == cudaSuccess ? cudaMalloc(&ns.colkey, static_cast<size_t>(cap) * idx->cpr * kBN * 4) : e1;
+      if (e1 != cudaSuccess || e2 != cudaSuccess) {
+        cudaGetLastError();
+        if (ns.desc) cudaFree(ns.desc);
+        return fail(TID_ENOMEM, "HBM arena allocation of %lld references failed", static_cast<long long>(cap));
+      }
+      ns.cap = cap;
+      idx->hbm_alloc += cap * rb + cap * idx->cpr * kBN * 4;
+      idx->segs.push_back(ns);
+      sg = &idx->segs.back();
+    }
+    const int64_t take = std::min(to_hbm - done, sg->cap - sg->count);
+    uint8_t* dst = sg->desc + sg->count * rb;
+    const uint8_t* src = desc + done * rb;
+    RefPrepParams rp{};
+    rp.desc = dst;
+    rp.m = idx->cfg.ref_kp;
+    rp.cpr = idx->cpr;
+    rp.count = take;
+    rp.colkey = sg->colkey + sg->count * idx->cpr * kBN;
+    if (dev_in) {
+      rp.src = src;
+    } else {
+      CU(cudaMemcpyAsync(dst, src, static_cast<size_t>(take * rb), cudaMemcpyHostToDevice, s));
+      rp.src = nullptr;
+    }
+    if (kp_counts) {
+      TRY(idx->ws_kp.ensure(static_cast<size_t>(take) * 4, "kp staging"));
+      CU(cudaMemcpyAsync(idx->ws_kp.p, kp_host.data() + done, static_cast<size_t>(take) * 4, cudaMemcpyHostToDevice, s));
+      rp.kp = idx->ws_kp.as<int32_t>();
+    }
+    launch_ref_prep(rp, s);
+    CU(cudaGetLastError());
+    CU(cudaStreamSynchronize(s));
+    sg->count += take;
+    idx->n_hbm += take;
+    done += take;
+  }
+  // ---- host tier part (raw bytes; zeroing + norms happen on the GPU when streamed)
+  int64_t hdone = 0;
+  while (hdone < to_host) {
+    HostSegment* hs = idx->hsegs.empty() ? nullptr : &idx->hsegs.back();
+    if (!hs || hs->count == hs->cap) {
+      const int64_t room = static_cast<int64_t>(idx->host_budget / rb) - idx->n_host;
+      int64_t cap = std::max<int64_t>(to_host - hdone, std::min<int64_t>(idx->n_host, room));
+      cap = std::min(cap, room);
+      HostSegment nh;
+      nh.first = idx->n_hbm + idx->n_host;
+      if (cudaHostAlloc(reinterpret_cast<void**>(&nh.desc), static_cast<size_t>(cap * rb), cudaHostAllocPortable) !=
+          cudaSuccess) {
+        cudaGetLastError();
+        return fail(TID_ENOMEM, "pinned host tier allocation of %lld bytes failed", static_cast<long long>(cap * rb));
+      }
+      nh.cap = cap;
+      idx->host_alloc += cap * rb;
+      idx->hsegs.push_back(nh);
+      hs = &idx->hsegs.back();
+    }
+    const int64_t take = std::min(to_host - hdone, hs->cap - hs->count);
+    const uint8_t* src = desc + (to_hbm + hdone) * rb;
+    CU(cudaMemcpy(hs->desc + hs->count * rb, src, static_cast<size_t>(take * rb), cudaMemcpyDefault));
+    for (int64_t i = 0; i < take; ++i)
+      idx->host_kp.push_back(kp_counts ? kp_host[to_hbm + hdone + i] : idx->cfg.ref_kp);
+    hs->count += take;
+    idx->n_host += take;
+    hdone += take;
+  }
+  return TID_OK;
+}
+
+tid_status tid_search_counts(tid_index* idx, const uint8_t* queries, const int32_t* n_q, int32_t n, int64_t B,
+                             uint32_t* counts_out, void* stream) {
+  TRY(check_search_args(idx, queries, n, B));
+  if (!counts_out) return fail(TID_EINVAL, "null counts_out");
+  TRY(set_device(idx));
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const uint8_t* dq;
+  const int32_t* dnv;
+  TRY(stage_queries(idx, queries, n_q, n, B, &dq, &dnv, s));
+  const int64_t R = idx->n_hbm + idx->n_host;
+  const bool dev_out = is_device_ptr(counts_out);
+  uint32_t* counts = counts_out;
+  if (!dev_out) {
+    TRY(idx->ws_counts.ensure(static_cast<size_t>(B) * R * 4, "count matrix"));
+    counts = idx->ws_counts.as<uint32_t>();
+  }
+  TRY(run_counts(idx, dq, dnv, n, B, counts, s));
+  bool host_out = false;
+  if (!dev_out) TRY(copy_out(idx, counts_out, counts, static_cast<size_t>(B) * R * 4, s, &host_out));
+  if (host_out) CU(cudaStreamSynchronize(s));
+  CU(cudaGetLastError());
+  return TID_OK;
+}
+
+tid_status tid_search(tid_index* idx, const uint8_t* queries, const int32_t* n_q, int32_t n, int64_t B, int32_t k,
+                      int64_t* ref_ids_out, int32_t* match_counts_out, void* stream) {
+  TRY(check_search_args(idx, queries, n, B));
+  if (!ref_ids_out || !match_counts_out) return fail(TID_EINVAL, "null outputs");
+  if (k < 1 || k > 64) return fail(TID_EINVAL, "k=%d outside 1..64", k);
+  const int64_t R = idx->n_hbm + idx->n_host;
+  if (idx->cfg.world_size == 1 && k > R)
+    return fail(TID_EINVAL, "k=%d exceeds the number of references (%lld)", k, static_cast<long long>(R));
+  TRY(set_device(idx));
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const uint8_t* dq;
+  const int32_t* dnv;
+  TRY(stage_queries(idx, queries, n_q, n, B, &dq, &dnv, s));
+  TRY(idx->ws_counts.ensure(static_cast<size_t>(B) * R * 4, "count matrix"));
+  uint32_t* counts = idx->ws_counts.as<uint32_t>();
+  TRY(run_counts(idx, dq, dnv, n, B, counts, s));
+  // a6: per-(query, segment) top-k, then merge the segments
+  int64_t segs = std::max<int64_t>(1, std::min<int64_t>(ceil_div(2LL * idx->num_sms, B), ceil_div(R, 4096)));
+  segs = std::min<int64_t>(segs, 1024);
+  TRY(idx->ws_cand.ensure(static_cast<size_t>(B) * segs * k * 8, "top-k candidates"));
+  launch_topk(counts, B, R, R, idx->cfg.id_base, k, static_cast<int32_t>(segs), idx->ws_cand.as<uint64_t>(), s);
+  count_kernel(idx);
+  TRY(idx->ws_ids.ensure(static_cast<size_t>(B) * k * 8, "ids"));
+  TRY(idx->ws_cnts.ensure(static_cast<size_t>(B) * k * 4, "counts"));
+  const bool dev_ids = is_device_ptr(ref_ids_out), dev_cnt = is_device_ptr(match_counts_out);
+  int64_t* ids = dev_ids ? ref_ids_out : idx->ws_ids.as<int64_t>();
+  int32_t* cnts = dev_cnt ? match_counts_out : idx->ws_cnts.as<int32_t>();
+  if (idx->cfg.world_size == 1) {
+    launch_merge(idx->ws_cand.as<uint64_t>(), static_cast<int32_t>(segs), B, k, segs * k, k, nullptr, ids, cnts, s);
+    count_kernel(idx);
+  } else {
+    // a9: local top-k -> NCCL all-gather over NVLink -> identical merge on every rank
+    const int G = idx->cfg.world_size;
+    TRY(idx->ws_keys.ensure(static_cast<size_t>(B) * k * 8, "local keys"));
+    TRY(idx->ws_gather.ensure(static_cast<size_t>(G) * B * k * 8, "gathered keys"));
+    launch_merge(idx->ws_cand.as<uint64_t>(), static_cast<int32_t>(segs), B, k, segs * k, k,
+                 idx->ws_keys.as<uint64_t>(), nullptr, nullptr, s);
+    NC(nccl().AllGather(idx->ws_keys.p, idx->ws_gather.p, static_cast<size_t>(B) * k, ncclUint64, idx->comm, s));
+    launch_merge(idx->ws_gather.as<uint64_t>(), G, B, k, k, B * k, nullptr, ids, cnts, s);
+    count_kernel(idx, 2);
+  }
+  CU(cudaGetLastError());
+  bool host_out = false;
+  if (!dev_ids) TRY(copy_out(idx, ref_ids_out, ids, static_cast<size_t>(B) * k * 8, s, &host_out));
+  if (!dev_cnt) TRY(copy_out(idx, match_counts_out, cnts, static_cast<size_t>(B) * k * 4, s, &host_out));
+  if (host_out) CU(cudaStreamSynchronize(s));
+  return TID_OK;
+}
+
+tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t* r, int32_t m, int64_t P,
+                      const int32_t* n_q, const int32_t* m_r, uint32_t* counts_out, int32_t* nn_out, void* stream) {
+  if (!idx) return fail(TID_EINVAL, "null index");
+  if (!q || !r || !counts_out) return fail(TID_EINVAL, "null argument");
+  if (n < 1 || n > idx->cfg.query_kp_max) return fail(TID_EINVAL, "n=%d outside 1..query_kp_max", n);
+  if (m < 2 || m > kMaxSlots * kBN) return fail(TID_EINVAL, "m=%d outside 2..%d", m, kMaxSlots * kBN);
+  if (P < 1 || P > (1LL << 31) - 1) return fail(TID_EINVAL, "P=%lld invalid", static_cast<long long>(P));
+  TRY(set_device(idx));
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const int cpr = static_cast<int>(ceil_div(m, kBN));
+  const int T = static_cast<int>(ceil_div(n, kBM));
+  const uint8_t* dq;
+  const int32_t* dnv;
+  TRY(stage_queries(idx, q, n_q, n, P, &dq, &dnv, s));
+  // references: device copy (host input) and packed column keys
+  const uint8_t* dr = r;
+  const size_t rbytes = static_cast<size_t>(P) * m * kDim;
+  const bool r_dev = is_device_ptr(r);
+  TRY(idx->ws_colkey.ensure(static_cast<size_t>(P) * cpr * kBN * 4, "pair keys"));
+  RefPrepParams rp{};
+  rp.m = m;
+  rp.cpr = cpr;
+  rp.count = P;
+  rp.colkey = idx->ws_colkey.as<int32_t>();
+  if (m_r) {
+    TRY(idx->ws_mr.ensure(static_cast<size_t>(P) * 4, "m_r"));
+    TRY(copy_in(idx, idx->ws_mr.p, m_r, static_cast<size_t>(P) * 4, s));
+    rp.kp = idx->ws_mr.as<int32_t>();
+  }
+  if (!r_dev || m_r) {
+    // host input, or masked rows to zero: work on our own copy
+    TRY(idx->ws_r.ensure(rbytes, "pair references"));
+    if (r_dev) {
+      rp.src = r;  // copy + zero rows >= m_r
+    } else {
+      TRY(copy_in(idx, idx->ws_r.p, r, rbytes, s));
+      rp.src = nullptr;
+    }
+    rp.desc = idx->ws_r.as<uint8_t>();
+    dr = idx->ws_r.as<uint8_t>();
+  } else {
+    if (reinterpret_cast<uintptr_t>(r) % 16) return fail(TID_EINVAL, "r must be 16-byte aligned");
+    rp.desc = nullptr;  // read-only: keys only
+    rp.src = r;
+  }
+  launch_ref_prep(rp, s);
+  count_kernel(idx);
+  TRY(idx->ws_nq.ensure(static_cast<size_t>(P) * T * kBM * 4, "query norms"));
+  launch_query_prep(dq, P, n, T, idx->ws_nq.as<int32_t>(), s);
+  count_kernel(idx);
+  const bool dev_counts = is_device_ptr(counts_out);
+  TRY(idx->ws_counts.ensure(static_cast<size_t>(P) * 4, "pair counts"));
+  uint32_t* counts = dev_counts ? counts_out : idx->ws_counts.as<uint32_t>();
+  CU(cudaMemsetAsync(counts, 0, static_cast<size_t>(P) * 4, s));
+  int32_t* nn = nullptr;
+  const bool dev_nn = nn_out && is_device_ptr(nn_out);
+  if (nn_out) {
+    if (dev_nn) {
+      nn = nn_out;
+    } else {
+      TRY(idx->ws_nn.ensure(static_cast<size_t>(P) * n * 16, "nn output"));
+      nn = idx->ws_nn.as<int32_t>();
+    }
+  }
+  CUtensorMap qmap, rmap;
+  TRY(make_map(&qmap, dq, P, n, kBM));
+  TRY(make_map(&rmap, dr, P, m, kBN));
+  MatchParams p{};
+  p.mode = kModeVerify;
+  p.n_jobs = static_cast<int32_t>(P);
+  p.refs_per_job = 1;
+  p.cpr = cpr;
+  p.tiles_per_q = T;
+  p.num_q = static_cast<int32_t>(P);
+  p.q_per_job = 1;
+  p.n_qchunks = 1;
+  p.n_refs = P;
+  p.ref_map_base = 0;
+  p.colkey = idx->ws_colkey.as<int32_t>();
+  p.nq = idx->ws_nq.as<int32_t>();
+  p.n_valid = dnv;
+  p.n_rows = n;
+  p.counts = counts;
+  p.ldc = 0;
+  p.col0 = 0;
+  p.nn_out = nn;
+  p.num2 = idx->cfg.ratio_num * idx->cfg.ratio_num;
+  p.den2 = idx->cfg.ratio_den * idx->cfg.ratio_den;
+  int grid = idx->tune.grid > 0 ? idx->tune.grid : idx->num_sms;
+  grid = static_cast<int>(std::min<int64_t>(grid, P));
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  if (idx->prof) {
+    if (idx->prof_used == idx->prof_ev.size()) {
+      cudaEvent_t a, b;
+      CU(cudaEventCreate(&a));
+      CU(cudaEventCreate(&b));
+      idx->prof_ev.push_back({a, b});
+    }
+    e0 = idx->prof_ev[idx->prof_used].first;
+    e1 = idx->prof_ev[idx->prof_used].second;
+    ++idx->prof_used;
+    CU(cudaEventRecord(e0, s));
+  }
+  cudaError_t e = launch_match(p, qmap, rmap, grid, s);
+  if (e != cudaSuccess) return fail(TID_ECUDA, "match kernel launch: %s", cudaGetErrorString(e));
+  if (idx->prof) {
+    CU(cudaEventRecord(e1, s));
+    idx->stats.match_launches++;
+    count_kernel(idx);
+  }
+  bool host_out = false;
+  if (!dev_counts) TRY(copy_out(idx, counts_out, counts, static_cast<size_t>(P) * 4, s, &host_out));
+  if (nn_out && !dev_nn) TRY(copy_out(idx, nn_out, nn, static_cast<size_t>(P) * n * 16, s, &host_out));
+  if (host_out) CU(cudaStreamSynchronize(s));
+  CU(cudaGetLastError());
+  return TID_OK;
+}
+
+tid_status tid_merge_topk(tid_index* idx, const int64_t* ids_in, const int32_t* counts_in, int32_t G, int64_t B,
+                          int32_t k, int64_t* ids_out, int32_t* counts_out, void* stream) {
+  if (!idx || !ids_in || !counts_in || !ids_out || !counts_out) return fail(TID_EINVAL, "null argument");
+  if (G < 1 || B < 1 || k < 1 || k > 64) return fail(TID_EINVAL, "bad G/B/k");
+  TRY(set_device(idx));
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const int64_t tot = static_cast<int64_t>(G) * B * k;
+  TRY(idx->ws_ids.ensure(static_cast<size_t>(tot) * 8, "merge ids"));
+  TRY(idx->ws_cnts.ensure(static_cast<size_t>(tot) * 4, "merge counts"));
+  TRY(idx->ws_gather.ensure(static_cast<size_t>(tot) * 8, "merge keys"));
+  TRY(copy_in(idx, idx->ws_ids.p, ids_in, static_cast<size_t>(tot) * 8, s));
+  TRY(copy_in(idx, idx->ws_cnts.p, counts_in, static_cast<size_t>(tot) * 4, s));
+  launch_pack_lists(idx->ws_ids.as<int64_t>(), idx->ws_cnts.as<int32_t>(), tot, idx->ws_gather.as<uint64_t>(), s);
+  TRY(idx->ws_keys.ensure(static_cast<size_t>(B) * k * 12, "merge out"));
+  int64_t* dids = reinterpret_cast<int64_t*>(idx->ws_keys.p);
+  int32_t* dcnt = reinterpret_cast<int32_t*>(idx->ws_keys.as<uint8_t>() + static_cast<size_t>(B) * k * 8);
+  launch_merge(idx->ws_gather.as<uint64_t>(), G, B, k, k, B * k, nullptr, dids, dcnt, s);
+  count_kernel(idx, 2);
+  CU(cudaGetLastError());
+  bool host_out = false;
+  TRY(copy_out(idx, ids_out, dids, static_cast<size_t>(B) * k * 8, s, &host_out));
+  TRY(copy_out(idx, counts_out, dcnt, static_cast<size_t>(B) * k * 4, s, &host_out));
+  if (host_out) CU(cudaStreamSynchronize(s));
+  return TID_OK;
+}
+
+tid_status tid_get_info(const tid_index* idx, tid_info* out) {
+  if (!idx || !out) return fail(TID_EINVAL, "null argument");
+  out->num_references = idx->n_hbm + idx->n_host;
+  out->hbm_references = idx->n_hbm;
+  out->host_references = idx->n_host;
+  out->hbm_bytes = idx->hbm_alloc;
+  out->host_bytes = idx->host_alloc;
+  out->num_sms = idx->num_sms;
+  out->world_size = idx->cfg.world_size;
+  return TID_OK;
+}
+
+tid_status tid_profile(tid_index* idx, int32_t enable) {
+  if (!idx) return fail(TID_EINVAL, "null index");
+  idx->prof = enable != 0;
+  idx->prof_used = 0;
+  memset(&idx->stats, 0, sizeof(idx->stats));
+  return TID_OK;
+}
+
+tid_status tid_get_stats(tid_index* idx, tid_stats* out) {
+  if (!idx || !out) return fail(TID_EINVAL, "null argument");
+  TRY(set_device(idx));
+  double ms = 0;
+  for (size_t i = 0; i < idx->prof_used; ++i) {
+    CU(cudaEventSynchronize(idx->prof_ev[i].second));
+    float t = 0;
+    CU(cudaEventElapsedTime(&t, idx->prof_ev[i].first, idx->prof_ev[i].second));
+    ms += t;
+  }
+  *out = idx->stats;
+  out->match_ms = ms;
+  return TID_OK;
+}
+
+tid_status tid_set_tuning(tid_index* idx, const tid_tuning* t) {
+  if (!idx || !t) return fail(TID_EINVAL, "null argument");
+  if (t->refs_per_job < 0 || t->refs_per_job > kMaxSlots) return fail(TID_EINVAL, "refs_per_job outside 0..4");
+  if (t->grid < 0) return fail(TID_EINVAL, "grid < 0");
+  if (t->host_chunk_refs < 0) return fail(TID_EINVAL, "host_chunk_refs < 0");
+  idx->tune = *t;
+  if (t->host_chunk_refs > 0) idx->host_chunk = t->host_chunk_refs;
+  return TID_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,82 @@
+// tid_kernels.cuh — sm_100a device code for the texture-identification hot path.
+//
+// Kernels:
+//   ref_prep_kernel    a1: zero padded reference rows, squared norms N_R -> packed column keys
+//   query_prep_kernel  a2: squared norms N_Q per query row
+//   match_kernel       a3+a4+a5: TMA -> tcgen05.mma.kind::i8 (u8 x u8 -> s32, TMEM) ->
+//                      exact top-2 epilogue in registers -> integer ratio test -> count
+//   topk_kernel        a6: per-(query, segment) top-k of the count matrix
+//   merge_kernel       a6/a9: merge ranked candidate lists (segments or shards)
+//
+// Everything is integer.  No distance matrix is ever written to HBM (P:374-386
+// materialised A in HBM; here the s32 accumulator lives only in TMEM).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+#include <cuda.h>
+
+namespace tid {
+
+constexpr int kDim = 128;          // SIFT descriptor length, bytes per keypoint row
+constexpr int kBM = 128;           // query keypoints per MMA tile (TMEM lanes)
+constexpr int kBN = 256;           // reference keypoints per chunk (MMA N, TMEM columns)
+constexpr int kQStages = 4;        // query-tile ring
+constexpr int kMaxSlots = 4;       // resident reference chunks per CTA
+constexpr int kNumThreads = 320;   // w0 TMA, w1 MMA, w2..w9 two epilogue groups of 4 warps
+constexpr uint32_t kQTileBytes = kBM * kDim;   // 16 KiB
+constexpr uint32_t kRTileBytes = kBN * kDim;   // 32 KiB
+constexpr uint32_t kColBytes = kBN * 4;        // 1 KiB of packed column keys per chunk
+constexpr int32_t kSentinelNorm = (1 << 23) - 1;  // > 128*255^2: padded columns never win
+
+// packed column key: colkey[i] = N_R[i] * 256 + i  (i = index within the 256-column chunk);
+// the epilogue forms key = colkey - 512 * S = 256 * (N_R - 2 q.r) + i, which orders
+// exactly like (d_ji, i) for a fixed query row (Alg. 1 step 4 + lowest-index tie-break).
+
+enum : int { kModeSearch = 0, kModeVerify = 1 };
+
+struct MatchParams {
+  int32_t mode;
+  int32_t n_jobs;
+  int32_t refs_per_job;      // G: references resident per job (search); 1 (verify)
+  int32_t cpr;               // 256-column chunks per reference (1..4)
+  int32_t tiles_per_q;       // ceil(n / 128)
+  int32_t num_q;             // queries in the launch (search: B; verify: P)
+  int32_t q_per_job;         // search: queries per job (splits B across jobs); verify: 1
+  int32_t n_qchunks;         // search: ceil(num_q / q_per_job)
+  int64_t n_refs;            // references in this launch
+  int64_t ref_map_base;      // index of the launch's first reference in the R tensor map
+  const int32_t* colkey;     // [n_refs][cpr*256] packed column keys (launch-relative)
+  const int32_t* nq;         // [num_q][tiles_per_q*128] squared query norms
+  const int32_t* n_valid;    // [num_q] valid query rows (nullable = n_rows)
+  int32_t n_rows;            // stored rows per query (n)
+  uint32_t* counts;          // search: [num_q][ldc] (+ col0); verify: [num_q]
+  int64_t ldc;
+  int64_t col0;
+  int32_t* nn_out;           // verify: [num_q][n_rows][4] or null
+  uint32_t num2, den2;       // ratio^2 = num2/den2
+};
+
+struct RefPrepParams {
+  uint8_t* desc;             // [count][m][128] destination (null = read-only, keys only)
+  const uint8_t* src;        // optional source to copy from (null = in place)
+  const int32_t* kp;         // [count] or null (= m)
+  int32_t* colkey;           // [count][cpr*256]
+  int64_t count;
+  int32_t m;
+  int32_t cpr;
+};
+
+void launch_ref_prep(const RefPrepParams& p, cudaStream_t s);
+void launch_query_prep(const uint8_t* q, int64_t B, int32_t n, int32_t tiles_per_q, int32_t* nq,
+                       cudaStream_t s);
+cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap,
+                         int grid, cudaStream_t s);
+void launch_topk(const uint32_t* counts, int64_t B, int64_t R, int64_t ldc, int64_t id_base, int32_t k,
+                 int32_t segs, uint64_t* cand_out, cudaStream_t s);
+void launch_merge(const uint64_t* cand, int32_t L, int64_t B, int32_t k, int64_t list_stride_b,
+                  int64_t list_stride_l, uint64_t* keys_out, int64_t* ids_out, int32_t* counts_out,
+                  cudaStream_t s);
+void launch_pack_lists(const int64_t* ids, const int32_t* counts, int64_t n, uint64_t* keys, cudaStream_t s);
+size_t match_smem_bytes();
+
+}  // namespace tid

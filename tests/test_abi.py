@@ -1,0 +1,79 @@
+"""CPU-side checks of the boundary: the C-ABI library builds for sm_100a, loads, and exports
+every symbol include/tid.h declares; the header and the binding agree.  No compute calls."""
+import ctypes
+import os
+import re
+import subprocess
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "tid.h")
+
+
+def _declared():
+    src = open(HEADER).read()
+    return sorted(set(re.findall(r"^\s*(?:tid_status|const char\*)\s+(tid_\w+)\s*\(", src, re.M)))
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_icpp_wangzll21_b200 import build
+    build.build()
+    import paper_conf_icpp_wangzll21_b200 as tid
+    return tid.load_library()
+
+
+def test_header_declares_boundary():
+    names = _declared()
+    for need in ("tid_index_create", "tid_add_references", "tid_verify", "tid_search", "tid_index_destroy",
+                 "tid_last_error"):
+        assert need in names
+
+
+def test_library_exports_every_declared_symbol(lib):
+    out = subprocess.check_output(["nm", "-D", "--defined-only", lib._name]).decode()
+    exported = set(re.findall(r" T (tid_\w+)", out))
+    missing = [n for n in _declared() if n not in exported]
+    assert not missing, f"declared in tid.h but not exported: {missing}"
+    import paper_conf_icpp_wangzll21_b200 as tid
+    assert sorted(tid.EXPORTS) == _declared()
+
+
+def test_library_is_sm100a_native(lib):
+    sass = subprocess.check_output(["/usr/local/cuda/bin/cuobjdump", "-sass", lib._name]).decode()
+    assert "sm_100a" in subprocess.check_output(["/usr/local/cuda/bin/cuobjdump", "-lelf", lib._name]).decode()
+    assert "UTCIMMA" in sass, "tcgen05.mma kind::i8 missing from SASS"
+    assert "LDTM" in sass, "tcgen05.ld missing from SASS"
+    assert "UTMALDG" in sass, "TMA tensor load missing from SASS"
+    assert not re.search(r"\s(HMMA|IMMA)\.", sass), "legacy mma.sync path present"
+
+
+def test_errors_without_gpu(lib):
+    """No GPU here: create must fail loudly (never fall back to the CPU)."""
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    import paper_conf_icpp_wangzll21_b200 as tid
+    with pytest.raises(tid.TidError):
+        tid.Index(ref_kp=256)
+    assert lib.tid_last_error() != b""
+
+
+def test_config_struct_matches_header():
+    import paper_conf_icpp_wangzll21_b200 as tid
+    src = open(HEADER).read()
+    body = re.search(r"typedef struct \{(.*?)\} tid_config;", src, re.S).group(1)
+    fields = re.findall(r"^\s*(?:const\s+)?\w+\*?\s+\*?(\w+)(?:,\s*(\w+))?;", body, re.M)
+    names = [x for f in fields for x in f if x]
+    assert names == [f for f, _ in tid.Config._fields_]
+    assert ctypes.sizeof(tid.Config) == 64
+
+
+def test_shard_plan_covers_exactly():
+    import paper_conf_icpp_wangzll21_b200 as tid
+    for R, G in [(1_000_000, 8), (10, 3), (7, 8), (100_000, 1)]:
+        spans = [tid.shard_plan(R, G, r) for r in range(G)]
+        assert spans[0][0] == 0 and spans[-1][1] == R
+        assert all(spans[i][1] == spans[i + 1][0] for i in range(G - 1))
+        assert max(e - s for s, e in spans) - min(e - s for s, e in spans) <= 1

@@ -1,0 +1,199 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, element by element.
+
+Bit-exact is the bar for everything (all arithmetic is integer): (d1, i1, d2, i2),
+good-match counts, the full count matrix and the top-k ids/counts.  Inputs come from
+tidgen (shared seeded generator) or are built here; expected values come only from
+oracle/.  Sizes span several tiles and ragged tails (n not a multiple of 128, m not a
+multiple of 256, partial reference groups).
+"""
+import numpy as np
+import pytest
+
+import oracle
+import tidgen
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def tid():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    from paper_conf_icpp_wangzll21_b200 import build
+    build.build()
+    import paper_conf_icpp_wangzll21_b200 as t
+    return t
+
+
+def nn_from_oracle(onn):
+    """oracle int64 nn (INT64_MAX / -1 for a missing neighbour) -> the ABI's int32 convention (-1, -1)."""
+    o = onn.copy()
+    big = np.iinfo(np.int64).max
+    o[..., 0][o[..., 0] == big] = -1
+    o[..., 2][o[..., 2] == big] = -1
+    return o.astype(np.int64)
+
+
+# ------------------------------------------------------------------------------ search (C1)
+def test_c1_search_bitexact(tid):
+    """Config 1: 1 query x 64 references x 256 keypoints, ratio 0.8, top-5."""
+    R, m, n, k = 64, 256, 256, 5
+    refs, _ = tidgen.refs(0, R, m)
+    qs, tg = tidgen.queries(0, 1, n, R_total=R, m=m)
+    with tid.Index(ref_kp=m, query_kp_max=1024) as idx:
+        idx.add_references(refs)
+        counts = idx.search_counts(qs)
+        ids, cnt = idx.search(qs, k)
+    e_ids, e_cnt, e_counts = oracle.search(qs, refs, k)
+    np.testing.assert_array_equal(counts.astype(np.int64), e_counts)
+    np.testing.assert_array_equal(ids, e_ids)
+    np.testing.assert_array_equal(cnt, e_cnt)
+    assert ids[0, 0] == tg[0]
+
+
+@pytest.mark.parametrize("n,R,m,B", [(1000, 37, 256, 3), (130, 9, 200, 5), (1, 6, 2, 2), (383, 150, 256, 2)])
+def test_search_shapes_bitexact(tid, n, R, m, B):
+    """Ragged n (tile tails), m < 256, odd reference counts (partial groups), B > 1."""
+    refs, _ = tidgen.refs(100, R, m)
+    qs, _ = tidgen.queries(7, B, n, R_total=R, m=m, n_planted=min(50, n, m))
+    with tid.Index(ref_kp=m, query_kp_max=1024) as idx:
+        idx.add_references(refs)
+        counts = idx.search_counts(qs)
+        ids, cnt = idx.search(qs, min(5, R))
+    e_ids, e_cnt, e_counts = oracle.search(qs, refs, min(5, R))
+    np.testing.assert_array_equal(counts.astype(np.int64), e_counts)
+    np.testing.assert_array_equal(ids, e_ids)
+    np.testing.assert_array_equal(cnt, e_cnt)
+
+
+def test_search_variable_kp_and_nq(tid):
+    """Per-reference keypoint counts (padding rows hold garbage 0xFF) and per-query n_q."""
+    R, m, n, B = 40, 256, 700, 3
+    refs, kp = tidgen.refs(0, R, m, kp_min=0, pad_byte=255)
+    kp[:3] = [0, 1, 2]  # degenerate references: never / never / can match
+    qs, _ = tidgen.queries(0, B, n, R_total=R, m=m, kp_min=0, n_planted=60)
+    n_q = np.array([700, 513, 129], np.int32)
+    with tid.Index(ref_kp=m, query_kp_max=1024) as idx:
+        idx.add_references(refs, kp)
+        counts = idx.search_counts(qs, n_q=n_q)
+        ids, cnt = idx.search(qs, 7, n_q=n_q)
+    e_ids, e_cnt, e_counts = oracle.search(qs, refs, 7, n_q=n_q, kp=kp)
+    np.testing.assert_array_equal(counts.astype(np.int64), e_counts)
+    np.testing.assert_array_equal(ids, e_ids)
+    np.testing.assert_array_equal(cnt, e_cnt)
+    assert (counts[:, :2] == 0).all()
+
+
+# ------------------------------------------------------------------------------ verify
+@pytest.mark.parametrize("n,m,P", [(300, 600, 6), (1000, 1000, 5), (128, 256, 4), (129, 257, 3), (5, 2, 3)])
+def test_verify_bitexact(tid, n, m, P):
+    """(d1, i1, d2, i2) per query row and counts; m > 256 exercises the cross-chunk merge."""
+    Q, Rr, _ = tidgen.pairs(P, n, m, n_planted=min(200, n, m))
+    with tid.Index(ref_kp=256, query_kp_max=1024) as idx:
+        c, nn = idx.verify(Q, Rr)
+    ec, enn = oracle.verify(Q, Rr)
+    np.testing.assert_array_equal(c.astype(np.int64), ec)
+    np.testing.assert_array_equal(nn.astype(np.int64), nn_from_oracle(enn))
+
+
+def test_verify_masks(tid):
+    Q, Rr, _ = tidgen.pairs(4, 400, 500, n_planted=100)
+    n_q = np.array([400, 1, 255, 129], np.int32)
+    m_r = np.array([500, 2, 1, 256], np.int32)
+    with tid.Index(ref_kp=256, query_kp_max=1024) as idx:
+        c, nn = idx.verify(Q, Rr, n_q=n_q, m_r=m_r)
+    ec, enn = oracle.verify(Q, Rr, n_q=n_q, m_r=m_r)
+    np.testing.assert_array_equal(c.astype(np.int64), ec)
+    for p in range(4):
+        np.testing.assert_array_equal(nn[p, :n_q[p]].astype(np.int64), nn_from_oracle(enn[p, :n_q[p]]))
+        assert (nn[p, n_q[p]:] == -1).all()
+
+
+def test_verify_adversarial(tid, rng):
+    """all-255 vs all-0, duplicates, heavy ties (values in {0,1,2}), exact copies."""
+    P, n, m = 6, 200, 300
+    Q = np.zeros((P, n, 128), np.uint8)
+    Rr = np.zeros((P, m, 128), np.uint8)
+    Q[0] = 255                                   # max distance 8,323,200 everywhere
+    Q[1] = rng.integers(0, 3, (n, 128)); Rr[1] = rng.integers(0, 3, (m, 128))    # ties
+    Rr[2, :] = 7; Q[2] = rng.integers(0, 256, (n, 128))                          # all-identical reference
+    Q[3] = rng.integers(0, 256, (n, 128)); Rr[3, :n] = Q[3]; Rr[3, n:] = Q[3, :m - n]  # duplicates of every row
+    Q[4] = rng.integers(0, 256, (n, 128)); Rr[4] = rng.integers(0, 256, (m, 128)); Rr[4, 5:100] = Q[4, 5:100]
+    Q[5] = 255; Rr[5] = 255
+    with tid.Index(ref_kp=256, query_kp_max=1024) as idx:
+        c, nn = idx.verify(Q, Rr)
+    ec, enn = oracle.verify(Q, Rr)
+    np.testing.assert_array_equal(c.astype(np.int64), ec)
+    np.testing.assert_array_equal(nn.astype(np.int64), nn_from_oracle(enn))
+    assert nn[0, 0, 0] == 8_323_200
+
+
+# ------------------------------------------------------------------------------ decompositions
+def test_host_tier_equals_hbm(tid):
+    """Host-streamed references (hbm_budget forces the level-2 tier) == HBM-resident."""
+    R, m, n, B = 300, 256, 400, 2
+    refs, kp = tidgen.refs(0, R, m, kp_min=100, pad_byte=9)
+    qs, _ = tidgen.queries(0, B, n, R_total=R, m=m, kp_min=100)
+    rb = m * 128
+    with tid.Index(ref_kp=m) as a:
+        a.add_references(refs, kp)
+        ca = a.search_counts(qs)
+        ia, na = a.search(qs, 10)
+    with tid.Index(ref_kp=m, hbm_budget_bytes=100 * rb, host_budget_bytes=1000 * rb) as b:
+        b.set_tuning(host_chunk_refs=64)
+        b.add_references(refs[:150], kp[:150])
+        b.add_references(refs[150:], kp[150:])
+        info = b.info()
+        cb = b.search_counts(qs)
+        ib, nb = b.search(qs, 10)
+    assert info["hbm_references"] == 100 and info["host_references"] == 200
+    np.testing.assert_array_equal(ca, cb)
+    np.testing.assert_array_equal(ia, ib)
+    np.testing.assert_array_equal(na, nb)
+    np.testing.assert_array_equal(ca.astype(np.int64), oracle.search_counts(qs, refs, kp=kp))
+
+
+def test_virtual_shards_merge_equals_single(tid):
+    """G shards run one after another on one GPU, merged by the shard-merge kernel == 1 GPU."""
+    R, m, n, B, k = 96, 256, 300, 3, 6
+    refs, _ = tidgen.refs(0, R, m, K=16)        # K=16 clusters: many equal counts -> id tie-breaks
+    qs, _ = tidgen.queries(0, B, n, R_total=R, m=m, K=16, n_planted=30)
+    with tid.Index(ref_kp=m) as one:
+        one.add_references(refs)
+        gi, gc = one.search(qs, k)
+    for G in (2, 3, 8):
+        li, lc = [], []
+        for r in range(G):
+            s, e = tid.shard_plan(R, G, r)
+            with tid.Index(ref_kp=m, id_base=s) as sh:
+                sh.add_references(refs[s:e])
+                i, c = sh.search(qs, min(k, e - s))
+                if e - s < k:  # pad short lists
+                    i = np.concatenate([i, np.full((B, k - (e - s)), -1)], 1)
+                    c = np.concatenate([c, np.zeros((B, k - (e - s)), np.int32)], 1)
+                li.append(i); lc.append(c)
+        with tid.Index(ref_kp=m) as mg:
+            mi, mc = mg.merge_topk(np.stack(li), np.stack(lc))
+        np.testing.assert_array_equal(mi, gi)
+        np.testing.assert_array_equal(mc, gc)
+
+
+def test_device_tensors_and_stream(tid):
+    """Torch CUDA tensors in, device outputs; same answer as host buffers."""
+    import torch
+    R, m, n, B, k = 50, 256, 500, 4, 5
+    refs, _ = tidgen.refs(0, R, m)
+    qs, _ = tidgen.queries(0, B, n, R_total=R, m=m)
+    with tid.Index(ref_kp=m) as idx:
+        idx.add_references(torch.from_numpy(refs).cuda())
+        dq = torch.from_numpy(qs).cuda()
+        ids = torch.empty((B, k), dtype=torch.int64, device="cuda")
+        cnt = torch.empty((B, k), dtype=torch.int32, device="cuda")
+        idx.search(dq, k, out=(ids, cnt))
+        torch.cuda.synchronize()
+        hi, hc = idx.search(qs, k)
+    np.testing.assert_array_equal(ids.cpu().numpy(), hi)
+    np.testing.assert_array_equal(cnt.cpu().numpy(), hc)
+    e_ids, e_cnt, _ = oracle.search(qs, refs, k)
+    np.testing.assert_array_equal(hi, e_ids)
