@@ -170,11 +170,15 @@ tid_status tid_get_stats(tid_index* idx, tid_stats* out); /* synchronises record
 
 /* Tuning knobs (0 = automatic).  refs_per_job: references resident per CTA job (1..4);
  * grid: persistent CTAs for the match kernel; host_chunk_refs: references per
- * host-tier staging buffer. */
+ * host-tier staging buffer; exact_only: disable the search fast path (16-bit packed
+ * top-2 with exact fallback) and scan every element with exact 32-bit keys.  Results
+ * are identical either way. */
 typedef struct {
   int32_t refs_per_job;
   int32_t grid;
   int64_t host_chunk_refs;
+  int32_t exact_only;
+  int32_t reserved;
 } tid_tuning;
 
 tid_status tid_set_tuning(tid_index* idx, const tid_tuning* t);

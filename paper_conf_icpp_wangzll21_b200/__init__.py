@@ -16,7 +16,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libtid.so")
+LIB_PATH = os.environ.get("TID_LIB") or os.path.join(_HERE, "libtid.so")
 
 TID_OK, TID_EINVAL, TID_ENOMEM, TID_ECUDA, TID_ENCCL, TID_EUNSUPPORTED, TID_ESTATE = 0, -1, -2, -3, -4, -5, -6
 STATUS = {0: "TID_OK", -1: "TID_EINVAL", -2: "TID_ENOMEM", -3: "TID_ECUDA", -4: "TID_ENCCL",
@@ -54,7 +54,8 @@ class Stats(ctypes.Structure):
 
 
 class Tuning(ctypes.Structure):
-    _fields_ = [("refs_per_job", ctypes.c_int32), ("grid", ctypes.c_int32), ("host_chunk_refs", ctypes.c_int64)]
+    _fields_ = [("refs_per_job", ctypes.c_int32), ("grid", ctypes.c_int32), ("host_chunk_refs", ctypes.c_int64),
+                ("exact_only", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 _lib = None
@@ -243,8 +244,8 @@ class Index:
         _check(self._lib.tid_get_stats(self._h, ctypes.byref(s)))
         return {f: getattr(s, f) for f, _ in Stats._fields_}
 
-    def set_tuning(self, refs_per_job: int = 0, grid: int = 0, host_chunk_refs: int = 0):
-        t = Tuning(refs_per_job, grid, host_chunk_refs)
+    def set_tuning(self, refs_per_job: int = 0, grid: int = 0, host_chunk_refs: int = 0, exact_only: bool = False):
+        t = Tuning(refs_per_job, grid, host_chunk_refs, 1 if exact_only else 0, 0)
         _check(self._lib.tid_set_tuning(self._h, ctypes.byref(t)))
 
 

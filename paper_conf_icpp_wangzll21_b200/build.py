@@ -23,15 +23,17 @@ def stale() -> bool:
     return any(os.path.getmtime(d) > t for d in DEPS)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if force or stale():
-        tmp = LIB + ".tmp%d" % os.getpid()
-        cmd = [NVCC, *FLAGS, "-o", tmp, *SOURCES, "-ldl"]
+def build(force: bool = False, verbose: bool = False, out: str | None = None, defines=()) -> str:
+    """Compile libtid.so (or a variant at `out` with extra -D defines, for experiments)."""
+    target = out or LIB
+    if force or out or stale():
+        tmp = target + ".tmp%d" % os.getpid()
+        cmd = [NVCC, *FLAGS, *[f"-D{d}" for d in defines], "-o", tmp, *SOURCES, "-ldl"]
         if verbose:
             print(" ".join(cmd), file=sys.stderr)
         subprocess.check_call(cmd)
-        os.replace(tmp, LIB)
-    return LIB
+        os.replace(tmp, target)
+    return target
 
 
 if __name__ == "__main__":

@@ -168,7 +168,7 @@ inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
 struct Segment {          // one cudaMalloc'd piece of the HBM arena
   uint8_t* desc = nullptr;   // [cap][m][128]
-  int32_t* colkey = nullptr; // [cap][cpr*256]
+  int32_t* colkey = nullptr; // [cap][cpr][512] column constants
   int64_t cap = 0, count = 0, first = 0;  // first = local index of its first reference
 };
 
@@ -281,6 +281,7 @@ tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const ui
   p.ldc = ldc;
   p.col0 = col0;
   p.nn_out = nullptr;
+  p.coarse = idx->tune.exact_only ? 0 : 1;
   p.num2 = idx->cfg.ratio_num * idx->cfg.ratio_num;
   p.den2 = idx->cfg.ratio_den * idx->cfg.ratio_den;
   int grid = idx->tune.grid > 0 ? idx->tune.grid : idx->num_sms;
@@ -328,7 +329,7 @@ tid_status run_counts(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, 
     const int64_t rb = idx->ref_bytes;
     for (int b = 0; b < 2; ++b) {
       TRY(idx->stage_desc[b].ensure(static_cast<size_t>(chunk * rb), "host-tier staging"));
-      TRY(idx->stage_colkey[b].ensure(static_cast<size_t>(chunk) * idx->cpr * kBN * 4, "staging keys"));
+      TRY(idx->stage_colkey[b].ensure(static_cast<size_t>(chunk) * idx->cpr * kColBytes, "staging keys"));
       TRY(idx->stage_kp[b].ensure(static_cast<size_t>(chunk) * 4, "staging kp"));
     }
     // the copy stream must not overwrite staging buffers still read by a previous call
@@ -550,14 +551,14 @@ tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t
       Segment ns;
       ns.first = idx->n_hbm;
       cudaError_t e1 = cudaMalloc(&ns.desc, static_cast<size_t>(cap * rb));
-      cudaError_t e2 = e1 == cudaSuccess ? cudaMalloc(&ns.colkey, static_cast<size_t>(cap) * idx->cpr * kBN * 4) : e1;
+      cudaError_t e2 = e1 == cudaSuccess ? cudaMalloc(&ns.colkey, static_cast<size_t>(cap) * idx->cpr * kColBytes) : e1;
       if (e1 != cudaSuccess || e2 != cudaSuccess) {
         cudaGetLastError();
         if (ns.desc) cudaFree(ns.desc);
         return fail(TID_ENOMEM, "HBM arena allocation of %lld references failed", static_cast<long long>(cap));
       }
       ns.cap = cap;
-      idx->hbm_alloc += cap * rb + cap * idx->cpr * kBN * 4;
+      idx->hbm_alloc += cap * rb + cap * idx->cpr * kColBytes;
       idx->segs.push_back(ns);
       sg = &idx->segs.back();
     }
@@ -569,7 +570,7 @@ tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t
     rp.m = idx->cfg.ref_kp;
     rp.cpr = idx->cpr;
     rp.count = take;
-    rp.colkey = sg->colkey + sg->count * idx->cpr * kBN;
+    rp.colkey = sg->colkey + sg->count * idx->cpr * kColInts;
     if (dev_in) {
       rp.src = src;
     } else {
@@ -711,7 +712,7 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
   const uint8_t* dr = r;
   const size_t rbytes = static_cast<size_t>(P) * m * kDim;
   const bool r_dev = is_device_ptr(r);
-  TRY(idx->ws_colkey.ensure(static_cast<size_t>(P) * cpr * kBN * 4, "pair keys"));
+  TRY(idx->ws_colkey.ensure(static_cast<size_t>(P) * cpr * kColBytes, "pair keys"));
   RefPrepParams rp{};
   rp.m = m;
   rp.cpr = cpr;

@@ -23,12 +23,30 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
   asm volatile(
       "{\n\t.reg .pred P1;\n\t"
       "TID_WAIT:\n\t"
-      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1, 1000000;\n\t"
       "@P1 bra TID_DONE;\n\t"
       "bra TID_WAIT;\n\t"
       "TID_DONE:\n\t}" ::"r"(bar),
       "r"(parity)
       : "memory");
+}
+// Polling wait with exponential nanosleep back-off: used by the control warps (TMA producer,
+// MMA issuers), which share SMSPs with the epilogue and must not steal its issue slots.
+__device__ __forceinline__ void mbar_wait_sleep(uint32_t bar, uint32_t parity) {
+  uint32_t ns = 32;
+  while (true) {
+    uint32_t done;
+    asm volatile(
+        "{\n\t.reg .pred P1;\n\t"
+        "mbarrier.test_wait.parity.shared::cta.b64 P1, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, P1;\n\t}"
+        : "=r"(done)
+        : "r"(bar), "r"(parity)
+        : "memory");
+    if (done) return;
+    __nanosleep(ns);
+    ns = ns < 512 ? ns * 2 : 512;
+  }
 }
 __device__ __forceinline__ void fence_barrier_init() {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -64,23 +82,49 @@ __device__ __forceinline__ uint64_t smem_desc_sw128(uint32_t addr) {
   return d;
 }
 
-// Instruction descriptor: kind::i8, A = u8, B = u8, D = s32, K-major A/B, M = 128, N = 256.
+// Instruction descriptor: kind::i8, A = u8, B = u8, D = s32, K-major A/B, M = 128, N = 128.
 constexpr uint32_t kIdescI8 = (2u << 4)                       // D format S32
                               | (0u << 7) | (0u << 10)        // A, B unsigned 8-bit
                               | (0u << 15) | (0u << 16)       // A, B K-major
-                              | (uint32_t(kBN >> 3) << 17)    // N >> 3
+                              | (uint32_t(kPiece >> 3) << 17) // N >> 3
                               | (uint32_t(kBM >> 4) << 24);   // M >> 4
 
+// Issued by the whole (converged) MMA warp: elect.sync picks one lane, so the descriptors stay in
+// uniform registers and ptxas emits a bare UTCIMMA (no per-lane broadcast loop).
 __device__ __forceinline__ void mma_i8(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t accum) {
   asm volatile(
-      "{\n\t.reg .pred p;\n\t"
+      "{\n\t.reg .pred p, e;\n\t"
       "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
       "l"(adesc), "l"(bdesc), "r"(kIdescI8), "r"(accum)
       : "memory");
 }
+// One accumulator piece: D = A * B over K = 128 bytes as four K = 32 MMAs (advancing both
+// SWIZZLE_128B descriptors by 32 B = 2 units) + commit to `bar`, from a single elected lane.
+__device__ __forceinline__ void mma_piece(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t bar) {
+  asm volatile(
+      "{\n\t.reg .pred e, f, t;\n\t.reg .b64 a1, a2, a3, b1, b2, b3;\n\t"
+      "setp.ne.b32 f, 0, 0;\n\t"
+      "setp.eq.b32 t, 0, 0;\n\t"
+      "add.s64 a1, %1, 2;\n\tadd.s64 a2, %1, 4;\n\tadd.s64 a3, %1, 6;\n\t"
+      "add.s64 b1, %2, 2;\n\tadd.s64 b2, %2, 4;\n\tadd.s64 b3, %2, 6;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, f;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], a1, b1, %3, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], a2, b2, %3, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], a3, b3, %3, t;\n\t"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%4];\n\t}" ::"r"(tmem_d),
+      "l"(adesc), "l"(bdesc), "r"(kIdescI8), "r"(bar)
+      : "memory");
+}
+
 __device__ __forceinline__ void mma_commit(uint32_t bar) {
-  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
+  asm volatile(
+      "{\n\t.reg .pred e;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(bar)
+      : "memory");
 }
 
 #define TID_LD32_OUT(v)                                                                                           \
@@ -110,6 +154,34 @@ __device__ __forceinline__ void reg_fence(uint32_t (&v)[32]) {
   for (int i = 0; i < 32; ++i) asm volatile("" : "+r"(v[i]));
 }
 
+// ------------------------------------------------------------------ optional cycle accounting
+// Built only with -DTID_PROF (experiments): per-warp clock64 buckets, read back with
+// tid_debug_read_prof().  Buckets: epilogue 0 wait-accumulator 1 scan 2 finalise 3 fallback
+// 4 wait-keys; MMA 0 wait-free-accumulator 1 wait-query 2 wait-ref 3 issue; producer 0 wait-ref-slot
+// 1 wait-query-stage; 7 = whole loop.
+#ifdef TID_PROF
+__device__ unsigned long long g_prof[148 * 32 * 8];
+#define PROF_DECL unsigned long long prof_acc[8] = {0, 0, 0, 0, 0, 0, 0, 0}; long long prof_t0 = 0, prof_all = clock64();
+#define PROF_B() prof_t0 = clock64();
+#define PROF_E(k) prof_acc[k] += clock64() - prof_t0;
+#define PROF_FLUSH()                                                                          \
+  do {                                                                                        \
+    prof_acc[7] = clock64() - prof_all;                                                       \
+    if (lane == 0 && blockIdx.x < 148)                                                        \
+      for (int k_ = 0; k_ < 8; ++k_) g_prof[(blockIdx.x * 32 + warp) * 8 + k_] = prof_acc[k_]; \
+  } while (0)
+#else
+#define PROF_DECL
+#define PROF_B()
+#define PROF_E(k)
+#define PROF_FLUSH()
+#endif
+
+constexpr int kProducerWarp = 0;               // warp 0: TMA producer
+constexpr int kFirstMmaWarp = 1;               // warps 1..4: MMA issuers (SMSPs 1, 2, 3, 0)
+constexpr int kFirstEpiWarp = 5;               // warps 5..: epilogue (4 per group)
+static_assert(kNG == 2, "4 MMA warps own the 4 TMEM buffers = 2 groups x 2 column halves");
+
 // ------------------------------------------------------------------ shared memory plan
 struct SmemPlan {
   static constexpr uint32_t kR = 0;                                        // kMaxSlots x 32 KiB
@@ -121,10 +193,10 @@ struct SmemPlan {
   static constexpr uint32_t kRFull = kQEmpty + 8 * kQStages;
   static constexpr uint32_t kREmpty = kRFull + 8 * kMaxSlots;
   static constexpr uint32_t kTFull = kREmpty + 8 * kMaxSlots;
-  static constexpr uint32_t kTEmpty = kTFull + 8 * 2;
-  static constexpr uint32_t kTmemPtr = kTEmpty + 8 * 2;
-  static constexpr uint32_t kCnt = kTmemPtr + 16;                          // [8 warps][kMaxSlots] u32
-  static constexpr uint32_t kEnd = kCnt + 8 * kMaxSlots * 4;
+  static constexpr uint32_t kTEmpty = kTFull + 8 * kTmemBufs;
+  static constexpr uint32_t kTmemPtr = kTEmpty + 8 * kTmemBufs;
+  static constexpr uint32_t kCnt = kTmemPtr + 16;                          // [4*kNG warps][kMaxSlots] u32
+  static constexpr uint32_t kEnd = kCnt + 4 * kNG * kMaxSlots * 4;
   static constexpr uint32_t kAlloc = kEnd + 1024;                          // + alignment slack
 };
 
@@ -150,10 +222,165 @@ __device__ __forceinline__ Job decode_job(const MatchParams& p, int32_t j) {
   return J;
 }
 
+// ------------------------------------------------------------------ epilogue scans
+// A "piece" = one 128-column accumulator buffer (MMA N = 128) of one (query tile, reference
+// chunk half).  Each epilogue thread owns one TMEM lane = one query row.
+
+// Exact top-2 over one piece, accumulated into running states (a1 <= a2, b1 <= b2) of packed keys
+// 256 * (N_R - 2S) + i (unique per column within a 256-column chunk).  ~2.5 ALU ops / element.
+__device__ __forceinline__ void scan_exact(uint32_t taddr, uint32_t ck_addr, int& a1, int& a2, int& b1, int& b2) {
+  uint32_t v[2][32];
+  tmem_ld32(taddr, v[0]);
+  tmem_wait_ld();
+  reg_fence(v[0]);
+#pragma unroll
+  for (int jj = 0; jj < kPiece / 32; ++jj) {
+    // software pipeline: the next 32 columns are in flight while these are scanned
+    if (jj + 1 < kPiece / 32) tmem_ld32(taddr + (jj + 1) * 32, v[(jj + 1) & 1]);
+    const uint32_t* w = v[jj & 1];
+#pragma unroll
+    for (int i = 0; i < 32; i += 4) {
+      const int4 c4 = lds128(ck_addr + (jj * 32 + i) * 4);
+      const int x0 = c4.x - 512 * static_cast<int>(w[i]);
+      const int x1 = c4.y - 512 * static_cast<int>(w[i + 1]);
+      const int x2 = c4.z - 512 * static_cast<int>(w[i + 2]);
+      const int x3 = c4.w - 512 * static_cast<int>(w[i + 3]);
+      int lo = min(x0, x1), hi = max(x0, x1);
+      int tt = max(a1, lo);
+      a2 = min(min(a2, tt), hi);
+      a1 = min(a1, lo);
+      lo = min(x2, x3); hi = max(x2, x3);
+      tt = max(b1, lo);
+      b2 = min(min(b2, tt), hi);
+      b1 = min(b1, lo);
+    }
+    // the state must be final before waiting for the next TMEM load (keeps the scan streaming)
+    asm volatile("" : "+r"(a1), "+r"(a2), "+r"(b1), "+r"(b2));
+    if (jj + 1 < kPiece / 32) { tmem_wait_ld(); reg_fence(v[(jj + 1) & 1]); }
+  }
+}
+
+__device__ __forceinline__ uint32_t prmt_top16x2(uint32_t a, uint32_t b) {  // a[31:16] | b[31:16] << 16
+  uint32_t r;
+  asm("prmt.b32 %0, %1, %2, 0x7632;" : "=r"(r) : "r"(a), "r"(b));
+  return r;
+}
+
+// Coarse top-2 over one piece (search fast path): the exact key 256*(N_R - 2S) + i is formed by
+// the same IMAD (FMA pipe); its top 16 bits floor((N_R - 2S)/256) are packed two columns per
+// register (one PRMT) and the top-2 runs on s16x2 lanes (VIMNMX.S16x2 and 3-input forms):
+// ~1.75 ALU ops per element instead of 2.5.  Accumulates into four sorted packed states; the two
+// smallest coarse keys u1 <= u2 of their union bound N_R - 2S of the true 1st / 2nd neighbour
+// to [256 u, 256 u + 255].
+__device__ __forceinline__ void scan_coarse(uint32_t taddr, uint32_t ck_addr, uint32_t& A1, uint32_t& A2,
+                                            uint32_t& B1, uint32_t& B2) {
+  uint32_t v[2][32];
+  int4 ck[2][8];  // column keys, loaded one 32-column chunk ahead (hides the LDS latency)
+  tmem_ld32(taddr, v[0]);
+#pragma unroll
+  for (int i = 0; i < 8; ++i) ck[0][i] = lds128(ck_addr + i * 16);
+  tmem_wait_ld();
+  reg_fence(v[0]);
+#pragma unroll
+  for (int jj = 0; jj < kPiece / 32; ++jj) {
+    if (jj + 1 < kPiece / 32) {
+      tmem_ld32(taddr + (jj + 1) * 32, v[(jj + 1) & 1]);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) ck[(jj + 1) & 1][i] = lds128(ck_addr + ((jj + 1) * 32 + i * 4) * 4);
+    }
+    const uint32_t* w = v[jj & 1];
+    const int4* c4 = ck[jj & 1];
+#pragma unroll
+    for (int i = 0; i < 32; i += 8) {
+      const int4 c0 = c4[i / 4], c1 = c4[i / 4 + 1];
+      const uint32_t k0 = static_cast<uint32_t>(c0.x - 512 * static_cast<int>(w[i]));
+      const uint32_t k1 = static_cast<uint32_t>(c0.y - 512 * static_cast<int>(w[i + 1]));
+      const uint32_t k2 = static_cast<uint32_t>(c0.z - 512 * static_cast<int>(w[i + 2]));
+      const uint32_t k3 = static_cast<uint32_t>(c0.w - 512 * static_cast<int>(w[i + 3]));
+      const uint32_t k4 = static_cast<uint32_t>(c1.x - 512 * static_cast<int>(w[i + 4]));
+      const uint32_t k5 = static_cast<uint32_t>(c1.y - 512 * static_cast<int>(w[i + 5]));
+      const uint32_t k6 = static_cast<uint32_t>(c1.z - 512 * static_cast<int>(w[i + 6]));
+      const uint32_t k7 = static_cast<uint32_t>(c1.w - 512 * static_cast<int>(w[i + 7]));
+      const uint32_t x = prmt_top16x2(k0, k1), y = prmt_top16x2(k2, k3);
+      const uint32_t z = prmt_top16x2(k4, k5), ww = prmt_top16x2(k6, k7);
+      uint32_t lo = __vmins2(x, y), hi = __vmaxs2(x, y);
+      uint32_t tt = __vmaxs2(A1, lo);
+      A2 = __vmins2(__vmins2(A2, tt), hi);
+      A1 = __vmins2(A1, lo);
+      lo = __vmins2(z, ww); hi = __vmaxs2(z, ww);
+      tt = __vmaxs2(B1, lo);
+      B2 = __vmins2(__vmins2(B2, tt), hi);
+      B1 = __vmins2(B1, lo);
+    }
+    asm volatile("" : "+r"(A1), "+r"(A2), "+r"(B1), "+r"(B2));
+    if (jj + 1 < kPiece / 32) { tmem_wait_ld(); reg_fence(v[(jj + 1) & 1]); }
+  }
+}
+
+// Top-2 (per 16-bit lane) of the union of two sorted packed states: (X1 <= X2) U (Y1 <= Y2).
+__device__ __forceinline__ void merge_top2_s16x2(uint32_t& X1, uint32_t& X2, uint32_t Y1, uint32_t Y2) {
+  const uint32_t m2 = __vmins2(__vmaxs2(X1, Y1), __vmins2(X2, Y2));
+  X1 = __vmins2(X1, Y1);
+  X2 = m2;
+}
+
+// Two smallest coarse keys u1 <= u2 (multiset order statistics) of four packed states.
+__device__ __forceinline__ void finish_coarse(uint32_t A1, uint32_t A2, uint32_t B1, uint32_t B2, int& u1, int& u2) {
+  merge_top2_s16x2(A1, A2, B1, B2);
+  const int l1 = static_cast<int16_t>(A1 & 0xFFFFu), h1 = static_cast<int16_t>(A1 >> 16);
+  const int l2 = static_cast<int16_t>(A2 & 0xFFFFu), h2 = static_cast<int16_t>(A2 >> 16);
+  u1 = min(l1, h1);
+  u2 = min(max(l1, h1), min(l2, h2));
+}
+
+// Exact fallback for one undecided query row (rare): the warp recomputes the 256 dot products of
+// that row against the resident reference chunk straight from shared memory (both tiles are
+// SWIZZLE_128B: 16-byte chunk c of row r sits at chunk c ^ (r & 7)), 8 columns per lane with
+// dp4a, and reduces the exact top-2 packed keys across the warp.
+__device__ __forceinline__ void exact_row_from_smem(uint32_t q_tile, int qrow, uint32_t r_tile, uint32_t ck_addr,
+                                                    int lane, int& k1, int& k2) {
+  uint4 q[8];
+#pragma unroll
+  for (int c = 0; c < 8; ++c) {
+    const int4 t = lds128(q_tile + qrow * 128 + ((c ^ (qrow & 7)) << 4));
+    q[c] = make_uint4(t.x, t.y, t.z, t.w);
+  }
+  int a1 = INT_MAX, a2 = INT_MAX;
+#pragma unroll 2
+  for (int jj = 0; jj < kBN / 32; ++jj) {
+    const int col = jj * 32 + lane;
+    uint32_t dot = 0;
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      const int4 r = lds128(r_tile + col * 128 + ((c ^ (col & 7)) << 4));
+      dot = __dp4a(q[c].x, static_cast<uint32_t>(r.x), dot);
+      dot = __dp4a(q[c].y, static_cast<uint32_t>(r.y), dot);
+      dot = __dp4a(q[c].z, static_cast<uint32_t>(r.z), dot);
+      dot = __dp4a(q[c].w, static_cast<uint32_t>(r.w), dot);
+    }
+    int ck;
+    asm volatile("ld.shared.s32 %0, [%1];" : "=r"(ck) : "r"(ck_addr + col * 4));
+    const int key = ck - 512 * static_cast<int>(dot);
+    a2 = min(a2, max(a1, key));
+    a1 = min(a1, key);
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const int b1 = __shfl_xor_sync(0xffffffffu, a1, o), b2 = __shfl_xor_sync(0xffffffffu, a2, o);
+    const int m2 = min(max(a1, b1), min(a2, b2));
+    a1 = min(a1, b1);
+    a2 = m2;
+  }
+  k1 = a1;
+  k2 = a2;
+}
+
 // ------------------------------------------------------------------ fused match kernel
-// One persistent CTA per SM.  A job = (reference group resident in SMEM) x (range of
-// query tiles streamed through a 4-stage ring).  Unit u = (query tile t, reference s);
-// unit u uses TMEM accumulator buffer u&1 and is drained by epilogue group u&1.
+// One persistent CTA per SM.  A job = (reference group resident in SMEM) x (range of query
+// tiles streamed through a 4-stage ring).  Unit u = (query tile t, reference s) belongs to
+// epilogue group u % kNG; each unit is 2*cpr pieces of 128 accumulator columns.  Group g owns
+// kNB TMEM buffers and double-buffers its pieces, so the MMA of its next piece overlaps the
+// scan of the current one.
 __global__ void __launch_bounds__(kNumThreads, 1)
     match_kernel(const __grid_constant__ CUtensorMap qmap, const __grid_constant__ CUtensorMap rmap,
                  const MatchParams p) {
@@ -171,17 +398,19 @@ __global__ void __launch_bounds__(kNumThreads, 1)
   auto tempty = [&](int i) { return sbase + SmemPlan::kTEmpty + 8 * i; };
   uint32_t* tmem_ptr_smem = reinterpret_cast<uint32_t*>(smem + SmemPlan::kTmemPtr);
   uint32_t* cnt_smem = reinterpret_cast<uint32_t*>(smem + SmemPlan::kCnt);
+  const bool use_coarse = p.coarse && cpr == 1 && p.mode == kModeSearch && p.nn_out == nullptr;
 
   if (threadIdx.x == 0) {
     prefetch_tmap(&qmap);
     prefetch_tmap(&rmap);
-    for (int i = 0; i < kQStages; ++i) { mbar_init(qfull(i), 1); mbar_init(qempty(i), 1); }
-    for (int i = 0; i < kMaxSlots; ++i) { mbar_init(rfull(i), 1); mbar_init(rempty(i), 1 + 8); }
-    for (int i = 0; i < 2; ++i) { mbar_init(tfull(i), 1); mbar_init(tempty(i), 4); }
+    // query stages: freed by the MMA commit and by every epilogue warp (the exact fallback reads them)
+    for (int i = 0; i < kQStages; ++i) { mbar_init(qfull(i), 1); mbar_init(qempty(i), 4 + 4 * kNG); }
+    for (int i = 0; i < kMaxSlots; ++i) { mbar_init(rfull(i), 1); mbar_init(rempty(i), 4 + 4 * kNG); }
+    for (int i = 0; i < kTmemBufs; ++i) { mbar_init(tfull(i), 1); mbar_init(tempty(i), 4); }
     fence_barrier_init();
   }
-  if (threadIdx.x < 8 * kMaxSlots) cnt_smem[threadIdx.x] = 0;
-  if (warp == 1) {  // TMEM: 2 accumulator buffers x 256 columns (all 512)
+  if (threadIdx.x < 4 * kNG * kMaxSlots) cnt_smem[threadIdx.x] = 0;
+  if (warp == kFirstMmaWarp) {  // TMEM: kTmemBufs accumulator buffers x 128 columns (all 512)
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(
                      smem_u32(tmem_ptr_smem))
                  : "memory");
@@ -192,7 +421,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
   tc_fence_after();
   const uint32_t tmem_base = *tmem_ptr_smem;
 
-  if (warp == 0) {
+  PROF_DECL
+  if (warp == kProducerWarp) {
     // ===================== TMA producer =====================
     if (lane == 0) {
       uint32_t qctr = 0;
@@ -201,62 +431,73 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         const Job J = decode_job(p, j);
         const int nslots = J.nr * cpr;
         for (int sl = 0; sl < nslots; ++sl) {
-          mbar_wait(rempty(sl), (slot_use[sl] & 1) ^ 1);
+          PROF_B(); mbar_wait_sleep(rempty(sl), (slot_use[sl] & 1) ^ 1); PROF_E(0);
           mbar_expect_tx(rfull(sl), kRTileBytes + kColBytes);
           const int s = sl / cpr, c = sl % cpr;
           const int64_t ref = J.ref_first + s;
           tma_load_3d(sbase + SmemPlan::kR + sl * kRTileBytes, &rmap, rfull(sl), 0, c * kBN,
                       static_cast<int>(p.ref_map_base + ref));
-          bulk_load(sbase + SmemPlan::kCol + sl * kColBytes, p.colkey + (ref * cpr + c) * kBN, kColBytes, rfull(sl));
+          bulk_load(sbase + SmemPlan::kCol + sl * kColBytes, p.colkey + (ref * cpr + c) * kColInts, kColBytes,
+                    rfull(sl));
           ++slot_use[sl];
         }
         const int ntiles = J.nq * T;
         for (int t = 0; t < ntiles; ++t, ++qctr) {
           const int st = qctr % kQStages;
-          mbar_wait(qempty(st), ((qctr / kQStages) & 1) ^ 1);
+          PROF_B(); mbar_wait_sleep(qempty(st), ((qctr / kQStages) & 1) ^ 1); PROF_E(1);
           mbar_expect_tx(qfull(st), kQTileBytes);
           tma_load_3d(sbase + SmemPlan::kQ + st * kQTileBytes, &qmap, qfull(st), 0, (t % T) * kBM, J.q_first + t / T);
         }
       }
     }
-  } else if (warp == 1) {
-    // ===================== MMA issuer (one thread) =====================
-    if (lane == 0) {
-      uint32_t qctr = 0;
+  } else if (warp >= kFirstMmaWarp && warp < kFirstMmaWarp + 4) {
+    // ===================== MMA issuers: 4 warps, one per SMSP, one per TMEM buffer ==============
+    // Issuing tcgen05.mma costs the issuing SMSP real throughput, and each SMSP's epilogue warps
+    // own one TMEM lane quarter, so the issue load is spread evenly: MMA warp mw owns accumulator
+    // buffer mw = (epilogue group g = mw / 2, column half h = mw % 2) and issues exactly the
+    // pieces (unit u with u % 2 == g, chunk c, half h), in order.  Whole warp, one elected lane.
+    {
+      const int mw = warp - kFirstMmaWarp;
+      const int my_g = mw >> 1, my_h = mw & 1;
+      uint32_t qctr = 0, pc = 0;
       uint32_t slot_use[kMaxSlots] = {0, 0, 0, 0};
-      uint32_t buf_use[2] = {0, 0};
+      const uint32_t dt = tmem_base + mw * kPiece;
       for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
         const Job J = decode_job(p, j);
         const int nslots = J.nr * cpr;
         const int U = J.nq * T * J.nr;
-        bool slot_ready[kMaxSlots] = {false, false, false, false};
-        int waited = 0;
-        for (int u0 = 0; u0 < U; u0 += 2) {
-          for (int c = 0; c < cpr; ++c) {
-            for (int b = 0; b < 2; ++b) {
-              const int u = u0 + b;
-              if (u >= U) break;
-              const int t = u / J.nr, s = u % J.nr, sl = s * cpr + c;
-              while (waited <= t) {
-                const uint32_t g = qctr + waited;
-                mbar_wait(qfull(g % kQStages), (g / kQStages) & 1);
-                ++waited;
-              }
-              if (!slot_ready[sl]) { mbar_wait(rfull(sl), slot_use[sl] & 1); slot_ready[sl] = true; }
-              mbar_wait(tempty(b), (buf_use[b] & 1) ^ 1);
+        uint32_t ready_mask = 0;
+        int waited = 0, t = 0, s = 0, g = 0;
+        for (int u = 0; u < U; ++u) {
+          if (g == my_g) {
+            while (waited <= t) {
+              const uint32_t gq = qctr + waited;
+              PROF_B(); mbar_wait_sleep(qfull(gq % kQStages), (gq / kQStages) & 1); PROF_E(1);
+              ++waited;
+            }
+            const uint32_t st = (qctr + t) % kQStages;
+            const uint64_t ad = smem_desc_sw128(sbase + SmemPlan::kQ + st * kQTileBytes);
+            for (int c = 0; c < cpr; ++c) {
+              const int sl = s * cpr + c;
+              if (!(ready_mask >> sl & 1u)) { PROF_B(); mbar_wait_sleep(rfull(sl), slot_use[sl] & 1); PROF_E(2); ready_mask |= 1u << sl; }
+              const uint64_t bd = smem_desc_sw128(sbase + SmemPlan::kR + sl * kRTileBytes) +
+                                  my_h * (kPiece * kDim >> 4);  // rows 128h.. of the chunk
+              PROF_B(); mbar_wait_sleep(tempty(mw), (pc & 1) ^ 1); PROF_E(0);
               tc_fence_after();
-              const uint32_t st = (qctr + t) % kQStages;
-              const uint64_t ad = smem_desc_sw128(sbase + SmemPlan::kQ + st * kQTileBytes);
-              const uint64_t bd = smem_desc_sw128(sbase + SmemPlan::kR + sl * kRTileBytes);
-              const uint32_t dt = tmem_base + b * kBN;
-#pragma unroll
-              for (int k = 0; k < kDim / 32; ++k)  // K = 32 bytes per tcgen05.mma.kind::i8
-                mma_i8(dt, ad + 2 * k, bd + 2 * k, k > 0 ? 1u : 0u);
-              mma_commit(tfull(b));
-              ++buf_use[b];
-              if (c == cpr - 1 && s == J.nr - 1) mma_commit(qempty(st));  // last reader of tile t
+              mma_piece(dt, ad, bd, tfull(mw));
+              ++pc;
             }
           }
+          if (s == J.nr - 1) {  // this warp's release of query tile t (covers all its prior MMAs)
+            if (waited <= t) {  // never touched tile t: still wait for it so the phase order holds
+              const uint32_t gq = qctr + t;
+              mbar_wait_sleep(qfull(gq % kQStages), (gq / kQStages) & 1);
+              waited = t + 1;
+            }
+            mma_commit(qempty((qctr + t) % kQStages));
+          }
+          if (++g == kNG) g = 0;
+          if (++s == J.nr) { s = 0; ++t; }
         }
         for (int sl = 0; sl < nslots; ++sl) { mma_commit(rempty(sl)); ++slot_use[sl]; }
         qctr += J.nq * T;
@@ -264,11 +505,12 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     }
   } else {
     // ===================== epilogue: TMEM -> registers -> top-2 -> ratio -> count =====================
-    const int e = (warp - 2) >> 2;          // group 0: warps 2..5, group 1: warps 6..9
-    const int quarter = warp & 3;           // TMEM lanes 32*quarter .. +31 (hardware restriction)
-    const int wslot = warp - 2;             // 0..7 for the count accumulators
-    const uint32_t taddr_base = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16) + e * kBN;
-    uint32_t buf_use = 0;
+    const int ew = warp - kFirstEpiWarp;     // 0 .. 4*kNG-1
+    const int g = ew >> 2;                   // epilogue group (units u with u % kNG == g)
+    const int quarter = warp & 3;            // TMEM lanes 32*quarter .. +31 (hardware restriction)
+    const uint32_t taddr_q = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16);
+    uint32_t mp = 0;                         // pieces consumed by this group
+    uint32_t qctr = 0;
     uint32_t slot_use[kMaxSlots] = {0, 0, 0, 0};
     const int row_in_tile = quarter * 32 + lane;
     const int nq_ld = T * kBM;
@@ -277,108 +519,161 @@ __global__ void __launch_bounds__(kNumThreads, 1)
       const Job J = decode_job(p, j);
       const int nslots = J.nr * cpr;
       const int U = J.nq * T * J.nr;
-      const int ustep = (J.nr % 2 == 0) ? J.nr : 2 * J.nr;  // next unit of this group with the same s
-      for (int u = e; u < U; u += 2) {
-        const int t = u / J.nr, s = u % J.nr;
-        const int qi = J.q_first + t / T;
-        const int row = (t % T) * kBM + row_in_tile;
-        const int nvalid = p.n_valid ? p.n_valid[qi] : p.n_rows;
-        const bool valid = row < nvalid && row < p.n_rows;
-        const int32_t nqv = p.nq[static_cast<int64_t>(qi) * nq_ld + row];
-
-        int g1d = INT_MAX, g1i = -1, g2d = INT_MAX, g2i = -1;  // running 2-NN over chunks
-        for (int c = 0; c < cpr; ++c) {
-          const int sl = s * cpr + c;
-          mbar_wait(rfull(sl), slot_use[sl] & 1);  // column keys of this chunk have landed
-          mbar_wait(tfull(e), buf_use & 1);
-          tc_fence_after();
-          const uint32_t ck_addr = sbase + SmemPlan::kCol + sl * kColBytes;
-          int a1 = INT_MAX, a2 = INT_MAX, b1 = INT_MAX, b2 = INT_MAX;
+      int t = 0, s = 0, tq = 0, qi = J.q_first, ug = 0;
+      bool touched = false;
+      for (int u = 0; u < U; ++u) {
+        if (ug == g) {
+          touched = true;
+          const int row = tq * kBM + row_in_tile;
+          const int nvalid = p.n_valid ? p.n_valid[qi] : p.n_rows;
+          const bool valid = row < nvalid && row < p.n_rows;
+          const int32_t nqv = p.nq[static_cast<int64_t>(qi) * nq_ld + row];
+          int g1d = INT_MAX, g1i = -1, g2d = INT_MAX, g2i = -1;  // running exact 2-NN over chunks
+          bool pass = false;
+          if (use_coarse) {
+            const int sl = s;
+            PROF_B(); mbar_wait(rfull(sl), slot_use[sl] & 1); PROF_E(4);  // column keys have landed
+            uint32_t A1 = 0x7FFF7FFFu, A2 = 0x7FFF7FFFu, B1 = 0x7FFF7FFFu, B2 = 0x7FFF7FFFu;
 #pragma unroll
-          for (int jj = 0; jj < kBN / 32; ++jj) {
-            uint32_t v[32];
-            tmem_ld32(taddr_base + jj * 32, v);
-            tmem_wait_ld();
-            reg_fence(v);
-#pragma unroll
-            for (int i = 0; i < 32; i += 4) {
-              const int4 c4 = lds128(ck_addr + (jj * 32 + i) * 4);
-              const int x0 = c4.x - 512 * static_cast<int>(v[i]);
-              const int x1 = c4.y - 512 * static_cast<int>(v[i + 1]);
-              const int x2 = c4.z - 512 * static_cast<int>(v[i + 2]);
-              const int x3 = c4.w - 512 * static_cast<int>(v[i + 3]);
-              int lo = min(x0, x1), hi = max(x0, x1);
-              int tt = max(a1, lo);
-              a2 = min(min(a2, tt), hi);
-              a1 = min(a1, lo);
-              lo = min(x2, x3); hi = max(x2, x3);
-              tt = max(b1, lo);
-              b2 = min(min(b2, tt), hi);
-              b1 = min(b1, lo);
+            for (int h = 0; h < 2; ++h) {
+              const uint32_t buf = g * kNB + mp % kNB;
+              PROF_B(); mbar_wait(tfull(buf), (mp / kNB) & 1); PROF_E(0);
+              tc_fence_after();
+              PROF_B();
+              scan_coarse(taddr_q + buf * kPiece, sbase + SmemPlan::kCol + sl * kColBytes + h * kPiece * 4, A1, A2,
+                          B1, B2);
+              PROF_E(1);
+              tc_fence_before();
+              __syncwarp();
+              if (lane == 0) mbar_arrive(tempty(buf));  // accumulator free as soon as it is scanned
+              ++mp;
             }
-            // keep the scan streaming: the state must be final before the next TMEM load
-            asm volatile("" : "+r"(a1), "+r"(a2), "+r"(b1), "+r"(b2));
+            PROF_B();
+            int u1, u2;
+            finish_coarse(A1, A2, B1, B2, u1, u2);
+            // bounds: N_R - 2S of the 1st / 2nd neighbour lies in [256 u, 256 u + 255]
+            const int64_t d1lo = static_cast<int64_t>(nqv) + 256 * static_cast<int64_t>(u1);
+            const int64_t d2lo = static_cast<int64_t>(nqv) + 256 * static_cast<int64_t>(u2);
+            const int64_t den2 = p.den2, num2 = p.num2;
+            // u == 0x7FFF only for padding columns (sentinel N_R); real keys are <= 32512
+            const bool fail_sure = (u2 >= 0x7FFF) || den2 * d1lo >= num2 * (d2lo + 255);
+            const bool pass_sure = !fail_sure && den2 * (d1lo + 255) < num2 * d2lo;
+            pass = valid && pass_sure;
+            uint32_t undecided = __ballot_sync(0xffffffffu, valid && !pass_sure && !fail_sure);
+            PROF_E(2);
+            if (undecided) {
+              PROF_B();
+              const uint32_t qt = sbase + SmemPlan::kQ + ((qctr + t) % kQStages) * kQTileBytes;
+              const uint32_t rt = sbase + SmemPlan::kR + sl * kRTileBytes;
+              const uint32_t ck = sbase + SmemPlan::kCol + sl * kColBytes;
+              while (undecided) {
+                const int l = __ffs(undecided) - 1;
+                undecided &= undecided - 1;
+                int k1, k2;
+                exact_row_from_smem(qt, quarter * 32 + l, rt, ck, lane, k1, k2);
+                if (lane == l) {
+                  const int64_t d1 = static_cast<int64_t>(nqv) + (k1 >> 8);
+                  const int64_t d2 = static_cast<int64_t>(nqv) + (k2 >> 8);
+                  pass = (k2 >> 8) < kSentinelNorm && den2 * d1 < num2 * d2;
+                }
+              }
+              PROF_E(3);
+            }
+          } else {
+            for (int c = 0; c < cpr; ++c) {
+              const int sl = s * cpr + c;
+              mbar_wait(rfull(sl), slot_use[sl] & 1);
+              int a1 = INT_MAX, a2 = INT_MAX, b1 = INT_MAX, b2 = INT_MAX;
+#pragma unroll
+              for (int h = 0; h < 2; ++h) {
+                const uint32_t buf = g * kNB + mp % kNB;
+                mbar_wait(tfull(buf), (mp / kNB) & 1);
+                tc_fence_after();
+                scan_exact(taddr_q + buf * kPiece, sbase + SmemPlan::kCol + sl * kColBytes + h * kPiece * 4, a1, a2,
+                           b1, b2);
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(tempty(buf));
+                ++mp;
+              }
+              const int k1 = min(a1, b1);
+              const int k2 = min(max(a1, b1), min(a2, b2));
+              const int c1d = k1 >> 8, c1i = (k1 & 255) + c * kBN;
+              const int c2d = k2 >> 8, c2i = (k2 & 255) + c * kBN;
+              // merge into the running 2-NN; earlier chunks win ties (lower index)
+              if (c1d < g1d) {
+                if (c2d < g1d) { g2d = c2d; g2i = c2i; } else { g2d = g1d; g2i = g1i; }
+                g1d = c1d; g1i = c1i;
+              } else if (c1d < g2d) {
+                g2d = c1d; g2i = c1i;
+              }
+            }
+            // ratio test in exact integers: den^2 * d1 < num^2 * d2
+            const bool real1 = g1d < kSentinelNorm, real2 = g2d < kSentinelNorm;
+            const int64_t d1 = static_cast<int64_t>(nqv) + g1d;
+            const int64_t d2 = static_cast<int64_t>(nqv) + g2d;
+            pass = valid && real2 &&
+                   static_cast<uint64_t>(p.den2) * static_cast<uint64_t>(d1) <
+                       static_cast<uint64_t>(p.num2) * static_cast<uint64_t>(d2);
+            if (p.nn_out != nullptr && row < p.n_rows) {
+              int4 o;
+              o.x = (valid && real1) ? static_cast<int>(d1) : -1; o.y = (valid && real1) ? g1i : -1;
+              o.z = (valid && real2) ? static_cast<int>(d2) : -1; o.w = (valid && real2) ? g2i : -1;
+              reinterpret_cast<int4*>(p.nn_out)[static_cast<int64_t>(qi) * p.n_rows + row] = o;
+            }
           }
-          tc_fence_before();
+          const uint32_t bal = __ballot_sync(0xffffffffu, pass);
+          if (lane == 0) {
+            uint32_t& acc = cnt_smem[ew * kMaxSlots + s];
+            acc += __popc(bal);
+            // flush when this group holds no further unit of this (query, reference) pair
+            if (tq == T - 1 || u + J.nr >= U || J.nr % kNG != 0) {
+              if (acc) {
+                const int64_t ci = (p.mode == kModeVerify)
+                                       ? qi : static_cast<int64_t>(qi) * p.ldc + p.col0 + J.ref_first + s;
+                atomicAdd(p.counts + ci, acc);
+              }
+              acc = 0;
+            }
+          }
+        }
+        if (s == J.nr - 1) {  // this warp is done with query tile t (fallback reads it)
+          const uint32_t gq = qctr + t;
+          // a warp with no unit in tile t must not arrive before tile t has landed, or its
+          // arrival would count towards the stage's previous phase
+          if (!touched) mbar_wait(qfull(gq % kQStages), (gq / kQStages) & 1);
+          touched = false;
           __syncwarp();
-          if (lane == 0) mbar_arrive(tempty(e));
-          ++buf_use;
-          // top-2 of the chunk from the two interleaved states (keys are unique: index bits)
-          const int k1 = min(a1, b1);
-          const int k2 = min(max(a1, b1), min(a2, b2));
-          const int c1d = k1 >> 8, c1i = (k1 & 255) + c * kBN;
-          const int c2d = k2 >> 8, c2i = (k2 & 255) + c * kBN;
-          // merge into the running 2-NN; earlier chunks win ties (lower index)
-          if (c1d < g1d) {
-            if (c2d < g1d) { g2d = c2d; g2i = c2i; } else { g2d = g1d; g2i = g1i; }
-            g1d = c1d; g1i = c1i;
-          } else if (c1d < g2d) {
-            g2d = c1d; g2i = c1i;
-          }
+          if (lane == 0) mbar_arrive(qempty(gq % kQStages));
         }
-        // ratio test in exact integers: den^2 * d1 < num^2 * d2
-        const bool real1 = g1d < kSentinelNorm, real2 = g2d < kSentinelNorm;
-        const int64_t d1 = static_cast<int64_t>(nqv) + g1d;
-        const int64_t d2 = static_cast<int64_t>(nqv) + g2d;
-        const bool pass = valid && real2 &&
-                          static_cast<uint64_t>(p.den2) * static_cast<uint64_t>(d1) <
-                              static_cast<uint64_t>(p.num2) * static_cast<uint64_t>(d2);
-        if (p.nn_out != nullptr && row < p.n_rows) {
-          int4 o;
-          o.x = (valid && real1) ? static_cast<int>(d1) : -1; o.y = (valid && real1) ? g1i : -1;
-          o.z = (valid && real2) ? static_cast<int>(d2) : -1; o.w = (valid && real2) ? g2i : -1;
-          reinterpret_cast<int4*>(p.nn_out)[static_cast<int64_t>(qi) * p.n_rows + row] = o;
-        }
-        const uint32_t bal = __ballot_sync(0xffffffffu, pass);
-        if (lane == 0) {
-          uint32_t& acc = cnt_smem[wslot * kMaxSlots + s];
-          acc += __popc(bal);
-          const int un = u + ustep;
-          const bool flush = (un >= U) || ((un / J.nr) / T != t / T);
-          if (flush) {
-            if (acc) {
-              const int64_t ci = (p.mode == kModeVerify) ? qi
-                                                         : static_cast<int64_t>(qi) * p.ldc + p.col0 + J.ref_first + s;
-              atomicAdd(p.counts + ci, acc);
-            }
-            acc = 0;
-          }
+        if (++ug == kNG) ug = 0;
+        if (++s == J.nr) {
+          s = 0; ++t;
+          if (++tq == T) { tq = 0; ++qi; }
         }
       }
       __syncwarp();
       if (lane == 0)
         for (int sl = 0; sl < nslots; ++sl) mbar_arrive(rempty(sl));
       for (int sl = 0; sl < nslots; ++sl) ++slot_use[sl];
+      qctr += J.nq * T;
     }
   }
 
+  PROF_FLUSH();
   tc_fence_before();
   __syncthreads();
-  if (warp == 1) {
+  if (warp == kFirstMmaWarp) {
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem_base) : "memory");
   }
 }
+
+#ifdef TID_PROF
+extern "C" int tid_debug_read_prof(void* host, size_t bytes) {
+  return static_cast<int>(cudaMemcpyFromSymbol(host, g_prof, bytes));
+}
+#endif
 
 cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap, int grid,
                          cudaStream_t s) {
@@ -421,7 +716,9 @@ __global__ void ref_prep_kernel(RefPrepParams p) {
       for (int w = 0; w < kDim / 16; ++w) dst[w] = make_uint4(0, 0, 0, 0);
     }
   }
-  p.colkey[r * cols + i] = norm * 256 + (i & (kBN - 1));
+  const int c = i / kBN, ii = i & (kBN - 1);
+  int32_t* ck = p.colkey + (r * p.cpr + c) * kColInts;
+  ck[ii] = norm * 256 + ii;
 }
 
 void launch_ref_prep(const RefPrepParams& p, cudaStream_t s) {

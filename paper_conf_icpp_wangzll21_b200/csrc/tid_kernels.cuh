@@ -22,15 +22,26 @@ constexpr int kBM = 128;           // query keypoints per MMA tile (TMEM lanes)
 constexpr int kBN = 256;           // reference keypoints per chunk (MMA N, TMEM columns)
 constexpr int kQStages = 4;        // query-tile ring
 constexpr int kMaxSlots = 4;       // resident reference chunks per CTA
-constexpr int kNumThreads = 320;   // w0 TMA, w1 MMA, w2..w9 two epilogue groups of 4 warps
+#ifndef TID_NG
+#define TID_NG 2
+#endif
+constexpr int kNG = TID_NG;                    // epilogue groups (2 or 4), 4 warps each
+constexpr int kPiece = 128;                    // accumulator columns per MMA piece (MMA N)
+constexpr int kTmemBufs = 512 / kPiece;        // 4 TMEM buffers of 128 columns
+constexpr int kNB = kTmemBufs / kNG;           // buffers per epilogue group
+constexpr int kNumThreads = 32 * (5 + 4 * kNG);  // w0 TMA, w1..w4 MMA, w5.. epilogue (4*kNG warps)
 constexpr uint32_t kQTileBytes = kBM * kDim;   // 16 KiB
 constexpr uint32_t kRTileBytes = kBN * kDim;   // 32 KiB
-constexpr uint32_t kColBytes = kBN * 4;        // 1 KiB of packed column keys per chunk
+constexpr int kColInts = kBN;                  // per chunk: 256 packed column keys
+constexpr uint32_t kColBytes = kColInts * 4;   // 1 KiB per chunk
 constexpr int32_t kSentinelNorm = (1 << 23) - 1;  // > 128*255^2: padded columns never win
 
-// packed column key: colkey[i] = N_R[i] * 256 + i  (i = index within the 256-column chunk);
-// the epilogue forms key = colkey - 512 * S = 256 * (N_R - 2 q.r) + i, which orders
-// exactly like (d_ji, i) for a fixed query row (Alg. 1 step 4 + lowest-index tie-break).
+// Packed column key, per 256-column chunk (global layout [ref][chunk][256] int32):
+//   colkey[i] = N_R[i] * 256 + i   (i = index within the chunk).
+// The epilogue forms key = colkey - 512 * S = 256 * (N_R - 2 q.r) + i with one IMAD, which
+// orders exactly like (d_ji, i) for a fixed query row (Alg. 1 step 4 + lowest-index
+// tie-break).  Its top 16 bits (arithmetic) are floor((N_R - 2 q.r) / 256): the coarse key
+// of the search fast path, packed two per register with one PRMT.
 
 enum : int { kModeSearch = 0, kModeVerify = 1 };
 
@@ -54,13 +65,14 @@ struct MatchParams {
   int64_t col0;
   int32_t* nn_out;           // verify: [num_q][n_rows][4] or null
   uint32_t num2, den2;       // ratio^2 = num2/den2
+  int32_t coarse;            // 1: 16-bit packed top-2 with exact fallback (search, cpr == 1)
 };
 
 struct RefPrepParams {
   uint8_t* desc;             // [count][m][128] destination (null = read-only, keys only)
   const uint8_t* src;        // optional source to copy from (null = in place)
   const int32_t* kp;         // [count] or null (= m)
-  int32_t* colkey;           // [count][cpr*256]
+  int32_t* colkey;           // [count][cpr][256]
   int64_t count;
   int32_t m;
   int32_t cpr;

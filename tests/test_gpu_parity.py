@@ -197,3 +197,44 @@ def test_device_tensors_and_stream(tid):
     np.testing.assert_array_equal(cnt.cpu().numpy(), hc)
     e_ids, e_cnt, _ = oracle.search(qs, refs, k)
     np.testing.assert_array_equal(hi, e_ids)
+
+
+@pytest.mark.parametrize("hi", [3, 24, 256])
+def test_search_fast_path_fallback(tid, rng, hi):
+    """Search fast path (16-bit packed keys + exact fallback): low-range data makes most rows
+    undecidable (exact re-scan), full-range data almost none; both must equal the oracle and
+    the exact-only path bit for bit."""
+    R, m, n, B = 24, 256, 300, 2
+    refs = rng.integers(0, hi, (R, m, 128), dtype=np.uint8)
+    qs = rng.integers(0, hi, (B, n, 128), dtype=np.uint8)
+    qs[0, :100] = refs[5, :100]                      # exact copies -> d1 = 0 rows
+    qs[1, :50] = np.minimum(refs[7, :50].astype(int) + 1, 255)
+    with tid.Index(ref_kp=m) as idx:
+        idx.add_references(refs)
+        fast = idx.search_counts(qs)
+        idx.set_tuning(exact_only=True)
+        exact = idx.search_counts(qs)
+    np.testing.assert_array_equal(fast, exact)
+    np.testing.assert_array_equal(fast.astype(np.int64), oracle.search_counts(qs, refs))
+
+
+def test_search_boundary_ratios(tid):
+    """Rows whose ratio sits exactly on / next to the 0.8 boundary at large distances (the
+    coarse bounds straddle, forcing the exact fallback): q = 0, two reference keypoints with
+    ||r||^2 = 16 s^2 and 25 s^2 (+/- 1)."""
+    m, n = 256, 8
+    R = np.zeros((1, m, 128), np.uint8)
+    # d1 = 16*s^2 via sixteen entries of s; d2 = 25*s^2 via twenty-five entries of s (+ tweak)
+    s = 40
+    R[0, 0, :16] = s
+    R[0, 1, :25] = s
+    R[0, 2:, :] = 250                                 # far keypoints
+    R2 = R.copy(); R2[0, 1, 25] = 1                    # d2 = 25 s^2 + 1 -> pass
+    R3 = R.copy(); R3[0, 0, 16] = 1                    # d1 = 16 s^2 + 1 -> fail
+    refs = np.concatenate([R, R2, R3], 0)
+    qs = np.zeros((1, n, 128), np.uint8)
+    with tid.Index(ref_kp=m) as idx:
+        idx.add_references(refs)
+        got = idx.search_counts(qs)
+    np.testing.assert_array_equal(got.astype(np.int64), oracle.search_counts(qs, refs))
+    assert got[0].tolist() == [0, n, 0]
