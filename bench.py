@@ -114,19 +114,21 @@ def peaks():
 
 # ----------------------------------------------------------------------------- oracle arm
 def time_oracle(qs, refs, seconds: float):
-    """Time the CPU oracle (as it stands) on a bounded sample: 1 query x S references, S sized
-    to ~`seconds` of work on all host cores.  Returns (comparisons/s, sample description, cores)."""
+    """Time the CPU oracle (as it stands, OpenMP over all host cores) on a bounded sample:
+    1 query x S references, S grown until one timed call takes >= `seconds`.
+    Returns (comparisons/s, sample description, cores, seconds)."""
     import oracle
     cores = len(os.sched_getaffinity(0))
     q = qs[:1]
-    probe = max(cores, 16)
-    t0 = time.perf_counter()
-    oracle.search_counts(q, refs[:probe])
-    dt = time.perf_counter() - t0
-    S = int(min(len(refs), max(probe, probe * seconds / max(dt, 1e-6))))
-    t0 = time.perf_counter()
-    oracle.search_counts(q, refs[:S])
-    dt = time.perf_counter() - t0
+    S = 4 * cores
+    oracle.search_counts(q, refs[:cores])  # warm the OpenMP pool
+    while True:
+        t0 = time.perf_counter()
+        oracle.search_counts(q, refs[:S])
+        dt = time.perf_counter() - t0
+        if dt >= seconds or S >= len(refs):
+            break
+        S = int(min(len(refs), S * max(2.0, 1.2 * seconds / max(dt, 1e-3))))
     return S / dt, f"1 query (n={q.shape[1]}) x {S} references (m={refs.shape[1]}), {dt:.1f} s", cores, dt
 
 

@@ -249,8 +249,4 @@ class Index:
         _check(self._lib.tid_set_tuning(self._h, ctypes.byref(t)))
 
 
-def shard_plan(R_total: int, world_size: int, rank: int) -> tuple[int, int]:
-    """References shard by image id into contiguous ranges: [start, end)."""
-    base, rem = divmod(R_total, world_size)
-    start = rank * base + min(rank, rem)
-    return start, start + base + (1 if rank < rem else 0)
+from .dist import shard_plan  # noqa: E402  (re-export)

@@ -68,12 +68,3 @@ def test_config_struct_matches_header():
     names = [x for f in fields for x in f if x]
     assert names == [f for f, _ in tid.Config._fields_]
     assert ctypes.sizeof(tid.Config) == 64
-
-
-def test_shard_plan_covers_exactly():
-    import paper_conf_icpp_wangzll21_b200 as tid
-    for R, G in [(1_000_000, 8), (10, 3), (7, 8), (100_000, 1)]:
-        spans = [tid.shard_plan(R, G, r) for r in range(G)]
-        assert spans[0][0] == 0 and spans[-1][1] == R
-        assert all(spans[i][1] == spans[i + 1][0] for i in range(G - 1))
-        assert max(e - s for s, e in spans) - min(e - s for s, e in spans) <= 1
