@@ -139,15 +139,12 @@ def run_reference(args, cfg_name):
         return
     import oracle
     import tidgen
-    per_step_refs = 2048
+    per_step_refs = 4096
     refs, _ = tidgen.refs(0, per_step_refs, m, seed=SEED)
     qs, _ = tidgen.queries(0, 1, n, R_total=Rg * args.gpus, m=m, seed=SEED)
-    cores = len(os.sched_getaffinity(0))
-    # size one step to ~8 s on this host so W + K steps finish in a few minutes
-    t0 = time.perf_counter()
-    oracle.search_counts(qs, refs[:cores * 2])
-    rate = cores * 2 / (time.perf_counter() - t0)
-    S = int(max(cores, min(per_step_refs, rate * 8.0)))
+    # size one step to ~6 s on this host so W + K steps finish in a few minutes
+    rate, _, cores, _ = time_oracle(qs, refs, 2.0)
+    S = int(max(cores, min(per_step_refs, rate * 6.0)))
     times = []
     for i in range(args.warmup + args.steps):
         t0 = time.perf_counter()
