@@ -64,7 +64,9 @@ typedef struct {
   int64_t  id_base;            /* global id of this rank's first reference (shard offset)         */
   int32_t  rank;               /* this process's rank; 0 when world_size == 1                     */
   int32_t  world_size;         /* number of shards (GPUs); 1 = single GPU                         */
-  const void* nccl_unique_id;  /* 128-byte ncclUniqueId (same on all ranks) when world_size > 1   */
+  const void* nccl_unique_id;  /* 128-byte ncclUniqueId (same on all ranks); required when
+                                  world_size > 1.  Given with world_size == 1, a one-rank NCCL
+                                  communicator runs the same all-gather + merge path (tests).   */
 } tid_config;
 
 /* Create an index on cfg->device.  Allocates the HBM arena lazily (on first add).

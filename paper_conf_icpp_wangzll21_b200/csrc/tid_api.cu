@@ -468,7 +468,7 @@ tid_status tid_index_create(const tid_config* cfg, tid_index** out) {
     tid_index_destroy(idx);
     return fail(TID_ECUDA, "stream/event creation: %s", cudaGetErrorString(e));
   }
-  if (cfg->world_size > 1) {
+  if (cfg->world_size > 1 || cfg->nccl_unique_id) {  // a 1-rank communicator exercises the same path
     ncclUniqueId id;
     memcpy(&id, cfg->nccl_unique_id, sizeof(id));
     if (!nccl().ok) {
@@ -651,7 +651,7 @@ tid_status tid_search(tid_index* idx, const uint8_t* queries, const int32_t* n_q
   if (!ref_ids_out || !match_counts_out) return fail(TID_EINVAL, "null outputs");
   if (k < 1 || k > 64) return fail(TID_EINVAL, "k=%d outside 1..64", k);
   const int64_t R = idx->n_hbm + idx->n_host;
-  if (idx->cfg.world_size == 1 && k > R)
+  if (idx->comm == nullptr && k > R)
     return fail(TID_EINVAL, "k=%d exceeds the number of references (%lld)", k, static_cast<long long>(R));
   TRY(set_device(idx));
   cudaStream_t s = static_cast<cudaStream_t>(stream);
@@ -672,7 +672,7 @@ tid_status tid_search(tid_index* idx, const uint8_t* queries, const int32_t* n_q
   const bool dev_ids = is_device_ptr(ref_ids_out), dev_cnt = is_device_ptr(match_counts_out);
   int64_t* ids = dev_ids ? ref_ids_out : idx->ws_ids.as<int64_t>();
   int32_t* cnts = dev_cnt ? match_counts_out : idx->ws_cnts.as<int32_t>();
-  if (idx->cfg.world_size == 1) {
+  if (idx->comm == nullptr) {
     launch_merge(idx->ws_cand.as<uint64_t>(), static_cast<int32_t>(segs), B, k, segs * k, k, nullptr, ids, cnts, s);
     count_kernel(idx);
   } else {

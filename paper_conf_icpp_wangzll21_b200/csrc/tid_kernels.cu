@@ -141,6 +141,19 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
       : TID_LD32_OUT(v)
       : "r"(taddr));
 }
+
+// 128 consecutive TMEM columns of this thread's lane in one load (32x32b shape, .x128).
+__device__ __forceinline__ void tmem_ld128(uint32_t taddr, uint32_t (&v)[128]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x128.b32 {"
+      "%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,"
+      "%30,%31,%32,%33,%34,%35,%36,%37,%38,%39,%40,%41,%42,%43,%44,%45,%46,%47,%48,%49,%50,%51,%52,%53,%54,%55,%56,%57,"
+      "%58,%59,%60,%61,%62,%63,%64,%65,%66,%67,%68,%69,%70,%71,%72,%73,%74,%75,%76,%77,%78,%79,%80,%81,%82,%83,%84,%85,"
+      "%86,%87,%88,%89,%90,%91,%92,%93,%94,%95,%96,%97,%98,%99,%100,%101,%102,%103,%104,%105,%106,%107,%108,%109,%110,"
+      "%111,%112,%113,%114,%115,%116,%117,%118,%119,%120,%121,%122,%123,%124,%125,%126,%127}, [%128];"
+      : TID_LD32_OUT(v), TID_LD32_OUT((v + 32)), TID_LD32_OUT((v + 64)), TID_LD32_OUT((v + 96))
+      : "r"(taddr));
+}
 __device__ __forceinline__ int4 lds128(uint32_t addr) {
   int4 r;
   asm volatile("ld.shared.v4.s32 {%0, %1, %2, %3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "r"(addr));
@@ -177,10 +190,13 @@ __device__ unsigned long long g_prof[148 * 32 * 8];
 #define PROF_FLUSH()
 #endif
 
+#ifndef TID_X128
+#define TID_X128 0
+#endif
 constexpr int kProducerWarp = 0;               // warp 0: TMA producer
 constexpr int kFirstMmaWarp = 1;               // warps 1..4: MMA issuers (SMSPs 1, 2, 3, 0)
 constexpr int kFirstEpiWarp = 5;               // warps 5..: epilogue (4 per group)
-static_assert(kNG == 2, "4 MMA warps own the 4 TMEM buffers = 2 groups x 2 column halves");
+static_assert(kNG == 2 || kNG == 4, "4 MMA warps own the 4 TMEM buffers (2 groups x 2 halves, or 4 groups)");
 
 // ------------------------------------------------------------------ shared memory plan
 struct SmemPlan {
@@ -314,6 +330,39 @@ __device__ __forceinline__ void scan_coarse(uint32_t taddr, uint32_t ck_addr, ui
     }
     asm volatile("" : "+r"(A1), "+r"(A2), "+r"(B1), "+r"(B2));
     if (jj + 1 < kPiece / 32) { tmem_wait_ld(); reg_fence(v[(jj + 1) & 1]); }
+  }
+}
+
+// Same scan, one .x128 TMEM load per piece and a single wait (latency exposed once per piece).
+__device__ __forceinline__ void scan_coarse_x128(uint32_t taddr, uint32_t ck_addr, uint32_t& A1, uint32_t& A2,
+                                                 uint32_t& B1, uint32_t& B2) {
+  uint32_t v[128];
+  tmem_ld128(taddr, v);
+  tmem_wait_ld();
+#pragma unroll
+  for (int i = 0; i < 128; ++i) asm volatile("" : "+r"(v[i]));
+#pragma unroll
+  for (int i = 0; i < 128; i += 8) {
+    const int4 c0 = lds128(ck_addr + i * 4), c1 = lds128(ck_addr + (i + 4) * 4);
+    const uint32_t k0 = static_cast<uint32_t>(c0.x - 512 * static_cast<int>(v[i]));
+    const uint32_t k1 = static_cast<uint32_t>(c0.y - 512 * static_cast<int>(v[i + 1]));
+    const uint32_t k2 = static_cast<uint32_t>(c0.z - 512 * static_cast<int>(v[i + 2]));
+    const uint32_t k3 = static_cast<uint32_t>(c0.w - 512 * static_cast<int>(v[i + 3]));
+    const uint32_t k4 = static_cast<uint32_t>(c1.x - 512 * static_cast<int>(v[i + 4]));
+    const uint32_t k5 = static_cast<uint32_t>(c1.y - 512 * static_cast<int>(v[i + 5]));
+    const uint32_t k6 = static_cast<uint32_t>(c1.z - 512 * static_cast<int>(v[i + 6]));
+    const uint32_t k7 = static_cast<uint32_t>(c1.w - 512 * static_cast<int>(v[i + 7]));
+    const uint32_t x = prmt_top16x2(k0, k1), y = prmt_top16x2(k2, k3);
+    const uint32_t z = prmt_top16x2(k4, k5), ww = prmt_top16x2(k6, k7);
+    uint32_t lo = __vmins2(x, y), hi = __vmaxs2(x, y);
+    uint32_t tt = __vmaxs2(A1, lo);
+    A2 = __vmins2(__vmins2(A2, tt), hi);
+    A1 = __vmins2(A1, lo);
+    lo = __vmins2(z, ww); hi = __vmaxs2(z, ww);
+    tt = __vmaxs2(B1, lo);
+    B2 = __vmins2(__vmins2(B2, tt), hi);
+    B1 = __vmins2(B1, lo);
+    if ((i & 31) == 24) asm volatile("" : "+r"(A1), "+r"(A2), "+r"(B1), "+r"(B2));
   }
 }
 
@@ -458,7 +507,9 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     // pieces (unit u with u % 2 == g, chunk c, half h), in order.  Whole warp, one elected lane.
     {
       const int mw = warp - kFirstMmaWarp;
-      const int my_g = mw >> 1, my_h = mw & 1;
+      // kNG == 2: buffer mw = (group mw/2, half mw%2); kNG == 4: buffer mw = group mw, both halves
+      const int my_g = kNG == 2 ? (mw >> 1) : mw;
+      const int h_lo = kNG == 2 ? (mw & 1) : 0, h_hi = kNG == 2 ? (mw & 1) : 1;
       uint32_t qctr = 0, pc = 0;
       uint32_t slot_use[kMaxSlots] = {0, 0, 0, 0};
       const uint32_t dt = tmem_base + mw * kPiece;
@@ -480,12 +531,14 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             for (int c = 0; c < cpr; ++c) {
               const int sl = s * cpr + c;
               if (!(ready_mask >> sl & 1u)) { PROF_B(); mbar_wait_sleep(rfull(sl), slot_use[sl] & 1); PROF_E(2); ready_mask |= 1u << sl; }
-              const uint64_t bd = smem_desc_sw128(sbase + SmemPlan::kR + sl * kRTileBytes) +
-                                  my_h * (kPiece * kDim >> 4);  // rows 128h.. of the chunk
-              PROF_B(); mbar_wait_sleep(tempty(mw), (pc & 1) ^ 1); PROF_E(0);
-              tc_fence_after();
-              mma_piece(dt, ad, bd, tfull(mw));
-              ++pc;
+              for (int h = h_lo; h <= h_hi; ++h) {
+                const uint64_t bd = smem_desc_sw128(sbase + SmemPlan::kR + sl * kRTileBytes) +
+                                    h * (kPiece * kDim >> 4);  // rows 128h.. of the chunk
+                PROF_B(); mbar_wait_sleep(tempty(mw), (pc & 1) ^ 1); PROF_E(0);
+                tc_fence_after();
+                mma_piece(dt, ad, bd, tfull(mw));
+                ++pc;
+              }
             }
           }
           if (s == J.nr - 1) {  // this warp's release of query tile t (covers all its prior MMAs)
@@ -524,10 +577,12 @@ __global__ void __launch_bounds__(kNumThreads, 1)
       for (int u = 0; u < U; ++u) {
         if (ug == g) {
           touched = true;
+          PROF_B();
           const int row = tq * kBM + row_in_tile;
           const int nvalid = p.n_valid ? p.n_valid[qi] : p.n_rows;
           const bool valid = row < nvalid && row < p.n_rows;
           const int32_t nqv = p.nq[static_cast<int64_t>(qi) * nq_ld + row];
+          PROF_E(6);
           int g1d = INT_MAX, g1i = -1, g2d = INT_MAX, g2i = -1;  // running exact 2-NN over chunks
           bool pass = false;
           if (use_coarse) {
@@ -540,12 +595,19 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               PROF_B(); mbar_wait(tfull(buf), (mp / kNB) & 1); PROF_E(0);
               tc_fence_after();
               PROF_B();
+#if TID_X128
+              scan_coarse_x128(taddr_q + buf * kPiece, sbase + SmemPlan::kCol + sl * kColBytes + h * kPiece * 4, A1,
+                               A2, B1, B2);
+#else
               scan_coarse(taddr_q + buf * kPiece, sbase + SmemPlan::kCol + sl * kColBytes + h * kPiece * 4, A1, A2,
                           B1, B2);
+#endif
               PROF_E(1);
+              PROF_B();
               tc_fence_before();
               __syncwarp();
               if (lane == 0) mbar_arrive(tempty(buf));  // accumulator free as soon as it is scanned
+              PROF_E(5);
               ++mp;
             }
             PROF_B();

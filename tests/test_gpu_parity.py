@@ -238,3 +238,26 @@ def test_search_boundary_ratios(tid):
         got = idx.search_counts(qs)
     np.testing.assert_array_equal(got.astype(np.int64), oracle.search_counts(qs, refs))
     assert got[0].tolist() == [0, n, 0]
+
+
+def test_nccl_collective_path_single_rank(tid):
+    """The multi-GPU path (local top-k -> ncclAllGather -> merge kernel) on a one-rank NCCL
+    communicator must return exactly the single-GPU result."""
+    import torch  # loads PyTorch's NCCL first; libtid resolves the already-loaded library
+    R, m, n, B, k = 80, 256, 300, 4, 7
+    refs, _ = tidgen.refs(0, R, m, K=16)
+    qs, _ = tidgen.queries(0, B, n, R_total=R, m=m, K=16, n_planted=40)
+    with tid.Index(ref_kp=m) as one:
+        one.add_references(refs)
+        gi, gc = one.search(qs, k)
+    with tid.Index(ref_kp=m, rank=0, world_size=1, nccl_id=tid.nccl_unique_id()) as col:
+        col.add_references(refs)
+        ci, cc = col.search(qs, k)
+        dq = torch.from_numpy(qs).cuda()
+        di, dc = col.search(dq, k, out=(torch.empty((B, k), dtype=torch.int64, device="cuda"),
+                                       torch.empty((B, k), dtype=torch.int32, device="cuda")))
+        torch.cuda.synchronize()
+    np.testing.assert_array_equal(ci, gi)
+    np.testing.assert_array_equal(cc, gc)
+    np.testing.assert_array_equal(di.cpu().numpy(), gi)
+    np.testing.assert_array_equal(dc.cpu().numpy(), gc)

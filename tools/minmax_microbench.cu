@@ -43,6 +43,16 @@ __global__ void __launch_bounds__(256) k(const uint32_t* __restrict__ in, uint32
                       a[i] = (uint32_t)(wv >> 32) ^ b[i]; b[i] = (uint32_t)wv; }
       if (OP == 15) { long long wv; asm volatile("mad.wide.s32 %0, %1, %2, %3;" : "=l"(wv) : "r"(a[i]), "r"(-33554432), "l"(((long long)c) << 16));
                       a[i] = (uint32_t)(wv >> 32); b[i] = b[i] * 65536u + a[i]; }                     // IMAD.WIDE + IMAD(pack)
+      if (OP == 16) { float f; asm volatile("cvt.rn.f32.s32 %0, %1;" : "=f"(f) : "r"(a[i])); a[i] = __float_as_uint(f) ^ b[i];
+                      asm volatile("cvt.rn.f32.s32 %0, %1;" : "=f"(f) : "r"(b[i])); b[i] = __float_as_uint(f) + c; }   // I2FP
+      if (OP == 17) { uint32_t h; asm volatile("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(h) : "f"(__uint_as_float(a[i])), "f"(__uint_as_float(b[i]))); a[i] = h;
+                      asm volatile("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(h) : "f"(__uint_as_float(b[i])), "f"(__uint_as_float(c))); b[i] = h; } // F2FP pack
+      if (OP == 18) { float x = __uint_as_float(a[i]), y = __uint_as_float(b[i]);
+                      asm volatile("fma.rn.f32 %0, %1, %2, %3;" : "=f"(x) : "f"(x), "f"(-2.0f), "f"(y));
+                      asm volatile("fma.rn.f32 %0, %1, %2, %3;" : "=f"(y) : "f"(y), "f"(-2.0f), "f"(__uint_as_float(c)));
+                      a[i] = __float_as_uint(x); b[i] = __float_as_uint(y); }                              // FFMA
+      if (OP == 19) { uint32_t h; asm volatile("fma.rn.f16x2 %0, %1, %2, %3;" : "=r"(h) : "r"(a[i]), "r"(b[i]), "r"(c)); a[i] = h;
+                      asm volatile("fma.rn.f16x2 %0, %1, %2, %3;" : "=r"(h) : "r"(b[i]), "r"(c), "r"(a[i])); b[i] = h; } // HFMA2
       if (OP == 13) { asm volatile("min.f16x2 %0, %1, %2;" : "=r"(a[i]) : "r"(a[i]), "r"(b[i]));
                       b[i] = b[i] - 512u * c; }                                                       // HMNMX2 + IMAD
     }
@@ -96,6 +106,10 @@ int main() {
     run<13>("HMNMX2 + IMAD", in, out, blocks, thr, clk);
     run<14>("IMAD.WIDE.U32 (+LOP)", in, out, blocks, thr, clk);
     run<15>("IMAD.WIDE + IMAD", in, out, blocks, thr, clk);
+    run<16>("I2FP (+LOP/IADD)", in, out, blocks, thr, clk);
+    run<17>("F2FP.PACK_AB", in, out, blocks, thr, clk);
+    run<18>("FFMA", in, out, blocks, thr, clk);
+    run<19>("HFMA2", in, out, blocks, thr, clk);
     cudaFree(in);
     cudaFree(out);
   }

@@ -30,4 +30,5 @@ for w in range(0, 32):
         continue
     tot = buf[:, w, 7].mean()
     parts = " ".join(f"{k}:{100 * buf[:, w, k].mean() / tot:5.1f}%" for k in range(7) if buf[:, w, k].sum() > 0)
+    parts += f" other:{100 * (1 - buf[:, w, :7].sum(1).mean() / tot):5.1f}%"
     print(f"warp {w:2d} ({names.get(w, 'epilogue')}): total {tot / 1e6:8.2f} Mcyc  {parts}")
