@@ -261,3 +261,20 @@ def test_nccl_collective_path_single_rank(tid):
     np.testing.assert_array_equal(cc, gc)
     np.testing.assert_array_equal(di.cpu().numpy(), gi)
     np.testing.assert_array_equal(dc.cpu().numpy(), gc)
+
+
+@pytest.mark.parametrize("m,n,kp_min", [(384, 768, 384), (384, 768, 100), (1024, 300, 500)])
+def test_search_m_above_256(tid, m, n, kp_min):
+    """The paper's operating point m = 384, n = 768 (Table 7) and m up to 1024:
+    references span several 256-column chunks, merged per query row in index order."""
+    R, B, k = 23, 2, 5
+    refs, kp = tidgen.refs(0, R, m, kp_min=kp_min, pad_byte=77)
+    qs, _ = tidgen.queries(0, B, n, R_total=R, m=m, kp_min=kp_min, n_planted=150)
+    with tid.Index(ref_kp=m, query_kp_max=1024) as idx:
+        idx.add_references(refs, kp)
+        counts = idx.search_counts(qs)
+        ids, cnt = idx.search(qs, k)
+    e_ids, e_cnt, e_counts = oracle.search(qs, refs, k, kp=kp)
+    np.testing.assert_array_equal(counts.astype(np.int64), e_counts)
+    np.testing.assert_array_equal(ids, e_ids)
+    np.testing.assert_array_equal(cnt, e_cnt)

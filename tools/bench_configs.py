@@ -1,0 +1,121 @@
+#!/usr/bin/env python
+"""Secondary measurements (one B200): C1 latency, C2 verification, C3 throughput, the batch
+sweep (B200 analogue of the paper's Fig. 4) and host-tier streaming (C5 analogue,
+§6).  Prints one JSON object per measurement; DESIGN.md §8 quotes them.
+
+    python tools/bench_configs.py [c1] [c2] [c3] [sweep] [host]
+"""
+from __future__ import annotations
+
+import json
+import os
+import statistics
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import tidgen  # noqa: E402
+import paper_conf_icpp_wangzll21_b200 as tid  # noqa: E402
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def timed(fn, reps, warm=3):
+    import torch
+    for _ in range(warm):
+        fn()
+    torch.cuda.synchronize()
+    ts = []
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        fn()
+        e1.record()
+        e1.synchronize()
+        ts.append(e0.elapsed_time(e1))
+    return ts
+
+
+def search_case(name, B, n, R, m, k, reps, hbm_budget=0, host_budget=0, chunk=0):
+    import torch
+    t0 = time.perf_counter()
+    idx = tid.Index(ref_kp=m, query_kp_max=max(n, 1), hbm_budget_bytes=hbm_budget, host_budget_bytes=host_budget)
+    if chunk:
+        idx.set_tuning(host_chunk_refs=chunk)
+    step = 100_000
+    for s in range(0, R, step):
+        refs, _ = tidgen.refs(s, min(step, R - s), m)
+        idx.add_references(refs)
+    qs, tg = tidgen.queries(0, B, n, R_total=R, m=m)
+    log(f"{name}: setup {time.perf_counter() - t0:.1f}s info {idx.info()}")
+    dq = torch.from_numpy(qs).cuda()
+    ids = torch.empty((B, k), dtype=torch.int64, device="cuda")
+    cnt = torch.empty((B, k), dtype=torch.int32, device="cuda")
+    for _ in range(3):
+        idx.search(dq, k, out=(ids, cnt))
+    idx.profile(True)
+    ts = timed(lambda: idx.search(dq, k, out=(ids, cnt)), reps, warm=0)
+    st = idx.stats()
+    hq = torch.from_numpy(qs).pin_memory()
+    ts_e2e = []
+    for _ in range(min(reps, 5)):
+        t = time.perf_counter()
+        idx.search(hq, k)
+        ts_e2e.append(1e3 * (time.perf_counter() - t))
+    top1 = float(np.mean(ids[:, 0].cpu().numpy() == tg))
+    p50 = statistics.median(ts)
+    out = {"case": name, "queries": B, "query_kp": n, "refs": R, "ref_kp": m, "top_k": k,
+           "p50_ms": p50, "p99_ms": float(np.percentile(ts, 99)), "comparisons_per_s": B * R / (p50 / 1e3),
+           "e2e_p50_ms": statistics.median(ts_e2e), "e2e_comparisons_per_s": B * R / (statistics.median(ts_e2e) / 1e3),
+           "match_kernel_ms_per_search": st["match_ms"] / reps if st["match_launches"] else None,
+           "h2d_GBps": (st["h2d_bytes"] / (sum(ts) / 1e3) / 1e9) if st["h2d_bytes"] else 0.0,
+           "planted_top1": top1, "info": idx.info()}
+    idx.close()
+    print(json.dumps(out), flush=True)
+    return out
+
+
+def verify_case(P=4096, n=1000, m=1000, reps=10):
+    import torch
+    Q, Rr, pos = tidgen.pairs(P, n, m)
+    idx = tid.Index(ref_kp=256, query_kp_max=max(n, 1))
+    dq, dr = torch.from_numpy(Q).cuda(), torch.from_numpy(Rr).cuda()
+    cnt = torch.empty(P, dtype=torch.int32, device="cuda")
+    nn = torch.empty((P, n, 4), dtype=torch.int32, device="cuda")
+    ts = timed(lambda: idx.verify(dq, dr, out=(cnt, None)), reps)
+    ts_nn = timed(lambda: idx.verify(dq, dr, out=(cnt, nn)), reps)
+    c = cnt.cpu().numpy()
+    out = {"case": "C2 verify", "pairs": P, "query_kp": n, "ref_kp": m, "p50_ms": statistics.median(ts),
+           "comparisons_per_s": P / (statistics.median(ts) / 1e3), "p50_ms_with_nn": statistics.median(ts_nn),
+           "positives_mean_count": float(c[pos].mean()), "negatives_mean_count": float(c[~pos].mean())}
+    idx.close()
+    print(json.dumps(out), flush=True)
+
+
+def main():
+    what = sys.argv[1:] or ["c1", "c3", "c2", "sweep"]
+    if "c1" in what:
+        search_case("C1", 1, 256, 64, 256, 5, reps=100)
+    if "c3" in what:
+        search_case("C3", 64, 1000, 100_000, 256, 5, reps=5)
+    if "c2" in what:
+        verify_case()
+    if "sweep" in what:
+        for B in (1, 8, 64, 256):
+            search_case(f"sweep B={B}", B, 1000, 100_000, 256, 5, reps=5 if B >= 64 else 20)
+    if "host" in what:
+        R = int(os.environ.get("HOST_REFS", "1000000"))
+        rb = 256 * 128
+        for B in (8, 64):
+            search_case(f"host-tier B={B}", B, 1000, R, 256, 5, reps=3, hbm_budget=rb, host_budget=(R + 1) * rb,
+                        chunk=32768)
+
+
+if __name__ == "__main__":
+    main()
