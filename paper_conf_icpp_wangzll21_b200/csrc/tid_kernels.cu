@@ -48,6 +48,9 @@ __device__ __forceinline__ void mbar_wait_sleep(uint32_t bar, uint32_t parity) {
     ns = ns < 512 ? ns * 2 : 512;
   }
 }
+__device__ __forceinline__ void named_bar(uint32_t id, uint32_t count) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
+}
 __device__ __forceinline__ void fence_barrier_init() {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 }
@@ -211,8 +214,9 @@ struct SmemPlan {
   static constexpr uint32_t kTFull = kREmpty + 8 * kMaxSlots;
   static constexpr uint32_t kTEmpty = kTFull + 8 * kTmemBufs;
   static constexpr uint32_t kTmemPtr = kTEmpty + 8 * kTmemBufs;
-  static constexpr uint32_t kCnt = kTmemPtr + 16;                          // [4*kNG warps][kMaxSlots] u32
-  static constexpr uint32_t kEnd = kCnt + 4 * kNG * kMaxSlots * 4;
+  static constexpr uint32_t kCnt = kTmemPtr + 16;                          // [4*kNG finalisers][kMaxSlots] u32
+  static constexpr uint32_t kXch = (kCnt + 4 * kNG * kMaxSlots * 4 + 15) & ~15u;  // split-warp state exchange
+  static constexpr uint32_t kEnd = kXch + 4 * kNG * 2 * 32 * (kSplit - 1) * 16 + 16;
   static constexpr uint32_t kAlloc = kEnd + 1024;                          // + alignment slack
 };
 
@@ -244,15 +248,16 @@ __device__ __forceinline__ Job decode_job(const MatchParams& p, int32_t j) {
 
 // Exact top-2 over one piece, accumulated into running states (a1 <= a2, b1 <= b2) of packed keys
 // 256 * (N_R - 2S) + i (unique per column within a 256-column chunk).  ~2.5 ALU ops / element.
+template <int NCOL>
 __device__ __forceinline__ void scan_exact(uint32_t taddr, uint32_t ck_addr, int& a1, int& a2, int& b1, int& b2) {
   uint32_t v[2][32];
   tmem_ld32(taddr, v[0]);
   tmem_wait_ld();
   reg_fence(v[0]);
 #pragma unroll
-  for (int jj = 0; jj < kPiece / 32; ++jj) {
+  for (int jj = 0; jj < NCOL / 32; ++jj) {
     // software pipeline: the next 32 columns are in flight while these are scanned
-    if (jj + 1 < kPiece / 32) tmem_ld32(taddr + (jj + 1) * 32, v[(jj + 1) & 1]);
+    if (jj + 1 < NCOL / 32) tmem_ld32(taddr + (jj + 1) * 32, v[(jj + 1) & 1]);
     const uint32_t* w = v[jj & 1];
 #pragma unroll
     for (int i = 0; i < 32; i += 4) {
@@ -272,7 +277,7 @@ __device__ __forceinline__ void scan_exact(uint32_t taddr, uint32_t ck_addr, int
     }
     // the state must be final before waiting for the next TMEM load (keeps the scan streaming)
     asm volatile("" : "+r"(a1), "+r"(a2), "+r"(b1), "+r"(b2));
-    if (jj + 1 < kPiece / 32) { tmem_wait_ld(); reg_fence(v[(jj + 1) & 1]); }
+    if (jj + 1 < NCOL / 32) { tmem_wait_ld(); reg_fence(v[(jj + 1) & 1]); }
   }
 }
 
@@ -288,6 +293,7 @@ __device__ __forceinline__ uint32_t prmt_top16x2(uint32_t a, uint32_t b) {  // a
 // ~1.75 ALU ops per element instead of 2.5.  Accumulates into four sorted packed states; the two
 // smallest coarse keys u1 <= u2 of their union bound N_R - 2S of the true 1st / 2nd neighbour
 // to [256 u, 256 u + 255].
+template <int NCOL>
 __device__ __forceinline__ void scan_coarse(uint32_t taddr, uint32_t ck_addr, uint32_t& A1, uint32_t& A2,
                                             uint32_t& B1, uint32_t& B2) {
   uint32_t v[2][32];
@@ -298,8 +304,8 @@ __device__ __forceinline__ void scan_coarse(uint32_t taddr, uint32_t ck_addr, ui
   tmem_wait_ld();
   reg_fence(v[0]);
 #pragma unroll
-  for (int jj = 0; jj < kPiece / 32; ++jj) {
-    if (jj + 1 < kPiece / 32) {
+  for (int jj = 0; jj < NCOL / 32; ++jj) {
+    if (jj + 1 < NCOL / 32) {
       tmem_ld32(taddr + (jj + 1) * 32, v[(jj + 1) & 1]);
 #pragma unroll
       for (int i = 0; i < 8; ++i) ck[(jj + 1) & 1][i] = lds128(ck_addr + ((jj + 1) * 32 + i * 4) * 4);
@@ -329,7 +335,7 @@ __device__ __forceinline__ void scan_coarse(uint32_t taddr, uint32_t ck_addr, ui
       B1 = __vmins2(B1, lo);
     }
     asm volatile("" : "+r"(A1), "+r"(A2), "+r"(B1), "+r"(B2));
-    if (jj + 1 < kPiece / 32) { tmem_wait_ld(); reg_fence(v[(jj + 1) & 1]); }
+    if (jj + 1 < NCOL / 32) { tmem_wait_ld(); reg_fence(v[(jj + 1) & 1]); }
   }
 }
 
@@ -447,15 +453,16 @@ __global__ void __launch_bounds__(kNumThreads, 1)
   auto tempty = [&](int i) { return sbase + SmemPlan::kTEmpty + 8 * i; };
   uint32_t* tmem_ptr_smem = reinterpret_cast<uint32_t*>(smem + SmemPlan::kTmemPtr);
   uint32_t* cnt_smem = reinterpret_cast<uint32_t*>(smem + SmemPlan::kCnt);
+  uint32_t* xch_smem = reinterpret_cast<uint32_t*>(smem + SmemPlan::kXch);
   const bool use_coarse = p.coarse && cpr == 1 && p.mode == kModeSearch && p.nn_out == nullptr;
 
   if (threadIdx.x == 0) {
     prefetch_tmap(&qmap);
     prefetch_tmap(&rmap);
     // query stages: freed by the MMA commit and by every epilogue warp (the exact fallback reads them)
-    for (int i = 0; i < kQStages; ++i) { mbar_init(qfull(i), 1); mbar_init(qempty(i), 4 + 4 * kNG); }
-    for (int i = 0; i < kMaxSlots; ++i) { mbar_init(rfull(i), 1); mbar_init(rempty(i), 4 + 4 * kNG); }
-    for (int i = 0; i < kTmemBufs; ++i) { mbar_init(tfull(i), 1); mbar_init(tempty(i), 4); }
+    for (int i = 0; i < kQStages; ++i) { mbar_init(qfull(i), 1); mbar_init(qempty(i), 4 + kEpiWarps); }
+    for (int i = 0; i < kMaxSlots; ++i) { mbar_init(rfull(i), 1); mbar_init(rempty(i), 4 + kEpiWarps); }
+    for (int i = 0; i < kTmemBufs; ++i) { mbar_init(tfull(i), 1); mbar_init(tempty(i), 4 * kSplit); }
     fence_barrier_init();
   }
   if (threadIdx.x < 4 * kNG * kMaxSlots) cnt_smem[threadIdx.x] = 0;
@@ -558,10 +565,14 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     }
   } else {
     // ===================== epilogue: TMEM -> registers -> top-2 -> ratio -> count =====================
-    const int ew = warp - kFirstEpiWarp;     // 0 .. 4*kNG-1
-    const int g = ew >> 2;                   // epilogue group (units u with u % kNG == g)
+    const int ew = warp - kFirstEpiWarp;     // 0 .. 4*kNG*kSplit-1
+    const int g = ew / (4 * kSplit);         // epilogue group (units u with u % kNG == g)
+    const int cq = (ew >> 2) % kSplit;       // column part of every piece this warp scans
     const int quarter = warp & 3;            // TMEM lanes 32*quarter .. +31 (hardware restriction)
-    const uint32_t taddr_q = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16);
+    const int fin = g * 4 + quarter;         // finaliser slot (the cq == 0 warp of this lane quarter)
+    const uint32_t pair_bar = 1 + fin;       // named barrier of the kSplit warps of (group, quarter)
+    uint32_t xc = 0;                         // exchanges done (parity selects the exchange slot)
+    const uint32_t taddr_q = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16) + cq * kCPW;
     uint32_t mp = 0;                         // pieces consumed by this group
     uint32_t qctr = 0;
     uint32_t slot_use[kMaxSlots] = {0, 0, 0, 0};
@@ -585,10 +596,10 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           PROF_E(6);
           int g1d = INT_MAX, g1i = -1, g2d = INT_MAX, g2i = -1;  // running exact 2-NN over chunks
           bool pass = false;
+          uint32_t A1 = 0x7FFF7FFFu, A2 = 0x7FFF7FFFu, B1 = 0x7FFF7FFFu, B2 = 0x7FFF7FFFu;
           if (use_coarse) {
             const int sl = s;
             PROF_B(); mbar_wait(rfull(sl), slot_use[sl] & 1); PROF_E(4);  // column keys have landed
-            uint32_t A1 = 0x7FFF7FFFu, A2 = 0x7FFF7FFFu, B1 = 0x7FFF7FFFu, B2 = 0x7FFF7FFFu;
 #pragma unroll
             for (int h = 0; h < 2; ++h) {
               const uint32_t buf = g * kNB + mp % kNB;
@@ -599,8 +610,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               scan_coarse_x128(taddr_q + buf * kPiece, sbase + SmemPlan::kCol + sl * kColBytes + h * kPiece * 4, A1,
                                A2, B1, B2);
 #else
-              scan_coarse(taddr_q + buf * kPiece, sbase + SmemPlan::kCol + sl * kColBytes + h * kPiece * 4, A1, A2,
-                          B1, B2);
+              scan_coarse<kCPW>(taddr_q + buf * kPiece,
+                                sbase + SmemPlan::kCol + sl * kColBytes + (h * kPiece + cq * kCPW) * 4, A1, A2, B1, B2);
 #endif
               PROF_E(1);
               PROF_B();
@@ -610,6 +621,23 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               PROF_E(5);
               ++mp;
             }
+            if (kSplit > 1) {  // the kSplit warps of this lane quarter merge their states
+              uint4* x = reinterpret_cast<uint4*>(xch_smem) + (fin * 2 + (xc & 1)) * 32 * (kSplit - 1);
+              if (cq > 0) x[(cq - 1) * 32 + lane] = make_uint4(A1, A2, B1, B2);
+              named_bar(pair_bar, 32 * kSplit);
+              if (cq == 0) {
+#pragma unroll
+                for (int o = 0; o < kSplit - 1; ++o) {
+                  const uint4 r = x[o * 32 + lane];
+                  merge_top2_s16x2(A1, A2, r.x, r.y);
+                  merge_top2_s16x2(B1, B2, r.z, r.w);
+                }
+              }
+              ++xc;
+            }
+          }
+          if (use_coarse && cq == 0) {
+            const int sl = s;
             PROF_B();
             int u1, u2;
             finish_coarse(A1, A2, B1, B2, u1, u2);
@@ -641,7 +669,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               }
               PROF_E(3);
             }
-          } else {
+          } else if (!use_coarse) {
             for (int c = 0; c < cpr; ++c) {
               const int sl = s * cpr + c;
               mbar_wait(rfull(sl), slot_use[sl] & 1);
@@ -651,15 +679,31 @@ __global__ void __launch_bounds__(kNumThreads, 1)
                 const uint32_t buf = g * kNB + mp % kNB;
                 mbar_wait(tfull(buf), (mp / kNB) & 1);
                 tc_fence_after();
-                scan_exact(taddr_q + buf * kPiece, sbase + SmemPlan::kCol + sl * kColBytes + h * kPiece * 4, a1, a2,
-                           b1, b2);
+                scan_exact<kCPW>(taddr_q + buf * kPiece,
+                                 sbase + SmemPlan::kCol + sl * kColBytes + (h * kPiece + cq * kCPW) * 4, a1, a2, b1, b2);
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(tempty(buf));
                 ++mp;
               }
-              const int k1 = min(a1, b1);
-              const int k2 = min(max(a1, b1), min(a2, b2));
+              int k1 = min(a1, b1);
+              int k2 = min(max(a1, b1), min(a2, b2));
+              if (kSplit > 1) {
+                uint4* x = reinterpret_cast<uint4*>(xch_smem) + (fin * 2 + (xc & 1)) * 32 * (kSplit - 1);
+                if (cq > 0) x[(cq - 1) * 32 + lane] = make_uint4(static_cast<uint32_t>(k1), static_cast<uint32_t>(k2), 0, 0);
+                named_bar(pair_bar, 32 * kSplit);
+                if (cq == 0) {
+#pragma unroll
+                  for (int o = 0; o < kSplit - 1; ++o) {
+                    const uint4 r = x[o * 32 + lane];
+                    const int p1 = static_cast<int>(r.x), p2 = static_cast<int>(r.y);
+                    const int m2 = min(max(k1, p1), min(k2, p2));
+                    k1 = min(k1, p1);
+                    k2 = m2;
+                  }
+                }
+                ++xc;
+              }
               const int c1d = k1 >> 8, c1i = (k1 & 255) + c * kBN;
               const int c2d = k2 >> 8, c2i = (k2 & 255) + c * kBN;
               // merge into the running 2-NN; earlier chunks win ties (lower index)
@@ -677,7 +721,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             pass = valid && real2 &&
                    static_cast<uint64_t>(p.den2) * static_cast<uint64_t>(d1) <
                        static_cast<uint64_t>(p.num2) * static_cast<uint64_t>(d2);
-            if (p.nn_out != nullptr && row < p.n_rows) {
+            if (cq == 0 && p.nn_out != nullptr && row < p.n_rows) {
               int4 o;
               o.x = (valid && real1) ? static_cast<int>(d1) : -1; o.y = (valid && real1) ? g1i : -1;
               o.z = (valid && real2) ? static_cast<int>(d2) : -1; o.w = (valid && real2) ? g2i : -1;
@@ -685,8 +729,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             }
           }
           const uint32_t bal = __ballot_sync(0xffffffffu, pass);
-          if (lane == 0) {
-            uint32_t& acc = cnt_smem[ew * kMaxSlots + s];
+          if (lane == 0 && cq == 0) {
+            uint32_t& acc = cnt_smem[fin * kMaxSlots + s];
             acc += __popc(bal);
             // flush when this group holds no further unit of this (query, reference) pair
             if (tq == T - 1 || u + J.nr >= U || J.nr % kNG != 0) {

@@ -29,7 +29,13 @@ constexpr int kNG = TID_NG;                    // epilogue groups (2 or 4), 4 wa
 constexpr int kPiece = 128;                    // accumulator columns per MMA piece (MMA N)
 constexpr int kTmemBufs = 512 / kPiece;        // 4 TMEM buffers of 128 columns
 constexpr int kNB = kTmemBufs / kNG;           // buffers per epilogue group
-constexpr int kNumThreads = 32 * (5 + 4 * kNG);  // w0 TMA, w1..w4 MMA, w5.. epilogue (4*kNG warps)
+#ifndef TID_SPLIT
+#define TID_SPLIT 1
+#endif
+constexpr int kSplit = TID_SPLIT;              // epilogue warps per (group, TMEM lane quarter)
+constexpr int kCPW = kPiece / kSplit;          // accumulator columns of each piece scanned per warp
+constexpr int kEpiWarps = 4 * kNG * kSplit;
+constexpr int kNumThreads = 32 * (5 + kEpiWarps);  // w0 TMA, w1..w4 MMA, w5.. epilogue
 constexpr uint32_t kQTileBytes = kBM * kDim;   // 16 KiB
 constexpr uint32_t kRTileBytes = kBN * kDim;   // 32 KiB
 constexpr int kColInts = kBN;                  // per chunk: 256 packed column keys
