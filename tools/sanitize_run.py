@@ -1,0 +1,27 @@
+"""Small search / verify / host-tier invocations for compute-sanitizer (memcheck, racecheck,
+synccheck).  Checks results against the oracle too, so a silent corruption also fails."""
+import os
+import sys
+
+import numpy as np
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import oracle  # noqa: E402
+import tidgen  # noqa: E402
+import paper_conf_icpp_wangzll21_b200 as tid  # noqa: E402
+
+refs, kp = tidgen.refs(0, 13, 256, kp_min=50, pad_byte=3)
+qs, _ = tidgen.queries(0, 3, 300, R_total=13, m=256, kp_min=50, n_planted=40)
+with tid.Index(ref_kp=256, query_kp_max=1024, hbm_budget_bytes=8 * 256 * 128, host_budget_bytes=64 * 256 * 128) as idx:
+    idx.set_tuning(host_chunk_refs=3)
+    idx.add_references(refs, kp)
+    c = idx.search_counts(qs)
+    ids, cn = idx.search(qs, 4)
+e_ids, e_cn, e_c = oracle.search(qs, refs, 4, kp=kp)
+assert np.array_equal(c.astype(np.int64), e_c) and np.array_equal(ids, e_ids)
+Q, R, _ = tidgen.pairs(3, 200, 300)
+with tid.Index(ref_kp=256) as idx:
+    vc, nn = idx.verify(Q, R)
+ec, _ = oracle.verify(Q, R)
+assert np.array_equal(vc.astype(np.int64), ec)
+print("sanitize run ok")
