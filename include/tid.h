@@ -67,6 +67,10 @@ typedef struct {
   const void* nccl_unique_id;  /* 128-byte ncclUniqueId (same on all ranks); required when
                                   world_size > 1.  Given with world_size == 1, a one-rank NCCL
                                   communicator runs the same all-gather + merge path (tests).   */
+  int32_t  cache_policy;       /* 0 = fill: HBM first, then the host tier (ids in insertion order);
+                                  1 = FIFO (§6.1): every new batch enters HBM and the
+                                  oldest batches are swapped out to the host tier when HBM is full */
+  int32_t  reserved;
 } tid_config;
 
 /* Create an index on cfg->device.  Allocates the HBM arena lazily (on first add).
@@ -93,10 +97,27 @@ tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t
                               int64_t count, int64_t* first_local_id);
 
 /*
+ * Index lifecycle (the service's delete / update calls; persistence).
+ *   tid_delete_references: the given local ids score 0 and are never ranked again.
+ *   tid_update_references: replace the descriptors (u8 [count][ref_kp][128], host or device)
+ *                          and keypoint counts (nullable = ref_kp) of existing local ids in
+ *                          place (un-deletes them).
+ *   tid_index_save / tid_index_load: binary file of every reference (descriptors with padding
+ *                          rows zeroed, keypoint counts, deleted flags) in local-id order; load
+ *                          appends to an index with the same ref_kp (its own budgets / policy).
+ */
+tid_status tid_delete_references(tid_index* idx, const int64_t* local_ids, int64_t count);
+tid_status tid_update_references(tid_index* idx, const int64_t* local_ids, const uint8_t* desc,
+                                 const int32_t* kp_counts, int64_t count);
+tid_status tid_index_save(const tid_index* idx, const char* path);
+tid_status tid_index_load(tid_index* idx, const char* path, int64_t* first_local_id);
+
+/*
  * One-to-many search, batched over B queries.
  *   queries          : u8 [B][n][128], host or device; n <= query_kp_max.
  *   n_q              : int32 [B] valid keypoints per query (<= n), host or device; NULL = all n.
- *   k                : 1..64 and k <= total references over all ranks.
+ *   k                : 1..64 and k <= total references over all ranks (deleted references are
+ *                      never ranked: if fewer than k live references exist, the tail is id -1).
  *   ref_ids_out      : int64 [B][k]  global reference ids, rank order (count desc, id asc).
  *   match_counts_out : int32 [B][k]  their good-match counts.
  * With world_size > 1 the call is collective: every rank passes the same queries

@@ -25,7 +25,8 @@ STATUS = {0: "TID_OK", -1: "TID_EINVAL", -2: "TID_ENOMEM", -3: "TID_ECUDA", -4: 
 # every symbol declared in include/tid.h
 EXPORTS = ("tid_index_create", "tid_index_destroy", "tid_add_references", "tid_search", "tid_search_counts",
            "tid_verify", "tid_merge_topk", "tid_nccl_unique_id", "tid_get_info", "tid_profile", "tid_get_stats",
-           "tid_set_tuning", "tid_last_error")
+           "tid_set_tuning", "tid_delete_references", "tid_update_references", "tid_index_save", "tid_index_load",
+           "tid_last_error")
 
 
 class TidError(RuntimeError):
@@ -39,7 +40,7 @@ class Config(ctypes.Structure):
                 ("query_kp_max", ctypes.c_int32), ("ratio_num", ctypes.c_uint32), ("ratio_den", ctypes.c_uint32),
                 ("hbm_budget_bytes", ctypes.c_uint64), ("host_budget_bytes", ctypes.c_uint64),
                 ("id_base", ctypes.c_int64), ("rank", ctypes.c_int32), ("world_size", ctypes.c_int32),
-                ("nccl_unique_id", ctypes.c_void_p)]
+                ("nccl_unique_id", ctypes.c_void_p), ("cache_policy", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 class Info(ctypes.Structure):
@@ -84,6 +85,10 @@ def load_library(path: str = LIB_PATH):
     lib.tid_profile.argtypes = [vp, i32]
     lib.tid_get_stats.argtypes = [vp, P(Stats)]
     lib.tid_set_tuning.argtypes = [vp, P(Tuning)]
+    lib.tid_delete_references.argtypes = [vp, vp, i64]
+    lib.tid_update_references.argtypes = [vp, vp, vp, vp, i64]
+    lib.tid_index_save.argtypes = [vp, ctypes.c_char_p]
+    lib.tid_index_load.argtypes = [vp, ctypes.c_char_p, P(i64)]
     lib.tid_last_error.restype = ctypes.c_char_p
     for name in EXPORTS[:-1]:
         getattr(lib, name).restype = ctypes.c_int
@@ -136,12 +141,13 @@ class Index:
 
     def __init__(self, ref_kp: int = 256, query_kp_max: int = 1024, ratio=(4, 5), device: int = 0,
                  hbm_budget_bytes: int = 0, host_budget_bytes: int = 0, id_base: int = 0, rank: int = 0,
-                 world_size: int = 1, nccl_id: bytes | None = None):
+                 world_size: int = 1, nccl_id: bytes | None = None, cache_policy: str = "fill"):
         self._lib = load_library()
         self._id_buf = ctypes.create_string_buffer(nccl_id, 128) if nccl_id is not None else None
         cfg = Config(device, 128, ref_kp, query_kp_max, ratio[0], ratio[1], hbm_budget_bytes, host_budget_bytes,
                      id_base, rank, world_size,
-                     ctypes.cast(self._id_buf, ctypes.c_void_p) if self._id_buf is not None else None)
+                     ctypes.cast(self._id_buf, ctypes.c_void_p) if self._id_buf is not None else None,
+                     {"fill": 0, "fifo": 1}[cache_policy], 0)
         h = ctypes.c_void_p()
         _check(self._lib.tid_index_create(ctypes.byref(cfg), ctypes.byref(h)))
         self._h = h
@@ -173,6 +179,24 @@ class Index:
         kp, k2 = _ptr(kp_counts, np.int32)
         first = ctypes.c_int64()
         _check(self._lib.tid_add_references(self._h, dp, kp, count, ctypes.byref(first)))
+        return first.value
+
+    def delete(self, local_ids):
+        ids, k1 = _ptr(np.asarray(local_ids, np.int64), np.int64)
+        _check(self._lib.tid_delete_references(self._h, ids, len(k1)))
+
+    def update(self, local_ids, desc, kp_counts=None):
+        ids, k1 = _ptr(np.asarray(local_ids, np.int64), np.int64)
+        dp, k2 = _ptr(desc, np.uint8)
+        kp, k3 = _ptr(kp_counts, np.int32)
+        _check(self._lib.tid_update_references(self._h, ids, dp, kp, len(k1)))
+
+    def save(self, path: str):
+        _check(self._lib.tid_index_save(self._h, os.fsencode(path)))
+
+    def load(self, path: str) -> int:
+        first = ctypes.c_int64()
+        _check(self._lib.tid_index_load(self._h, os.fsencode(path), ctypes.byref(first)))
         return first.value
 
     def search(self, queries, k: int, n_q=None, out=None):

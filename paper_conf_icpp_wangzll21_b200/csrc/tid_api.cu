@@ -166,15 +166,15 @@ bool is_device_ptr(const void* p) {
 
 inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
-struct Segment {          // one cudaMalloc'd piece of the HBM arena
-  uint8_t* desc = nullptr;   // [cap][m][128]
-  int32_t* colkey = nullptr; // [cap][cpr][512] column constants
-  int64_t cap = 0, count = 0, first = 0;  // first = local index of its first reference
-};
-
-struct HostSegment {      // one cudaHostAlloc'd piece of the pinned host tier
-  uint8_t* desc = nullptr;   // [cap][m][128] raw (as added)
+// A contiguous range of local ids [first, first + count) stored together, either in the HBM
+// arena (level-1 cache: descriptors + precomputed column keys) or in the pinned host tier
+// (level 2: raw descriptors, streamed and keyed on the GPU per search).  §6.1 P:784-795.
+struct Segment {
+  bool on_host = false;
+  uint8_t* desc = nullptr;    // [cap][m][128]: device (HBM) or pinned host
+  int32_t* colkey = nullptr;  // device, HBM segments only: [cap][cpr][256] packed column keys
   int64_t cap = 0, count = 0, first = 0;
+  std::vector<int32_t> kp;    // keypoint count per reference (0 = deleted / empty)
 };
 
 }  // namespace
@@ -186,10 +186,11 @@ struct tid_index {
   int cpr = 1;                    // chunks per reference = ceil(ref_kp / 256)
   int64_t ref_bytes = 0;          // bytes per stored reference
   uint64_t hbm_budget = 0, host_budget = 0;
-  std::vector<Segment> segs;
-  std::vector<HostSegment> hsegs;
-  std::vector<int32_t> host_kp;   // keypoint counts of host-tier references
-  int64_t n_hbm = 0, n_host = 0;
+  std::vector<Segment> segs;      // id order; HBM and host segments may interleave (FIFO policy)
+  int64_t n_hbm = 0, n_host = 0;  // references held in each tier
+  std::vector<uint8_t> dead;      // per local id: deleted (excluded from ranking)
+  DevBuf dead_dev;                // device copy of `dead` (valid when any_dead)
+  bool any_dead = false, dead_dirty = false;
   int64_t hbm_alloc = 0, host_alloc = 0;
   cudaStream_t copy_stream = nullptr;
   cudaEvent_t ev_h2d[2] = {nullptr, nullptr}, ev_free[2] = {nullptr, nullptr};
@@ -322,7 +323,9 @@ tid_status run_counts(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, 
   TRY(make_map(&qmap, dq, B, n, kBM));
   // level 1: HBM-resident segments
   for (const Segment& sg : idx->segs)
-    TRY(launch_search_range(idx, qmap, sg.desc, sg.cap, 0, sg.colkey, sg.count, B, n, T, nvalid, counts, R, sg.first, s));
+    if (!sg.on_host && sg.count > 0)
+      TRY(launch_search_range(idx, qmap, sg.desc, sg.cap, 0, sg.colkey, sg.count, B, n, T, nvalid, counts, R, sg.first,
+                              s));
   // level 2: pinned host tier, streamed through two HBM staging buffers on the copy stream
   if (idx->n_host > 0) {
     const int64_t chunk = idx->host_chunk;
@@ -335,18 +338,19 @@ tid_status run_counts(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, 
     // the copy stream must not overwrite staging buffers still read by a previous call
     CU(cudaEventRecord(idx->ev_free[0], s));
     CU(cudaEventRecord(idx->ev_free[1], s));
-    struct Piece { const HostSegment* hs; int64_t off, cnt; };
+    struct Piece { const Segment* sg; int64_t off, cnt; };
     std::vector<Piece> pieces;
-    for (const HostSegment& hs : idx->hsegs)
-      for (int64_t off = 0; off < hs.count; off += chunk) pieces.push_back({&hs, off, std::min(chunk, hs.count - off)});
+    for (const Segment& sg : idx->segs)
+      if (sg.on_host)
+        for (int64_t off = 0; off < sg.count; off += chunk) pieces.push_back({&sg, off, std::min(chunk, sg.count - off)});
     auto issue_copy = [&](size_t i) -> tid_status {
       const int b = static_cast<int>(i & 1);
       const Piece& pc = pieces[i];
       CU(cudaStreamWaitEvent(idx->copy_stream, idx->ev_free[b], 0));
-      CU(cudaMemcpyAsync(idx->stage_desc[b].p, pc.hs->desc + pc.off * rb, static_cast<size_t>(pc.cnt * rb),
+      CU(cudaMemcpyAsync(idx->stage_desc[b].p, pc.sg->desc + pc.off * rb, static_cast<size_t>(pc.cnt * rb),
                          cudaMemcpyHostToDevice, idx->copy_stream));
-      CU(cudaMemcpyAsync(idx->stage_kp[b].p, idx->host_kp.data() + (pc.hs->first - idx->n_hbm) + pc.off,
-                         static_cast<size_t>(pc.cnt) * 4, cudaMemcpyHostToDevice, idx->copy_stream));
+      CU(cudaMemcpyAsync(idx->stage_kp[b].p, pc.sg->kp.data() + pc.off, static_cast<size_t>(pc.cnt) * 4,
+                         cudaMemcpyHostToDevice, idx->copy_stream));
       CU(cudaEventRecord(idx->ev_h2d[b], idx->copy_stream));
       if (idx->prof) idx->stats.h2d_bytes += pc.cnt * rb + pc.cnt * 4;
       return TID_OK;
@@ -368,10 +372,119 @@ tid_status run_counts(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, 
       launch_ref_prep(rp, s);
       count_kernel(idx);
       TRY(launch_search_range(idx, qmap, idx->stage_desc[b].as<uint8_t>(), chunk, 0, rp.colkey, pc.cnt, B, n, T,
-                              nvalid, counts, R, pc.hs->first + pc.off, s));
+                              nvalid, counts, R, pc.sg->first + pc.off, s));
       CU(cudaEventRecord(idx->ev_free[b], s));
     }
   }
+  return TID_OK;
+}
+
+// Allocate a segment of `cap` references in one tier (all-or-nothing).
+tid_status alloc_segment(tid_index* idx, bool on_host, int64_t cap, Segment* out) {
+  const int64_t rb = idx->ref_bytes;
+  Segment sg;
+  sg.on_host = on_host;
+  sg.cap = cap;
+  if (on_host) {
+    if (cudaHostAlloc(reinterpret_cast<void**>(&sg.desc), static_cast<size_t>(cap * rb), cudaHostAllocPortable) !=
+        cudaSuccess) {
+      cudaGetLastError();
+      return fail(TID_ENOMEM, "pinned host tier allocation of %lld bytes failed", static_cast<long long>(cap * rb));
+    }
+    idx->host_alloc += cap * rb;
+  } else {
+    cudaError_t e1 = cudaMalloc(&sg.desc, static_cast<size_t>(cap * rb));
+    cudaError_t e2 = e1 == cudaSuccess ? cudaMalloc(&sg.colkey, static_cast<size_t>(cap) * idx->cpr * kColBytes) : e1;
+    if (e1 != cudaSuccess || e2 != cudaSuccess) {
+      cudaGetLastError();
+      if (sg.desc) cudaFree(sg.desc);
+      return fail(TID_ENOMEM, "HBM arena allocation of %lld references failed", static_cast<long long>(cap));
+    }
+    idx->hbm_alloc += cap * rb + cap * idx->cpr * kColBytes;
+  }
+  *out = std::move(sg);
+  return TID_OK;
+}
+
+void free_segment(tid_index* idx, Segment& sg) {
+  if (sg.on_host) {
+    if (sg.desc) cudaFreeHost(sg.desc);
+    idx->host_alloc -= sg.cap * idx->ref_bytes;
+  } else {
+    if (sg.desc) cudaFree(sg.desc);
+    if (sg.colkey) cudaFree(sg.colkey);
+    idx->hbm_alloc -= sg.cap * idx->ref_bytes + sg.cap * idx->cpr * kColBytes;
+  }
+  sg.desc = nullptr;
+  sg.colkey = nullptr;
+}
+
+// Ingest `take` references (host or device `src`, kp_host per reference) into HBM segment sg at
+// position `pos`: copy, zero padding rows, N_R -> packed column keys (Alg. 1 step 1).
+tid_status ingest_hbm(tid_index* idx, Segment& sg, int64_t pos, const uint8_t* src, bool src_dev,
+                      const int32_t* kp_host, int64_t take) {
+  const int64_t rb = idx->ref_bytes;
+  uint8_t* dst = sg.desc + pos * rb;
+  RefPrepParams rp{};
+  rp.desc = dst;
+  rp.m = idx->cfg.ref_kp;
+  rp.cpr = idx->cpr;
+  rp.count = take;
+  rp.colkey = sg.colkey + pos * idx->cpr * kColInts;
+  if (src_dev) {
+    rp.src = src;
+  } else {
+    CU(cudaMemcpy(dst, src, static_cast<size_t>(take * rb), cudaMemcpyHostToDevice));
+    rp.src = nullptr;
+  }
+  TRY(idx->ws_kp.ensure(static_cast<size_t>(take) * 4, "kp staging"));
+  CU(cudaMemcpy(idx->ws_kp.p, kp_host, static_cast<size_t>(take) * 4, cudaMemcpyHostToDevice));
+  rp.kp = idx->ws_kp.as<int32_t>();
+  launch_ref_prep(rp, nullptr);
+  CU(cudaGetLastError());
+  CU(cudaStreamSynchronize(nullptr));
+  return TID_OK;
+}
+
+// FIFO swap-out (§6.1): move the oldest HBM segment to the pinned host tier.
+tid_status evict_oldest_hbm(tid_index* idx) {
+  Segment* victim = nullptr;
+  for (Segment& sg : idx->segs)
+    if (!sg.on_host && sg.count > 0) { victim = &sg; break; }
+  if (!victim) return fail(TID_ENOMEM, "nothing to evict from HBM");
+  const int64_t rb = idx->ref_bytes;
+  if (static_cast<uint64_t>(idx->n_host + victim->count) * rb > idx->host_budget)
+    return fail(TID_ENOMEM, "host tier full: cannot swap out %lld references", static_cast<long long>(victim->count));
+  Segment hs;
+  TRY(alloc_segment(idx, true, victim->count, &hs));
+  // the arena copy has padding rows zeroed and is otherwise identical to what was added
+  if (cudaMemcpy(hs.desc, victim->desc, static_cast<size_t>(victim->count * rb), cudaMemcpyDeviceToHost) != cudaSuccess) {
+    cudaGetLastError();
+    free_segment(idx, hs);
+    return fail(TID_ECUDA, "swap-out copy failed");
+  }
+  hs.first = victim->first;
+  hs.count = victim->count;
+  hs.kp = std::move(victim->kp);
+  idx->n_hbm -= victim->count;
+  idx->n_host += victim->count;
+  free_segment(idx, *victim);
+  *victim = std::move(hs);
+  return TID_OK;
+}
+
+Segment* find_segment(tid_index* idx, int64_t id, int64_t* off) {
+  for (Segment& sg : idx->segs)
+    if (id >= sg.first && id < sg.first + sg.count) { *off = id - sg.first; return &sg; }
+  return nullptr;
+}
+
+tid_status sync_dead(tid_index* idx, cudaStream_t s) {
+  if (!idx->any_dead || !idx->dead_dirty) return TID_OK;
+  TRY(idx->dead_dev.ensure(idx->dead.size(), "dead flags"));
+  CU(cudaMemcpyAsync(idx->dead_dev.p, idx->dead.data(), idx->dead.size(), cudaMemcpyHostToDevice, s));
+  CU(cudaStreamSynchronize(s));
+  idx->dead_dirty = false;
   return TID_OK;
 }
 
@@ -490,8 +603,8 @@ tid_status tid_index_destroy(tid_index* idx) {
   if (!idx) return TID_OK;
   cudaSetDevice(idx->device);
   cudaDeviceSynchronize();
-  for (Segment& s : idx->segs) { cudaFree(s.desc); cudaFree(s.colkey); }
-  for (HostSegment& h : idx->hsegs) cudaFreeHost(h.desc);
+  for (Segment& sg : idx->segs) free_segment(idx, sg);
+  idx->dead_dev.release();
   DevBuf* bufs[] = {&idx->ws_q, &idx->ws_nq, &idx->ws_nvalid, &idx->ws_counts, &idx->ws_cand, &idx->ws_keys,
                     &idx->ws_gather, &idx->ws_ids, &idx->ws_cnts, &idx->ws_r, &idx->ws_colkey, &idx->ws_nn,
                     &idx->ws_kp, &idx->ws_mr, &idx->stage_desc[0], &idx->stage_desc[1], &idx->stage_colkey[0],
@@ -519,105 +632,227 @@ tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t
   if (count == 0) return TID_OK;
   const int64_t rb = idx->ref_bytes;
   const bool dev_in = is_device_ptr(desc);
-  // how many go to HBM (FIFO: HBM fills first, then the host tier; §6.1)
-  int64_t hbm_room = idx->n_host > 0 ? 0 : static_cast<int64_t>(idx->hbm_budget / rb) - idx->n_hbm;
-  hbm_room = std::max<int64_t>(hbm_room, 0);
-  const int64_t to_hbm = std::min(count, hbm_room);
-  const int64_t to_host = count - to_hbm;
-  if (to_host > 0) {
-    const int64_t host_room = static_cast<int64_t>(idx->host_budget / rb) - idx->n_host;
-    if (to_host > host_room)
-      return fail(TID_ENOMEM, "capacity exceeded: %lld references do not fit (HBM room %lld, host room %lld)",
-                  static_cast<long long>(count), static_cast<long long>(hbm_room), static_cast<long long>(host_room));
-  }
-  // kp counts -> host copy (validated) and device copy
-  std::vector<int32_t> kp_host;
+  // keypoint counts: host copy, validated
+  std::vector<int32_t> kp(static_cast<size_t>(count), idx->cfg.ref_kp);
   if (kp_counts) {
-    kp_host.resize(count);
-    CU(cudaMemcpy(kp_host.data(), kp_counts, static_cast<size_t>(count) * 4, cudaMemcpyDefault));
+    CU(cudaMemcpy(kp.data(), kp_counts, static_cast<size_t>(count) * 4, cudaMemcpyDefault));
     for (int64_t i = 0; i < count; ++i)
-      if (kp_host[i] < 0 || kp_host[i] > idx->cfg.ref_kp)
-        return fail(TID_EINVAL, "kp_counts[%lld]=%d outside 0..ref_kp", static_cast<long long>(i), kp_host[i]);
+      if (kp[i] < 0 || kp[i] > idx->cfg.ref_kp)
+        return fail(TID_EINVAL, "kp_counts[%lld]=%d outside 0..ref_kp", static_cast<long long>(i), kp[i]);
   }
-  cudaStream_t s = nullptr;  // ingest is synchronous on the legacy stream
-  // ---- HBM part
+  const int64_t hbm_cap = static_cast<int64_t>(idx->hbm_budget / rb);
+  const int64_t host_cap = static_cast<int64_t>(idx->host_budget / rb);
+  int64_t to_hbm, to_host;
+  if (idx->cfg.cache_policy == 1) {
+    // FIFO (paper §6.1): the new batch enters HBM; the oldest batches are swapped to the host tier
+    if (count > hbm_cap) return fail(TID_ENOMEM, "batch of %lld exceeds the HBM budget", static_cast<long long>(count));
+    int64_t evict_need = idx->n_hbm + count - hbm_cap;
+    if (evict_need > 0 && idx->n_host + evict_need > host_cap)
+      return fail(TID_ENOMEM, "capacity exceeded: HBM full and host tier cannot take the swapped-out batches");
+    while (idx->n_hbm + count > hbm_cap) TRY(evict_oldest_hbm(idx));
+    to_hbm = count;
+    to_host = 0;
+  } else {
+    // fill: HBM first, then the host tier (ids stay in insertion order)
+    const int64_t hbm_room = idx->n_host > 0 ? 0 : std::max<int64_t>(hbm_cap - idx->n_hbm, 0);
+    to_hbm = std::min(count, hbm_room);
+    to_host = count - to_hbm;
+    if (to_host > host_cap - idx->n_host)
+      return fail(TID_ENOMEM, "capacity exceeded: %lld references do not fit (HBM room %lld, host room %lld)",
+                  static_cast<long long>(count), static_cast<long long>(hbm_room),
+                  static_cast<long long>(host_cap - idx->n_host));
+  }
+  // ---- HBM part (append to the last HBM segment if it is the id-tail and has room, else a new one)
   int64_t done = 0;
   while (done < to_hbm) {
     Segment* sg = idx->segs.empty() ? nullptr : &idx->segs.back();
-    if (!sg || sg->count == sg->cap) {
-      const int64_t remaining_budget = static_cast<int64_t>(idx->hbm_budget / rb) - idx->n_hbm;
-      int64_t cap = std::max<int64_t>(to_hbm - done, std::min<int64_t>(idx->n_hbm, remaining_budget));
-      cap = std::min(cap, remaining_budget);
+    const bool can_append = sg && !sg->on_host && sg->count < sg->cap && idx->cfg.cache_policy == 0;
+    if (!can_append) {
+      const int64_t room = hbm_cap - idx->n_hbm;
+      int64_t cap = idx->cfg.cache_policy == 1 ? (to_hbm - done)
+                                               : std::max<int64_t>(to_hbm - done, std::min<int64_t>(idx->n_hbm, room));
+      cap = std::min(cap, room);
       Segment ns;
-      ns.first = idx->n_hbm;
-      cudaError_t e1 = cudaMalloc(&ns.desc, static_cast<size_t>(cap * rb));
-      cudaError_t e2 = e1 == cudaSuccess ? cudaMalloc(&ns.colkey, static_cast<size_t>(cap) * idx->cpr * kColBytes) : e1;
-      if (e1 != cudaSuccess || e2 != cudaSuccess) {
-        cudaGetLastError();
-        if (ns.desc) cudaFree(ns.desc);
-        return fail(TID_ENOMEM, "HBM arena allocation of %lld references failed", static_cast<long long>(cap));
-      }
-      ns.cap = cap;
-      idx->hbm_alloc += cap * rb + cap * idx->cpr * kColBytes;
-      idx->segs.push_back(ns);
+      TRY(alloc_segment(idx, false, cap, &ns));
+      ns.first = first + done;
+      idx->segs.push_back(std::move(ns));
       sg = &idx->segs.back();
     }
     const int64_t take = std::min(to_hbm - done, sg->cap - sg->count);
-    uint8_t* dst = sg->desc + sg->count * rb;
-    const uint8_t* src = desc + done * rb;
-    RefPrepParams rp{};
-    rp.desc = dst;
-    rp.m = idx->cfg.ref_kp;
-    rp.cpr = idx->cpr;
-    rp.count = take;
-    rp.colkey = sg->colkey + sg->count * idx->cpr * kColInts;
-    if (dev_in) {
-      rp.src = src;
-    } else {
-      CU(cudaMemcpyAsync(dst, src, static_cast<size_t>(take * rb), cudaMemcpyHostToDevice, s));
-      rp.src = nullptr;
-    }
-    if (kp_counts) {
-      TRY(idx->ws_kp.ensure(static_cast<size_t>(take) * 4, "kp staging"));
-      CU(cudaMemcpyAsync(idx->ws_kp.p, kp_host.data() + done, static_cast<size_t>(take) * 4, cudaMemcpyHostToDevice, s));
-      rp.kp = idx->ws_kp.as<int32_t>();
-    }
-    launch_ref_prep(rp, s);
-    CU(cudaGetLastError());
-    CU(cudaStreamSynchronize(s));
+    TRY(ingest_hbm(idx, *sg, sg->count, desc + done * rb, dev_in, kp.data() + done, take));
+    sg->kp.insert(sg->kp.end(), kp.begin() + done, kp.begin() + done + take);
     sg->count += take;
     idx->n_hbm += take;
     done += take;
   }
-  // ---- host tier part (raw bytes; zeroing + norms happen on the GPU when streamed)
+  // ---- host-tier part (raw bytes; zeroing + keys happen on the GPU when streamed)
   int64_t hdone = 0;
   while (hdone < to_host) {
-    HostSegment* hs = idx->hsegs.empty() ? nullptr : &idx->hsegs.back();
-    if (!hs || hs->count == hs->cap) {
-      const int64_t room = static_cast<int64_t>(idx->host_budget / rb) - idx->n_host;
+    Segment* sg = idx->segs.empty() ? nullptr : &idx->segs.back();
+    if (!sg || !sg->on_host || sg->count == sg->cap) {
+      const int64_t room = host_cap - idx->n_host;
       int64_t cap = std::max<int64_t>(to_host - hdone, std::min<int64_t>(idx->n_host, room));
       cap = std::min(cap, room);
-      HostSegment nh;
-      nh.first = idx->n_hbm + idx->n_host;
-      if (cudaHostAlloc(reinterpret_cast<void**>(&nh.desc), static_cast<size_t>(cap * rb), cudaHostAllocPortable) !=
-          cudaSuccess) {
-        cudaGetLastError();
-        return fail(TID_ENOMEM, "pinned host tier allocation of %lld bytes failed", static_cast<long long>(cap * rb));
-      }
-      nh.cap = cap;
-      idx->host_alloc += cap * rb;
-      idx->hsegs.push_back(nh);
-      hs = &idx->hsegs.back();
+      Segment ns;
+      TRY(alloc_segment(idx, true, cap, &ns));
+      ns.first = first + to_hbm + hdone;
+      idx->segs.push_back(std::move(ns));
+      sg = &idx->segs.back();
     }
-    const int64_t take = std::min(to_host - hdone, hs->cap - hs->count);
-    const uint8_t* src = desc + (to_hbm + hdone) * rb;
-    CU(cudaMemcpy(hs->desc + hs->count * rb, src, static_cast<size_t>(take * rb), cudaMemcpyDefault));
-    for (int64_t i = 0; i < take; ++i)
-      idx->host_kp.push_back(kp_counts ? kp_host[to_hbm + hdone + i] : idx->cfg.ref_kp);
-    hs->count += take;
+    const int64_t take = std::min(to_host - hdone, sg->cap - sg->count);
+    CU(cudaMemcpy(sg->desc + sg->count * rb, desc + (to_hbm + hdone) * rb, static_cast<size_t>(take * rb),
+                  cudaMemcpyDefault));
+    sg->kp.insert(sg->kp.end(), kp.begin() + to_hbm + hdone, kp.begin() + to_hbm + hdone + take);
+    sg->count += take;
     idx->n_host += take;
     hdone += take;
   }
+  idx->dead.resize(static_cast<size_t>(first + count), 0);
+  idx->dead_dirty = true;
+  return TID_OK;
+}
+
+tid_status tid_delete_references(tid_index* idx, const int64_t* local_ids, int64_t count) {
+  if (!idx) return fail(TID_EINVAL, "null index");
+  if (count < 0 || (count > 0 && !local_ids)) return fail(TID_EINVAL, "bad ids");
+  TRY(set_device(idx));
+  std::vector<int64_t> ids(static_cast<size_t>(count));
+  if (count) CU(cudaMemcpy(ids.data(), local_ids, static_cast<size_t>(count) * 8, cudaMemcpyDefault));
+  const int64_t R = idx->n_hbm + idx->n_host;
+  for (int64_t id : ids)
+    if (id < 0 || id >= R) return fail(TID_EINVAL, "local id %lld out of range", static_cast<long long>(id));
+  const int32_t zero = 0;
+  for (int64_t id : ids) {
+    int64_t off;
+    Segment* sg = find_segment(idx, id, &off);
+    sg->kp[off] = 0;  // no keypoints: every column becomes padding -> count 0
+    if (!sg->on_host) {
+      RefPrepParams rp{};
+      rp.desc = sg->desc + off * idx->ref_bytes;
+      rp.src = nullptr;
+      TRY(idx->ws_kp.ensure(4, "kp"));
+      CU(cudaMemcpy(idx->ws_kp.p, &zero, 4, cudaMemcpyHostToDevice));
+      rp.kp = idx->ws_kp.as<int32_t>();
+      rp.colkey = sg->colkey + off * idx->cpr * kColInts;
+      rp.count = 1;
+      rp.m = idx->cfg.ref_kp;
+      rp.cpr = idx->cpr;
+      launch_ref_prep(rp, nullptr);
+      CU(cudaStreamSynchronize(nullptr));
+    }
+    idx->dead[static_cast<size_t>(id)] = 1;
+  }
+  idx->any_dead = idx->any_dead || count > 0;
+  idx->dead_dirty = true;
+  return TID_OK;
+}
+
+tid_status tid_update_references(tid_index* idx, const int64_t* local_ids, const uint8_t* desc,
+                                 const int32_t* kp_counts, int64_t count) {
+  if (!idx) return fail(TID_EINVAL, "null index");
+  if (count < 0 || (count > 0 && (!local_ids || !desc))) return fail(TID_EINVAL, "bad arguments");
+  TRY(set_device(idx));
+  std::vector<int64_t> ids(static_cast<size_t>(count));
+  if (count) CU(cudaMemcpy(ids.data(), local_ids, static_cast<size_t>(count) * 8, cudaMemcpyDefault));
+  std::vector<int32_t> kp(static_cast<size_t>(count), idx->cfg.ref_kp);
+  if (kp_counts && count) CU(cudaMemcpy(kp.data(), kp_counts, static_cast<size_t>(count) * 4, cudaMemcpyDefault));
+  const int64_t R = idx->n_hbm + idx->n_host;
+  for (int64_t i = 0; i < count; ++i) {
+    if (ids[i] < 0 || ids[i] >= R) return fail(TID_EINVAL, "local id %lld out of range", static_cast<long long>(ids[i]));
+    if (kp[i] < 0 || kp[i] > idx->cfg.ref_kp) return fail(TID_EINVAL, "kp_counts[%lld] out of range", static_cast<long long>(i));
+  }
+  const int64_t rb = idx->ref_bytes;
+  const bool dev_in = is_device_ptr(desc);
+  for (int64_t i = 0; i < count; ++i) {
+    int64_t off;
+    Segment* sg = find_segment(idx, ids[i], &off);
+    if (sg->on_host) {
+      CU(cudaMemcpy(sg->desc + off * rb, desc + i * rb, static_cast<size_t>(rb), cudaMemcpyDefault));
+    } else {
+      TRY(ingest_hbm(idx, *sg, off, desc + i * rb, dev_in, &kp[i], 1));
+    }
+    sg->kp[off] = kp[i];
+    idx->dead[static_cast<size_t>(ids[i])] = 0;
+  }
+  idx->dead_dirty = true;
+  return TID_OK;
+}
+
+// File layout (little endian): "TIDX" u32 version=1 | i32 dim | i32 ref_kp | i64 num_refs |
+// i32 kp[num_refs] | u8 dead[num_refs] | u8 desc[num_refs][ref_kp][128] (padding rows zeroed).
+tid_status tid_index_save(const tid_index* cidx, const char* path) {
+  tid_index* idx = const_cast<tid_index*>(cidx);
+  if (!idx || !path) return fail(TID_EINVAL, "null argument");
+  TRY(set_device(idx));
+  FILE* f = fopen(path, "wb");
+  if (!f) return fail(TID_EINVAL, "cannot open %s for writing", path);
+  const int64_t R = idx->n_hbm + idx->n_host, rb = idx->ref_bytes;
+  const uint32_t ver = 1;
+  const int32_t dim = kDim, m = idx->cfg.ref_kp;
+  bool ok = fwrite("TIDX", 1, 4, f) == 4 && fwrite(&ver, 4, 1, f) == 1 && fwrite(&dim, 4, 1, f) == 1 &&
+            fwrite(&m, 4, 1, f) == 1 && fwrite(&R, 8, 1, f) == 1;
+  for (const Segment& sg : idx->segs) ok = ok && fwrite(sg.kp.data(), 4, sg.kp.size(), f) == sg.kp.size();
+  ok = ok && fwrite(idx->dead.data(), 1, idx->dead.size(), f) == idx->dead.size();
+  std::vector<uint8_t> buf;
+  for (const Segment& sg : idx->segs) {
+    const int64_t chunk = 4096;
+    for (int64_t off = 0; ok && off < sg.count; off += chunk) {
+      const int64_t c = std::min(chunk, sg.count - off);
+      buf.resize(static_cast<size_t>(c * rb));
+      if (cudaMemcpy(buf.data(), sg.desc + off * rb, buf.size(), cudaMemcpyDefault) != cudaSuccess) {
+        cudaGetLastError();
+        ok = false;
+        break;
+      }
+      if (sg.on_host)  // the host tier keeps raw rows: zero padding rows so the file is canonical
+        for (int64_t r = 0; r < c; ++r)
+          for (int32_t i = sg.kp[off + r]; i < m; ++i) memset(buf.data() + (r * m + i) * kDim, 0, kDim);
+      ok = ok && fwrite(buf.data(), 1, buf.size(), f) == buf.size();
+    }
+  }
+  fclose(f);
+  if (!ok) return fail(TID_ECUDA, "write to %s failed", path);
+  return TID_OK;
+}
+
+tid_status tid_index_load(tid_index* idx, const char* path, int64_t* first_local_id) {
+  if (!idx || !path) return fail(TID_EINVAL, "null argument");
+  FILE* f = fopen(path, "rb");
+  if (!f) return fail(TID_EINVAL, "cannot open %s", path);
+  char magic[4];
+  uint32_t ver = 0;
+  int32_t dim = 0, m = 0;
+  int64_t R = 0;
+  bool ok = fread(magic, 1, 4, f) == 4 && memcmp(magic, "TIDX", 4) == 0 && fread(&ver, 4, 1, f) == 1 && ver == 1 &&
+            fread(&dim, 4, 1, f) == 1 && fread(&m, 4, 1, f) == 1 && fread(&R, 8, 1, f) == 1;
+  if (!ok || dim != kDim || m != idx->cfg.ref_kp || R < 0) {
+    fclose(f);
+    return fail(TID_EINVAL, "%s: not a tid index file for ref_kp=%d", path, idx->cfg.ref_kp);
+  }
+  std::vector<int32_t> kp(static_cast<size_t>(R));
+  std::vector<uint8_t> dead(static_cast<size_t>(R));
+  ok = fread(kp.data(), 4, kp.size(), f) == kp.size() && fread(dead.data(), 1, dead.size(), f) == dead.size();
+  const int64_t rb = idx->ref_bytes, first = idx->n_hbm + idx->n_host;
+  std::vector<uint8_t> buf;
+  int64_t chunk = 16384;
+  if (idx->cfg.cache_policy == 1)  // FIFO batches must fit in HBM; keep half of it for the swap
+    chunk = std::max<int64_t>(1, std::min<int64_t>(chunk, static_cast<int64_t>(idx->hbm_budget / rb) / 2));
+  for (int64_t off = 0; ok && off < R; off += chunk) {
+    const int64_t c = std::min(chunk, R - off);
+    buf.resize(static_cast<size_t>(c * rb));
+    ok = fread(buf.data(), 1, buf.size(), f) == buf.size();
+    if (ok) {
+      tid_status st = tid_add_references(idx, buf.data(), kp.data() + off, c, nullptr);
+      if (st != TID_OK) { fclose(f); return st; }
+    }
+  }
+  fclose(f);
+  if (!ok) return fail(TID_EINVAL, "%s: truncated", path);
+  std::vector<int64_t> del;
+  for (int64_t i = 0; i < R; ++i)
+    if (dead[i]) del.push_back(first + i);
+  if (!del.empty()) TRY(tid_delete_references(idx, del.data(), static_cast<int64_t>(del.size())));
+  if (first_local_id) *first_local_id = first;
   return TID_OK;
 }
 
@@ -665,7 +900,9 @@ tid_status tid_search(tid_index* idx, const uint8_t* queries, const int32_t* n_q
   int64_t segs = std::max<int64_t>(1, std::min<int64_t>(ceil_div(2LL * idx->num_sms, B), ceil_div(R, 4096)));
   segs = std::min<int64_t>(segs, 1024);
   TRY(idx->ws_cand.ensure(static_cast<size_t>(B) * segs * k * 8, "top-k candidates"));
-  launch_topk(counts, B, R, R, idx->cfg.id_base, k, static_cast<int32_t>(segs), idx->ws_cand.as<uint64_t>(), s);
+  TRY(sync_dead(idx, s));
+  launch_topk(counts, B, R, R, idx->cfg.id_base, k, static_cast<int32_t>(segs),
+              idx->any_dead ? idx->dead_dev.as<uint8_t>() : nullptr, idx->ws_cand.as<uint64_t>(), s);
   count_kernel(idx);
   TRY(idx->ws_ids.ensure(static_cast<size_t>(B) * k * 8, "ids"));
   TRY(idx->ws_cnts.ensure(static_cast<size_t>(B) * k * 4, "counts"));

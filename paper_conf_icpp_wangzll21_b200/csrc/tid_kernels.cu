@@ -901,7 +901,7 @@ __device__ void block_select(const uint64_t* lists, int k, uint64_t* out, uint64
 
 // grid (B, segs), 256 threads, dyn smem = 256*k*8 + 33*8.
 __global__ void topk_kernel(const uint32_t* __restrict__ counts, int64_t R, int64_t ldc, int64_t id_base, int32_t k,
-                            uint64_t* __restrict__ cand_out) {
+                            const uint8_t* __restrict__ dead, uint64_t* __restrict__ cand_out) {
   extern __shared__ uint64_t tk_smem[];
   uint64_t* lists = tk_smem;
   uint64_t* red = tk_smem + blockDim.x * k;
@@ -913,6 +913,7 @@ __global__ void topk_kernel(const uint32_t* __restrict__ counts, int64_t R, int6
   uint64_t kth = 0;
   const uint32_t* row = counts + static_cast<int64_t>(b) * ldc;
   for (int64_t r = r0 + threadIdx.x; r < r1; r += blockDim.x) {
+    if (dead && dead[r]) continue;  // deleted references are never ranked
     const uint64_t key = make_key(row[r], id_base + r);
     if (key > kth) {  // insertion into the thread's descending list
       int pos = k - 1;
@@ -926,7 +927,7 @@ __global__ void topk_kernel(const uint32_t* __restrict__ counts, int64_t R, int6
 }
 
 void launch_topk(const uint32_t* counts, int64_t B, int64_t R, int64_t ldc, int64_t id_base, int32_t k, int32_t segs,
-                 uint64_t* cand_out, cudaStream_t s) {
+                 const uint8_t* dead, uint64_t* cand_out, cudaStream_t s) {
   const size_t smem = (256 * static_cast<size_t>(k) + 33) * 8;
   static size_t attr = 0;
   if (smem > 48 * 1024 && smem > attr) {
@@ -934,7 +935,7 @@ void launch_topk(const uint32_t* counts, int64_t B, int64_t R, int64_t ldc, int6
     attr = smem;
   }
   topk_kernel<<<dim3(static_cast<unsigned>(B), static_cast<unsigned>(segs)), 256, smem, s>>>(counts, R, ldc, id_base,
-                                                                                              k, cand_out);
+                                                                                              k, dead, cand_out);
 }
 
 // ------------------------------------------------------------------ a6/a9: merge ranked lists

@@ -90,7 +90,7 @@ void launch_query_prep(const uint8_t* q, int64_t B, int32_t n, int32_t tiles_per
 cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap,
                          int grid, cudaStream_t s);
 void launch_topk(const uint32_t* counts, int64_t B, int64_t R, int64_t ldc, int64_t id_base, int32_t k,
-                 int32_t segs, uint64_t* cand_out, cudaStream_t s);
+                 int32_t segs, const uint8_t* dead, uint64_t* cand_out, cudaStream_t s);
 void launch_merge(const uint64_t* cand, int32_t L, int64_t B, int32_t k, int64_t list_stride_b,
                   int64_t list_stride_l, uint64_t* keys_out, int64_t* ids_out, int32_t* counts_out,
                   cudaStream_t s);

@@ -67,4 +67,4 @@ def test_config_struct_matches_header():
     fields = re.findall(r"^\s*(?:const\s+)?\w+\*?\s+\*?(\w+)(?:,\s*(\w+))?;", body, re.M)
     names = [x for f in fields for x in f if x]
     assert names == [f for f, _ in tid.Config._fields_]
-    assert ctypes.sizeof(tid.Config) == 64
+    assert ctypes.sizeof(tid.Config) == 72

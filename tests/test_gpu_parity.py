@@ -278,3 +278,67 @@ def test_search_m_above_256(tid, m, n, kp_min):
     np.testing.assert_array_equal(counts.astype(np.int64), e_counts)
     np.testing.assert_array_equal(ids, e_ids)
     np.testing.assert_array_equal(cnt, e_cnt)
+
+
+# ------------------------------------------------------------------------------ index lifecycle (f3)
+def _search_all(idx, qs, k):
+    return idx.search_counts(qs), idx.search(qs, k)
+
+
+def test_fifo_policy_swaps_oldest_batches(tid):
+    """Paper §6.1: new batches enter HBM, the oldest are swapped to the host tier
+    when HBM is full; results equal the all-HBM index."""
+    R, m, n, B, k = 120, 256, 300, 3, 6
+    refs, kp = tidgen.refs(0, R, m, kp_min=60, pad_byte=5)
+    qs, _ = tidgen.queries(0, B, n, R_total=R, m=m, kp_min=60, n_planted=50)
+    rb = m * 128
+    with tid.Index(ref_kp=m) as a:
+        a.add_references(refs, kp)
+        ca, (ia, na) = _search_all(a, qs, k)
+    with tid.Index(ref_kp=m, hbm_budget_bytes=50 * rb, host_budget_bytes=200 * rb, cache_policy="fifo") as b:
+        b.set_tuning(host_chunk_refs=17)
+        for s in range(0, R, 30):
+            b.add_references(refs[s:s + 30], kp[s:s + 30])
+        info = b.info()
+        cb, (ib, nb) = _search_all(b, qs, k)
+    assert info["hbm_references"] == 30 and info["host_references"] == 90  # newest batch in HBM
+    np.testing.assert_array_equal(ca, cb)
+    np.testing.assert_array_equal(ia, ib)
+    np.testing.assert_array_equal(na, nb)
+
+
+def test_delete_update_save_load(tid, tmp_path):
+    R, m, n, B, k = 60, 256, 300, 3, 8
+    refs, kp = tidgen.refs(0, R, m, kp_min=80, pad_byte=7)
+    qs, tg = tidgen.queries(0, B, n, R_total=R, m=m, kp_min=80, n_planted=60)
+    new_refs, new_kp = tidgen.refs(1000, 4, m, kp_min=80)
+    upd_ids = np.array([3, 17, 41, 59])
+    rb = m * 128
+    with tid.Index(ref_kp=m, hbm_budget_bytes=35 * rb, host_budget_bytes=100 * rb) as idx:  # spans both tiers
+        idx.add_references(refs, kp)
+        idx.delete([int(tg[0]), 5, 50])
+        idx.update(upd_ids, new_refs, new_kp)
+        counts = idx.search_counts(qs)
+        ids, cnt = idx.search(qs, k)
+        path = str(tmp_path / "index.tid")
+        idx.save(path)
+    # expected: the same edits applied to plain arrays, then the oracle
+    e_refs, e_kp = refs.copy(), kp.copy()
+    e_refs[upd_ids], e_kp[upd_ids] = new_refs, new_kp
+    dead = {int(tg[0]), 5, 50}
+    for d in dead:
+        e_kp[d] = 0
+    e_counts = oracle.search_counts(qs, e_refs, kp=e_kp)
+    np.testing.assert_array_equal(counts.astype(np.int64), e_counts)
+    live = np.array([i for i in range(R) if i not in dead])
+    li, lc = oracle.topk(e_counts[:, live], k)
+    np.testing.assert_array_equal(ids, live[li])
+    np.testing.assert_array_equal(cnt, lc)
+    assert not np.isin(ids, list(dead)).any()
+    with tid.Index(ref_kp=m, cache_policy="fifo", hbm_budget_bytes=40 * rb, host_budget_bytes=100 * rb) as idx2:
+        assert idx2.load(path) == 0
+        c2 = idx2.search_counts(qs)
+        i2, n2 = idx2.search(qs, k)
+    np.testing.assert_array_equal(c2, counts)
+    np.testing.assert_array_equal(i2, ids)
+    np.testing.assert_array_equal(n2, cnt)
