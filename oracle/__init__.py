@@ -199,3 +199,70 @@ def np_rank(counts, k: int, id_base: int = 0):
         out_i[b] = ids[order[:k]]
         out_c[b] = counts[b, order[:k]]
     return out_i, out_c
+
+
+# ------------------------------------------------- f1: RootSIFT + FP16 float path (§4.2, §5.1, Alg. 2)
+def rootsift(X) -> np.ndarray:
+    """RootSIFT: L1-normalise each SIFT vector, then take the element-wise square
+    root; the result has unit L2 norm and Euclidean distance = Hellinger kernel distance."""
+    X = np.asarray(X, np.float64)
+    s = X.sum(-1, keepdims=True)
+    return np.sqrt(np.divide(X, s, out=np.zeros_like(X), where=s > 0))
+
+
+def to_fp16(X, scale: float = 1.0) -> np.ndarray:
+    """FP16 storage with a scale factor applied before the conversion (2^-7 in
+    practice, P:529-530).  Round-to-nearest-even (IEEE)."""
+    return (np.asarray(X, np.float64) * scale).astype(np.float16)
+
+
+def fp16_accumulate_sq_norm(x_fp16) -> np.float16:
+    """||x||^2 accumulated in FP16 arithmetic (each product and partial sum rounded to fp16), the
+    arithmetic of an fp16-accumulating HGEMM.  Pins the Table 2 overflow boundary."""
+    acc = np.float16(0)
+    with np.errstate(over="ignore"):
+        for v in np.asarray(x_fp16, np.float16):
+            acc = np.float16(acc + np.float16(v * v))
+    return acc
+
+
+def f16_dist_matrix(Q16, R16) -> np.ndarray:
+    """Squared distances of fp16-stored descriptors, computed exactly in float64 (the oracle
+    of what the GPU's fp16 x fp16 -> fp32 path approximates)."""
+    Q = np.asarray(Q16, np.float16).astype(np.float64)
+    R = np.asarray(R16, np.float16).astype(np.float64)
+    return ((Q[:, None, :] - R[None, :, :]) ** 2).sum(-1)
+
+
+def f16_match_count(Q16, R16, num: int = 4, den: int = 5, n_q=None, m_r=None) -> int:
+    """2-NN per query row + ratio test on squared distances in the rational form of
+    reading R1, den^2 * d1 < num^2 * d2 (strict), in float64 for fp16-stored
+    descriptors (num/den = 4/5: no rounding of the threshold itself)."""
+    nq = len(Q16) if n_q is None else n_q
+    mr = len(R16) if m_r is None else m_r
+    if mr < 2 or nq == 0:
+        return 0
+    D = f16_dist_matrix(Q16[:nq], R16[:mr])
+    part = np.partition(D, 1, axis=1)[:, :2]
+    d1, d2 = part[:, 0], part[:, 1]
+    return int(np.sum(den * den * d1 < num * num * d2))
+
+
+def f16_search_counts(Qs16, Rs16, num: int = 4, den: int = 5, n_q=None, kp=None) -> np.ndarray:
+    B, R = len(Qs16), len(Rs16)
+    out = np.zeros((B, R), np.int32)
+    for b in range(B):
+        for r in range(R):
+            out[b, r] = f16_match_count(Qs16[b], Rs16[r], num, den, None if n_q is None else n_q[b],
+                                        None if kp is None else kp[r])
+    return out
+
+
+def compression_error(Qf, Rf, Q16, R16) -> float:
+    """Eq. 2: mean over all (i, j) of |rho(R_i, Q_j) - rho_FP16(R_i, Q_j)| / rho(R_i, Q_j),
+    rho = Euclidean distance; the fp16 distances are those of the fp16-stored (scaled)
+    descriptors, un-scaled by the caller's scale factor (pass Q16/R16 already divided)."""
+    rho = np.sqrt(((np.asarray(Rf, np.float64)[:, None, :] - np.asarray(Qf, np.float64)[None, :, :]) ** 2).sum(-1))
+    rho16 = np.sqrt(((np.asarray(R16, np.float64)[:, None, :] - np.asarray(Q16, np.float64)[None, :, :]) ** 2).sum(-1))
+    ok = rho > 0
+    return float(np.mean(np.abs(rho - rho16)[ok] / rho[ok]))
