@@ -240,7 +240,8 @@ tid_status copy_out(tid_index* idx, void* dst, const void* src, size_t bytes, cu
 
 // Choose job decomposition of a search launch: refs per job G and queries per job.
 void plan_search(const tid_index* idx, int64_t n_refs, int64_t B, int T, int* G_out, int* qpj_out) {
-  const int max_g = kMaxSlots / idx->cpr;
+  // refs per job: one per epilogue group (group g <-> resident reference g), fewer for m > 256
+  const int max_g = std::min(kMaxSlots / idx->cpr, kNG);
   int G = idx->tune.refs_per_job > 0 ? std::min(idx->tune.refs_per_job, max_g) : max_g;
   const int64_t target_jobs = 2LL * idx->num_sms;
   // spread small reference sets over more CTAs (fewer resident refs per job)
@@ -282,7 +283,7 @@ tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const ui
   p.ldc = ldc;
   p.col0 = col0;
   p.nn_out = nullptr;
-  p.coarse = idx->tune.exact_only ? 0 : 1;
+  (void)idx->tune.exact_only;  // the scan is always exact (two-partition top-2)
   p.num2 = idx->cfg.ratio_num * idx->cfg.ratio_num;
   p.den2 = idx->cfg.ratio_den * idx->cfg.ratio_den;
   int grid = idx->tune.grid > 0 ? idx->tune.grid : idx->num_sms;

@@ -117,6 +117,9 @@ __device__ __forceinline__ void mma_piece(uint32_t tmem_d, uint64_t adesc, uint6
       "@e tcgen05.mma.cta_group::1.kind::i8 [%0], a1, b1, %3, t;\n\t"
       "@e tcgen05.mma.cta_group::1.kind::i8 [%0], a2, b2, %3, t;\n\t"
       "@e tcgen05.mma.cta_group::1.kind::i8 [%0], a3, b3, %3, t;\n\t"
+#ifdef TID_FAKE_FOLD
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], a3, b3, %3, t;\n\t"
+#endif
       "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%4];\n\t}" ::"r"(tmem_d),
       "l"(adesc), "l"(bdesc), "r"(kIdescI8), "r"(bar)
       : "memory");
@@ -145,16 +148,14 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
       : "r"(taddr));
 }
 
-// 128 consecutive TMEM columns of this thread's lane in one load (32x32b shape, .x128).
-__device__ __forceinline__ void tmem_ld128(uint32_t taddr, uint32_t (&v)[128]) {
+// 64 consecutive TMEM columns of this thread's lane (32x32b shape, .x64).
+__device__ __forceinline__ void tmem_ld64(uint32_t taddr, uint32_t (&v)[64]) {
   asm volatile(
-      "tcgen05.ld.sync.aligned.32x32b.x128.b32 {"
+      "tcgen05.ld.sync.aligned.32x32b.x64.b32 {"
       "%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,"
       "%30,%31,%32,%33,%34,%35,%36,%37,%38,%39,%40,%41,%42,%43,%44,%45,%46,%47,%48,%49,%50,%51,%52,%53,%54,%55,%56,%57,"
-      "%58,%59,%60,%61,%62,%63,%64,%65,%66,%67,%68,%69,%70,%71,%72,%73,%74,%75,%76,%77,%78,%79,%80,%81,%82,%83,%84,%85,"
-      "%86,%87,%88,%89,%90,%91,%92,%93,%94,%95,%96,%97,%98,%99,%100,%101,%102,%103,%104,%105,%106,%107,%108,%109,%110,"
-      "%111,%112,%113,%114,%115,%116,%117,%118,%119,%120,%121,%122,%123,%124,%125,%126,%127}, [%128];"
-      : TID_LD32_OUT(v), TID_LD32_OUT((v + 32)), TID_LD32_OUT((v + 64)), TID_LD32_OUT((v + 96))
+      "%58,%59,%60,%61,%62,%63}, [%64];"
+      : TID_LD32_OUT(v), TID_LD32_OUT((v + 32))
       : "r"(taddr));
 }
 __device__ __forceinline__ int4 lds128(uint32_t addr) {
@@ -170,11 +171,16 @@ __device__ __forceinline__ void reg_fence(uint32_t (&v)[32]) {
   for (int i = 0; i < 32; ++i) asm volatile("" : "+r"(v[i]));
 }
 
+__device__ __forceinline__ void reg_fence64(uint32_t (&v)[64]) {
+#pragma unroll
+  for (int i = 0; i < 64; ++i) asm volatile("" : "+r"(v[i]));
+}
+
 // ------------------------------------------------------------------ optional cycle accounting
 // Built only with -DTID_PROF (experiments): per-warp clock64 buckets, read back with
-// tid_debug_read_prof().  Buckets: epilogue 0 wait-accumulator 1 scan 2 finalise 3 fallback
-// 4 wait-keys; MMA 0 wait-free-accumulator 1 wait-query 2 wait-ref 3 issue; producer 0 wait-ref-slot
-// 1 wait-query-stage; 7 = whole loop.
+// tid_debug_read_prof().  Buckets: epilogue 0 wait-accumulator 1 scan 2 finalise 4 wait-keys;
+// MMA 0 wait-free-accumulator 1 wait-query 2 wait-ref; producer 0 wait-ref-slot 1 wait-query-stage;
+// 7 = whole loop.
 #ifdef TID_PROF
 __device__ unsigned long long g_prof[148 * 32 * 8];
 #define PROF_DECL unsigned long long prof_acc[8] = {0, 0, 0, 0, 0, 0, 0, 0}; long long prof_t0 = 0, prof_all = clock64();
@@ -193,13 +199,11 @@ __device__ unsigned long long g_prof[148 * 32 * 8];
 #define PROF_FLUSH()
 #endif
 
-#ifndef TID_X128
-#define TID_X128 0
-#endif
 constexpr int kProducerWarp = 0;               // warp 0: TMA producer
-constexpr int kFirstMmaWarp = 1;               // warps 1..4: MMA issuers (SMSPs 1, 2, 3, 0)
-constexpr int kFirstEpiWarp = 5;               // warps 5..: epilogue (4 per group)
-static_assert(kNG == 2 || kNG == 4, "4 MMA warps own the 4 TMEM buffers (2 groups x 2 halves, or 4 groups)");
+constexpr int kFirstMmaWarp = 1;               // warps 1..3: MMA issuer of group mw (SMSPs 1, 2, 3)
+constexpr int kFirstEpiWarp = 1 + kNG;         // warps 4..15: epilogue, group (w-4)/4, lane quarter w%4
+// (any 4 consecutive warps cover the 4 TMEM lane quarters w % 4)
+static_assert(kNB == 2 && kNumThreads <= 512, "at most 16 warps: >= 128 registers per thread");
 
 // ------------------------------------------------------------------ shared memory plan
 struct SmemPlan {
@@ -214,9 +218,7 @@ struct SmemPlan {
   static constexpr uint32_t kTFull = kREmpty + 8 * kMaxSlots;
   static constexpr uint32_t kTEmpty = kTFull + 8 * kTmemBufs;
   static constexpr uint32_t kTmemPtr = kTEmpty + 8 * kTmemBufs;
-  static constexpr uint32_t kCnt = kTmemPtr + 16;                          // [4*kNG finalisers][kMaxSlots] u32
-  static constexpr uint32_t kXch = (kCnt + 4 * kNG * kMaxSlots * 4 + 15) & ~15u;  // split-warp state exchange
-  static constexpr uint32_t kEnd = kXch + 4 * kNG * 2 * 32 * (kSplit - 1) * 16 + 16;
+  static constexpr uint32_t kEnd = kTmemPtr + 16;
   static constexpr uint32_t kAlloc = kEnd + 1024;                          // + alignment slack
 };
 
@@ -242,200 +244,77 @@ __device__ __forceinline__ Job decode_job(const MatchParams& p, int32_t j) {
   return J;
 }
 
-// ------------------------------------------------------------------ epilogue scans
-// A "piece" = one 128-column accumulator buffer (MMA N = 128) of one (query tile, reference
-// chunk half).  Each epilogue thread owns one TMEM lane = one query row.
-
-// Exact top-2 over one piece, accumulated into running states (a1 <= a2, b1 <= b2) of packed keys
-// 256 * (N_R - 2S) + i (unique per column within a 256-column chunk).  ~2.5 ALU ops / element.
-template <int NCOL>
-__device__ __forceinline__ void scan_exact(uint32_t taddr, uint32_t ck_addr, int& a1, int& a2, int& b1, int& b2) {
-  uint32_t v[2][32];
-  tmem_ld32(taddr, v[0]);
-  tmem_wait_ld();
-  reg_fence(v[0]);
-#pragma unroll
-  for (int jj = 0; jj < NCOL / 32; ++jj) {
-    // software pipeline: the next 32 columns are in flight while these are scanned
-    if (jj + 1 < NCOL / 32) tmem_ld32(taddr + (jj + 1) * 32, v[(jj + 1) & 1]);
-    const uint32_t* w = v[jj & 1];
-#pragma unroll
-    for (int i = 0; i < 32; i += 4) {
-      const int4 c4 = lds128(ck_addr + (jj * 32 + i) * 4);
-      const int x0 = c4.x - 512 * static_cast<int>(w[i]);
-      const int x1 = c4.y - 512 * static_cast<int>(w[i + 1]);
-      const int x2 = c4.z - 512 * static_cast<int>(w[i + 2]);
-      const int x3 = c4.w - 512 * static_cast<int>(w[i + 3]);
-      int lo = min(x0, x1), hi = max(x0, x1);
-      int tt = max(a1, lo);
-      a2 = min(min(a2, tt), hi);
-      a1 = min(a1, lo);
-      lo = min(x2, x3); hi = max(x2, x3);
-      tt = max(b1, lo);
-      b2 = min(min(b2, tt), hi);
-      b1 = min(b1, lo);
-    }
-    // the state must be final before waiting for the next TMEM load (keeps the scan streaming)
-    asm volatile("" : "+r"(a1), "+r"(a2), "+r"(b1), "+r"(b2));
-    if (jj + 1 < NCOL / 32) { tmem_wait_ld(); reg_fence(v[(jj + 1) & 1]); }
-  }
+// ------------------------------------------------------------------ epilogue: two-partition top-2
+// Each epilogue thread owns one TMEM lane = one query row j, and needs the two smallest packed
+// keys 256 * (N_R - 2 q_j.r_i) + i over the 256 columns i of a reference chunk (Alg. 1 steps
+// 4-7 P:375-382; "keep two registers" P:420-425).  Instead of a running top-2 (min + max + min
+// per element), the columns are covered by two partitions that separate every pair:
+//   P : (x32 load c, half h)        -> 16 groups of 16 columns      (c = 0..7, h = j >= 16)
+//   P': column position b = j % 16  -> 16 groups of 16 columns      (j = position in the load)
+// Two columns in the same P group differ in b, so no pair shares both groups.  Then
+//   min(all) = min(P minima)  and  second(all) = min(second(P minima), second(P' minima)):
+// if the two smallest columns fall in different P groups, both are P minima; otherwise they
+// are in different P' groups and both are P' minima; and neither side can undercut the true
+// second.  Both partitions are pure 3-input minima (VIMNMX3, one per two new elements), so the
+// scan costs ~1.3 ALU ops per element instead of 2.5, and it is exact (keys carry the index).
+__device__ __forceinline__ int min3i(int a, int b, int c) { return __vimin3_s32(a, b, c); }
+__device__ __forceinline__ int min16(const int* k) {
+  const int a = min3i(k[0], k[1], k[2]), b = min3i(k[3], k[4], k[5]), c = min3i(k[6], k[7], k[8]);
+  const int d = min3i(k[9], k[10], k[11]), e = min3i(k[12], k[13], k[14]);
+  return min(min3i(a, b, c), min3i(d, e, k[15]));
 }
 
-__device__ __forceinline__ uint32_t prmt_top16x2(uint32_t a, uint32_t b) {  // a[31:16] | b[31:16] << 16
-  uint32_t r;
-  asm("prmt.b32 %0, %1, %2, 0x7632;" : "=r"(r) : "r"(a), "r"(b));
-  return r;
+// 32 consecutive columns of this lane (one x32 TMEM load, already landed in v) folded into the
+// partition state: R[b] = P' minima, (T1 <= T2) = the two smallest P minima so far.
+__device__ __forceinline__ void scan32_regs(const uint32_t* v, uint32_t ck_addr, int (&R)[16], int& T1, int& T2) {
+  int k[32];
+#pragma unroll
+  for (int i = 0; i < 32; i += 4) {
+#ifdef TID_FAKE_FOLD  // timing experiment only: keys straight from TMEM (wrong results)
+    k[i] = v[i]; k[i + 1] = v[i + 1]; k[i + 2] = v[i + 2]; k[i + 3] = v[i + 3];
+#else
+    const int4 c4 = lds128(ck_addr + i * 4);
+    k[i] = c4.x - 512 * static_cast<int>(v[i]);
+    k[i + 1] = c4.y - 512 * static_cast<int>(v[i + 1]);
+    k[i + 2] = c4.z - 512 * static_cast<int>(v[i + 2]);
+    k[i + 3] = c4.w - 512 * static_cast<int>(v[i + 3]);
+#endif
+  }
+  const int x = min16(k), y = min16(k + 16);
+#pragma unroll
+  for (int b = 0; b < 16; ++b) R[b] = min3i(R[b], k[b], k[b + 16]);
+  const int lo = min(x, y), hi = max(x, y);
+  T2 = min3i(T2, max(T1, lo), hi);
+  T1 = min(T1, lo);
 }
 
-// Coarse top-2 over one piece (search fast path): the exact key 256*(N_R - 2S) + i is formed by
-// the same IMAD (FMA pipe); its top 16 bits floor((N_R - 2S)/256) are packed two columns per
-// register (one PRMT) and the top-2 runs on s16x2 lanes (VIMNMX.S16x2 and 3-input forms):
-// ~1.75 ALU ops per element instead of 2.5.  Accumulates into four sorted packed states; the two
-// smallest coarse keys u1 <= u2 of their union bound N_R - 2S of the true 1st / 2nd neighbour
-// to [256 u, 256 u + 255].
-template <int NCOL>
-__device__ __forceinline__ void scan_coarse(uint32_t taddr, uint32_t ck_addr, uint32_t& A1, uint32_t& A2,
-                                            uint32_t& B1, uint32_t& B2) {
-  uint32_t v[2][32];
-  int4 ck[2][8];  // column keys, loaded one 32-column chunk ahead (hides the LDS latency)
-  tmem_ld32(taddr, v[0]);
+// Two smallest keys (k1 < k2) of a 256-column chunk from the partition state.  The 16 P'
+// minima are themselves split by a 4 x 4 grid (rows R[4a..4a+3], columns R[b], R[b+4], ...),
+// which again separates every pair, so second(R) = min(second(row minima), second(col minima)).
+__device__ __forceinline__ void finish_partition(const int (&R)[16], int T1, int T2, int& k1, int& k2) {
+  int rm[4], cm[4];
 #pragma unroll
-  for (int i = 0; i < 8; ++i) ck[0][i] = lds128(ck_addr + i * 16);
-  tmem_wait_ld();
-  reg_fence(v[0]);
-#pragma unroll
-  for (int jj = 0; jj < NCOL / 32; ++jj) {
-    if (jj + 1 < NCOL / 32) {
-      tmem_ld32(taddr + (jj + 1) * 32, v[(jj + 1) & 1]);
-#pragma unroll
-      for (int i = 0; i < 8; ++i) ck[(jj + 1) & 1][i] = lds128(ck_addr + ((jj + 1) * 32 + i * 4) * 4);
-    }
-    const uint32_t* w = v[jj & 1];
-    const int4* c4 = ck[jj & 1];
-#pragma unroll
-    for (int i = 0; i < 32; i += 8) {
-      const int4 c0 = c4[i / 4], c1 = c4[i / 4 + 1];
-      const uint32_t k0 = static_cast<uint32_t>(c0.x - 512 * static_cast<int>(w[i]));
-      const uint32_t k1 = static_cast<uint32_t>(c0.y - 512 * static_cast<int>(w[i + 1]));
-      const uint32_t k2 = static_cast<uint32_t>(c0.z - 512 * static_cast<int>(w[i + 2]));
-      const uint32_t k3 = static_cast<uint32_t>(c0.w - 512 * static_cast<int>(w[i + 3]));
-      const uint32_t k4 = static_cast<uint32_t>(c1.x - 512 * static_cast<int>(w[i + 4]));
-      const uint32_t k5 = static_cast<uint32_t>(c1.y - 512 * static_cast<int>(w[i + 5]));
-      const uint32_t k6 = static_cast<uint32_t>(c1.z - 512 * static_cast<int>(w[i + 6]));
-      const uint32_t k7 = static_cast<uint32_t>(c1.w - 512 * static_cast<int>(w[i + 7]));
-      const uint32_t x = prmt_top16x2(k0, k1), y = prmt_top16x2(k2, k3);
-      const uint32_t z = prmt_top16x2(k4, k5), ww = prmt_top16x2(k6, k7);
-      uint32_t lo = __vmins2(x, y), hi = __vmaxs2(x, y);
-      uint32_t tt = __vmaxs2(A1, lo);
-      A2 = __vmins2(__vmins2(A2, tt), hi);
-      A1 = __vmins2(A1, lo);
-      lo = __vmins2(z, ww); hi = __vmaxs2(z, ww);
-      tt = __vmaxs2(B1, lo);
-      B2 = __vmins2(__vmins2(B2, tt), hi);
-      B1 = __vmins2(B1, lo);
-    }
-    asm volatile("" : "+r"(A1), "+r"(A2), "+r"(B1), "+r"(B2));
-    if (jj + 1 < NCOL / 32) { tmem_wait_ld(); reg_fence(v[(jj + 1) & 1]); }
+  for (int a = 0; a < 4; ++a) {
+    rm[a] = min(min3i(R[4 * a], R[4 * a + 1], R[4 * a + 2]), R[4 * a + 3]);
+    cm[a] = min(min3i(R[a], R[a + 4], R[a + 8]), R[a + 12]);
   }
-}
-
-// Same scan, one .x128 TMEM load per piece and a single wait (latency exposed once per piece).
-__device__ __forceinline__ void scan_coarse_x128(uint32_t taddr, uint32_t ck_addr, uint32_t& A1, uint32_t& A2,
-                                                 uint32_t& B1, uint32_t& B2) {
-  uint32_t v[128];
-  tmem_ld128(taddr, v);
-  tmem_wait_ld();
-#pragma unroll
-  for (int i = 0; i < 128; ++i) asm volatile("" : "+r"(v[i]));
-#pragma unroll
-  for (int i = 0; i < 128; i += 8) {
-    const int4 c0 = lds128(ck_addr + i * 4), c1 = lds128(ck_addr + (i + 4) * 4);
-    const uint32_t k0 = static_cast<uint32_t>(c0.x - 512 * static_cast<int>(v[i]));
-    const uint32_t k1 = static_cast<uint32_t>(c0.y - 512 * static_cast<int>(v[i + 1]));
-    const uint32_t k2 = static_cast<uint32_t>(c0.z - 512 * static_cast<int>(v[i + 2]));
-    const uint32_t k3 = static_cast<uint32_t>(c0.w - 512 * static_cast<int>(v[i + 3]));
-    const uint32_t k4 = static_cast<uint32_t>(c1.x - 512 * static_cast<int>(v[i + 4]));
-    const uint32_t k5 = static_cast<uint32_t>(c1.y - 512 * static_cast<int>(v[i + 5]));
-    const uint32_t k6 = static_cast<uint32_t>(c1.z - 512 * static_cast<int>(v[i + 6]));
-    const uint32_t k7 = static_cast<uint32_t>(c1.w - 512 * static_cast<int>(v[i + 7]));
-    const uint32_t x = prmt_top16x2(k0, k1), y = prmt_top16x2(k2, k3);
-    const uint32_t z = prmt_top16x2(k4, k5), ww = prmt_top16x2(k6, k7);
-    uint32_t lo = __vmins2(x, y), hi = __vmaxs2(x, y);
-    uint32_t tt = __vmaxs2(A1, lo);
-    A2 = __vmins2(__vmins2(A2, tt), hi);
-    A1 = __vmins2(A1, lo);
-    lo = __vmins2(z, ww); hi = __vmaxs2(z, ww);
-    tt = __vmaxs2(B1, lo);
-    B2 = __vmins2(__vmins2(B2, tt), hi);
-    B1 = __vmins2(B1, lo);
-    if ((i & 31) == 24) asm volatile("" : "+r"(A1), "+r"(A2), "+r"(B1), "+r"(B2));
-  }
-}
-
-// Top-2 (per 16-bit lane) of the union of two sorted packed states: (X1 <= X2) U (Y1 <= Y2).
-__device__ __forceinline__ void merge_top2_s16x2(uint32_t& X1, uint32_t& X2, uint32_t Y1, uint32_t Y2) {
-  const uint32_t m2 = __vmins2(__vmaxs2(X1, Y1), __vmins2(X2, Y2));
-  X1 = __vmins2(X1, Y1);
-  X2 = m2;
-}
-
-// Two smallest coarse keys u1 <= u2 (multiset order statistics) of four packed states.
-__device__ __forceinline__ void finish_coarse(uint32_t A1, uint32_t A2, uint32_t B1, uint32_t B2, int& u1, int& u2) {
-  merge_top2_s16x2(A1, A2, B1, B2);
-  const int l1 = static_cast<int16_t>(A1 & 0xFFFFu), h1 = static_cast<int16_t>(A1 >> 16);
-  const int l2 = static_cast<int16_t>(A2 & 0xFFFFu), h2 = static_cast<int16_t>(A2 >> 16);
-  u1 = min(l1, h1);
-  u2 = min(max(l1, h1), min(l2, h2));
-}
-
-// Exact fallback for one undecided query row (rare): the warp recomputes the 256 dot products of
-// that row against the resident reference chunk straight from shared memory (both tiles are
-// SWIZZLE_128B: 16-byte chunk c of row r sits at chunk c ^ (r & 7)), 8 columns per lane with
-// dp4a, and reduces the exact top-2 packed keys across the warp.
-__device__ __forceinline__ void exact_row_from_smem(uint32_t q_tile, int qrow, uint32_t r_tile, uint32_t ck_addr,
-                                                    int lane, int& k1, int& k2) {
-  uint4 q[8];
-#pragma unroll
-  for (int c = 0; c < 8; ++c) {
-    const int4 t = lds128(q_tile + qrow * 128 + ((c ^ (qrow & 7)) << 4));
-    q[c] = make_uint4(t.x, t.y, t.z, t.w);
-  }
-  int a1 = INT_MAX, a2 = INT_MAX;
-#pragma unroll 2
-  for (int jj = 0; jj < kBN / 32; ++jj) {
-    const int col = jj * 32 + lane;
-    uint32_t dot = 0;
-#pragma unroll
-    for (int c = 0; c < 8; ++c) {
-      const int4 r = lds128(r_tile + col * 128 + ((c ^ (col & 7)) << 4));
-      dot = __dp4a(q[c].x, static_cast<uint32_t>(r.x), dot);
-      dot = __dp4a(q[c].y, static_cast<uint32_t>(r.y), dot);
-      dot = __dp4a(q[c].z, static_cast<uint32_t>(r.z), dot);
-      dot = __dp4a(q[c].w, static_cast<uint32_t>(r.w), dot);
-    }
-    int ck;
-    asm volatile("ld.shared.s32 %0, [%1];" : "=r"(ck) : "r"(ck_addr + col * 4));
-    const int key = ck - 512 * static_cast<int>(dot);
-    a2 = min(a2, max(a1, key));
-    a1 = min(a1, key);
-  }
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    const int b1 = __shfl_xor_sync(0xffffffffu, a1, o), b2 = __shfl_xor_sync(0xffffffffu, a2, o);
-    const int m2 = min(max(a1, b1), min(a2, b2));
-    a1 = min(a1, b1);
-    a2 = m2;
-  }
-  k1 = a1;
-  k2 = a2;
+  const int sr = min3i(max(min(rm[0], rm[1]), min(rm[2], rm[3])), max(rm[0], rm[1]), max(rm[2], rm[3]));
+  const int sc = min3i(max(min(cm[0], cm[1]), min(cm[2], cm[3])), max(cm[0], cm[1]), max(cm[2], cm[3]));
+  k1 = T1;  // the P minima cover every column
+  k2 = min3i(T2, sr, sc);
 }
 
 // ------------------------------------------------------------------ fused match kernel
-// One persistent CTA per SM.  A job = (reference group resident in SMEM) x (range of query
-// tiles streamed through a 4-stage ring).  Unit u = (query tile t, reference s) belongs to
-// epilogue group u % kNG; each unit is 2*cpr pieces of 128 accumulator columns.  Group g owns
-// kNB TMEM buffers and double-buffers its pieces, so the MMA of its next piece overlaps the
-// scan of the current one.
+// One persistent CTA per SM.  A job = (up to 4 references resident in SMEM) x (range of query
+// tiles streamed through a 4-stage ring).  Unit u = (query tile t, reference s), s fastest,
+// belongs to epilogue group u % 4 (with 4 resident references: group g <-> reference g, so its
+// counts accumulate in a register over the query's tiles).  Each 256-column reference chunk of
+// a unit is computed as 4 MMA pieces of 64 columns; group g owns TMEM buffers 2g, 2g+1 and its
+// own MMA warp, so the MMA of the next piece overlaps the scan of the current one, and the 4
+// groups (4 epilogue warps per SMSP) hide each other's TMEM-load and barrier latency.
+// kSimple: one 256-column chunk per reference and no (d1, i1, d2, i2) output (the search
+// path), which frees the registers of the cross-chunk merge.
+template <bool kSimple>
 __global__ void __launch_bounds__(kNumThreads, 1)
     match_kernel(const __grid_constant__ CUtensorMap qmap, const __grid_constant__ CUtensorMap rmap,
                  const MatchParams p) {
@@ -443,7 +322,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const uint32_t sbase = smem_u32(smem);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int T = p.tiles_per_q, cpr = p.cpr;
+  const int T = p.tiles_per_q, cpr = kSimple ? 1 : p.cpr;
 
   auto qfull = [&](int i) { return sbase + SmemPlan::kQFull + 8 * i; };
   auto qempty = [&](int i) { return sbase + SmemPlan::kQEmpty + 8 * i; };
@@ -452,21 +331,18 @@ __global__ void __launch_bounds__(kNumThreads, 1)
   auto tfull = [&](int i) { return sbase + SmemPlan::kTFull + 8 * i; };
   auto tempty = [&](int i) { return sbase + SmemPlan::kTEmpty + 8 * i; };
   uint32_t* tmem_ptr_smem = reinterpret_cast<uint32_t*>(smem + SmemPlan::kTmemPtr);
-  uint32_t* cnt_smem = reinterpret_cast<uint32_t*>(smem + SmemPlan::kCnt);
-  uint32_t* xch_smem = reinterpret_cast<uint32_t*>(smem + SmemPlan::kXch);
-  const bool use_coarse = p.coarse && cpr == 1 && p.mode == kModeSearch && p.nn_out == nullptr;
 
   if (threadIdx.x == 0) {
     prefetch_tmap(&qmap);
     prefetch_tmap(&rmap);
-    // query stages: freed by the MMA commit and by every epilogue warp (the exact fallback reads them)
-    for (int i = 0; i < kQStages; ++i) { mbar_init(qfull(i), 1); mbar_init(qempty(i), 4 + kEpiWarps); }
-    for (int i = 0; i < kMaxSlots; ++i) { mbar_init(rfull(i), 1); mbar_init(rempty(i), 4 + kEpiWarps); }
-    for (int i = 0; i < kTmemBufs; ++i) { mbar_init(tfull(i), 1); mbar_init(tempty(i), 4 * kSplit); }
+    // query stages are read only by the tensor core: freed by the 4 MMA warps' commits
+    for (int i = 0; i < kQStages; ++i) { mbar_init(qfull(i), 1); mbar_init(qempty(i), kNG); }
+    // reference slots: MMA operands + column keys read by every epilogue warp
+    for (int i = 0; i < kMaxSlots; ++i) { mbar_init(rfull(i), 1); mbar_init(rempty(i), kNG + kEpiWarps); }
+    for (int i = 0; i < kTmemBufs; ++i) { mbar_init(tfull(i), 1); mbar_init(tempty(i), 4); }
     fence_barrier_init();
   }
-  if (threadIdx.x < 4 * kNG * kMaxSlots) cnt_smem[threadIdx.x] = 0;
-  if (warp == kFirstMmaWarp) {  // TMEM: kTmemBufs accumulator buffers x 128 columns (all 512)
+  if (warp == kFirstMmaWarp) {  // TMEM: 8 accumulator buffers x 64 columns (all 512)
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(
                      smem_u32(tmem_ptr_smem))
                  : "memory");
@@ -482,12 +358,12 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     // ===================== TMA producer =====================
     if (lane == 0) {
       uint32_t qctr = 0;
-      uint32_t slot_use[kMaxSlots] = {0, 0, 0, 0};
+      uint32_t slot_par = 0;  // bit sl = phase parity of reference slot sl
       for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
         const Job J = decode_job(p, j);
         const int nslots = J.nr * cpr;
         for (int sl = 0; sl < nslots; ++sl) {
-          PROF_B(); mbar_wait_sleep(rempty(sl), (slot_use[sl] & 1) ^ 1); PROF_E(0);
+          PROF_B(); mbar_wait_sleep(rempty(sl), (slot_par >> sl & 1u) ^ 1); PROF_E(0);
           mbar_expect_tx(rfull(sl), kRTileBytes + kColBytes);
           const int s = sl / cpr, c = sl % cpr;
           const int64_t ref = J.ref_first + s;
@@ -495,7 +371,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
                       static_cast<int>(p.ref_map_base + ref));
           bulk_load(sbase + SmemPlan::kCol + sl * kColBytes, p.colkey + (ref * cpr + c) * kColInts, kColBytes,
                     rfull(sl));
-          ++slot_use[sl];
+          slot_par ^= 1u << sl;
         }
         const int ntiles = J.nq * T;
         for (int t = 0; t < ntiles; ++t, ++qctr) {
@@ -506,263 +382,191 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         }
       }
     }
-  } else if (warp >= kFirstMmaWarp && warp < kFirstMmaWarp + 4) {
-    // ===================== MMA issuers: 4 warps, one per SMSP, one per TMEM buffer ==============
-    // Issuing tcgen05.mma costs the issuing SMSP real throughput, and each SMSP's epilogue warps
-    // own one TMEM lane quarter, so the issue load is spread evenly: MMA warp mw owns accumulator
-    // buffer mw = (epilogue group g = mw / 2, column half h = mw % 2) and issues exactly the
-    // pieces (unit u with u % 2 == g, chunk c, half h), in order.  Whole warp, one elected lane.
-    {
-      const int mw = warp - kFirstMmaWarp;
-      // kNG == 2: buffer mw = (group mw/2, half mw%2); kNG == 4: buffer mw = group mw, both halves
-      const int my_g = kNG == 2 ? (mw >> 1) : mw;
-      const int h_lo = kNG == 2 ? (mw & 1) : 0, h_hi = kNG == 2 ? (mw & 1) : 1;
-      uint32_t qctr = 0, pc = 0;
-      uint32_t slot_use[kMaxSlots] = {0, 0, 0, 0};
-      const uint32_t dt = tmem_base + mw * kPiece;
-      for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
-        const Job J = decode_job(p, j);
-        const int nslots = J.nr * cpr;
-        const int U = J.nq * T * J.nr;
-        uint32_t ready_mask = 0;
-        int waited = 0, t = 0, s = 0, g = 0;
-        for (int u = 0; u < U; ++u) {
-          if (g == my_g) {
-            while (waited <= t) {
-              const uint32_t gq = qctr + waited;
-              PROF_B(); mbar_wait_sleep(qfull(gq % kQStages), (gq / kQStages) & 1); PROF_E(1);
-              ++waited;
+  } else if (warp < kFirstEpiWarp) {
+    // ===================== MMA issuers: warp mw serves epilogue group mw =====================
+    // Issuing tcgen05.mma costs the issuing SMSP throughput, so the 4 issuers sit on 4 SMSPs.
+    // Warp mw issues the pieces of the units u with u % 4 == mw, in order, into its group's two
+    // 64-column buffers (whole warp, one elected lane).  Every warp commits the release of every
+    // query tile (waiting for tiles it never used, so the stage phases stay in order).
+    const int mw = warp - kFirstMmaWarp;
+    uint32_t qctr = 0, pc = 0;
+    uint32_t slot_par = 0;  // bit sl = phase parity of reference slot sl
+    for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
+      const Job J = decode_job(p, j);
+      const int nslots = J.nr * cpr;
+      const int U = J.nq * T * J.nr;
+      uint32_t ready_mask = 0;
+      int waited = 0, t = 0, s = 0, g = 0;
+      for (int u = 0; u < U; ++u) {
+        if (g == mw) {
+          while (waited <= t) {
+            const uint32_t gq = qctr + waited;
+            PROF_B(); mbar_wait(qfull(gq % kQStages), (gq / kQStages) & 1); PROF_E(1);
+            ++waited;
+          }
+          const uint32_t st = (qctr + t) % kQStages;
+          const uint64_t ad = smem_desc_sw128(sbase + SmemPlan::kQ + st * kQTileBytes);
+          for (int c = 0; c < cpr; ++c) {
+            const int sl = s * cpr + c;
+            if (!(ready_mask >> sl & 1u)) {
+              PROF_B(); mbar_wait(rfull(sl), (slot_par >> sl & 1u)); PROF_E(2);
+              ready_mask |= 1u << sl;
             }
-            const uint32_t st = (qctr + t) % kQStages;
-            const uint64_t ad = smem_desc_sw128(sbase + SmemPlan::kQ + st * kQTileBytes);
-            for (int c = 0; c < cpr; ++c) {
-              const int sl = s * cpr + c;
-              if (!(ready_mask >> sl & 1u)) { PROF_B(); mbar_wait_sleep(rfull(sl), slot_use[sl] & 1); PROF_E(2); ready_mask |= 1u << sl; }
-              for (int h = h_lo; h <= h_hi; ++h) {
-                const uint64_t bd = smem_desc_sw128(sbase + SmemPlan::kR + sl * kRTileBytes) +
-                                    h * (kPiece * kDim >> 4);  // rows 128h.. of the chunk
-                PROF_B(); mbar_wait_sleep(tempty(mw), (pc & 1) ^ 1); PROF_E(0);
-                tc_fence_after();
-                mma_piece(dt, ad, bd, tfull(mw));
-                ++pc;
-              }
+            const uint64_t bd0 = smem_desc_sw128(sbase + SmemPlan::kR + sl * kRTileBytes);
+#pragma unroll 1
+            for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
+              const uint32_t buf = mw * kNB + (pc & 1);
+              PROF_B(); mbar_wait(tempty(buf), ((pc >> 1) & 1) ^ 1); PROF_E(0);
+              tc_fence_after();
+              // rows 64pp.. of the chunk: 8 SWIZZLE_128B core groups of 1024 B each
+              mma_piece(tmem_base + buf * kPiece, ad, bd0 + pp * (kPiece * kDim >> 4), tfull(buf));
+              ++pc;
             }
           }
-          if (s == J.nr - 1) {  // this warp's release of query tile t (covers all its prior MMAs)
-            if (waited <= t) {  // never touched tile t: still wait for it so the phase order holds
-              const uint32_t gq = qctr + t;
-              mbar_wait_sleep(qfull(gq % kQStages), (gq / kQStages) & 1);
-              waited = t + 1;
-            }
-            mma_commit(qempty((qctr + t) % kQStages));
-          }
-          if (++g == kNG) g = 0;
-          if (++s == J.nr) { s = 0; ++t; }
         }
-        for (int sl = 0; sl < nslots; ++sl) { mma_commit(rempty(sl)); ++slot_use[sl]; }
-        qctr += J.nq * T;
+        if (s == J.nr - 1) {  // this warp's release of query tile t (covers all its prior MMAs)
+          if (waited <= t) {  // never touched tile t: still wait for it so the phase order holds
+            const uint32_t gq = qctr + t;
+            mbar_wait(qfull(gq % kQStages), (gq / kQStages) & 1);
+            waited = t + 1;
+          }
+          mma_commit(qempty((qctr + t) % kQStages));
+        }
+        if (++g == kNG) g = 0;
+        if (++s == J.nr) { s = 0; ++t; }
       }
+      for (int sl = 0; sl < nslots; ++sl) {
+        if (!(ready_mask >> sl & 1u)) mbar_wait(rfull(sl), (slot_par >> sl & 1u));  // keep rempty phases ordered
+        mma_commit(rempty(sl));
+        slot_par ^= 1u << sl;
+      }
+      qctr += J.nq * T;
     }
   } else {
     // ===================== epilogue: TMEM -> registers -> top-2 -> ratio -> count =====================
-    const int ew = warp - kFirstEpiWarp;     // 0 .. 4*kNG*kSplit-1
-    const int g = ew / (4 * kSplit);         // epilogue group (units u with u % kNG == g)
-    const int cq = (ew >> 2) % kSplit;       // column part of every piece this warp scans
-    const int quarter = warp & 3;            // TMEM lanes 32*quarter .. +31 (hardware restriction)
-    const int fin = g * 4 + quarter;         // finaliser slot (the cq == 0 warp of this lane quarter)
-    const uint32_t pair_bar = 1 + fin;       // named barrier of the kSplit warps of (group, quarter)
-    uint32_t xc = 0;                         // exchanges done (parity selects the exchange slot)
-    const uint32_t taddr_q = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16) + cq * kCPW;
-    uint32_t mp = 0;                         // pieces consumed by this group
-    uint32_t qctr = 0;
-    uint32_t slot_use[kMaxSlots] = {0, 0, 0, 0};
+    // Each piece (64 columns) is fetched with one x64 TMEM load and its buffer released as soon
+    // as the load has landed, so the MMA of the group's next-but-one piece overlaps the scan; the
+    // 3 groups (3 epilogue warps per SMSP) hide each other's load latency.
+    const int ew = warp - kFirstEpiWarp;  // 0 .. 4*kNG-1
+    const int g = ew >> 2;                // group: units u with u % kNG == g
+    const int quarter = warp & 3;         // TMEM lanes 32*quarter .. +31 (hardware restriction)
+    const uint32_t taddr_q = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16);
     const int row_in_tile = quarter * 32 + lane;
     const int nq_ld = T * kBM;
+    const bool ratio32 = p.num2 <= 511u && p.den2 <= 511u;  // den^2 * d fits 32 bits (d <= 8,323,200)
+    uint32_t mp = 0;                      // pieces consumed by this warp (buffer + phase)
+    uint32_t slot_par = 0;                // bit sl = phase parity of reference slot sl
+    uint32_t v[64];
 
     for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
       const Job J = decode_job(p, j);
       const int nslots = J.nr * cpr;
       const int U = J.nq * T * J.nr;
-      int t = 0, s = 0, tq = 0, qi = J.q_first, ug = 0;
-      bool touched = false;
-      for (int u = 0; u < U; ++u) {
-        if (ug == g) {
-          touched = true;
-          PROF_B();
-          const int row = tq * kBM + row_in_tile;
-          const int nvalid = p.n_valid ? p.n_valid[qi] : p.n_rows;
-          const bool valid = row < nvalid && row < p.n_rows;
-          const int32_t nqv = p.nq[static_cast<int64_t>(qi) * nq_ld + row];
-          PROF_E(6);
-          int g1d = INT_MAX, g1i = -1, g2d = INT_MAX, g2i = -1;  // running exact 2-NN over chunks
-          bool pass = false;
-          uint32_t A1 = 0x7FFF7FFFu, A2 = 0x7FFF7FFFu, B1 = 0x7FFF7FFFu, B2 = 0x7FFF7FFFu;
-          if (use_coarse) {
-            const int sl = s;
-            PROF_B(); mbar_wait(rfull(sl), slot_use[sl] & 1); PROF_E(4);  // column keys have landed
+      // column keys of every slot of the job (also orders this warp's rempty arrivals)
+      PROF_B();
+      for (int sl = 0; sl < nslots; ++sl) mbar_wait(rfull(sl), slot_par >> sl & 1u);
+      PROF_E(4);
+      // own units u = g, g + kNG, ...; unit u = (tile t = u / nr, reference s = u % nr), and
+      // t = (query qi - q_first) * T + tq.  Tracked incrementally (no divisions per unit).
+      int u = g, s = g % J.nr, tq = g / J.nr, qi = J.q_first;
+      while (tq >= T) { tq -= T; ++qi; }
+      int nvalid = u < U ? min(p.n_valid ? p.n_valid[qi] : p.n_rows, p.n_rows) : 0;
+      const int32_t* nq_row = p.nq + static_cast<int64_t>(qi) * nq_ld + row_in_tile;
+      uint32_t cnt = 0;
+      while (u < U) {
+        const int row = tq * kBM + row_in_tile;
+        const bool valid = row < nvalid;
+        const int32_t nqv = valid ? nq_row[tq * kBM] : 0;
+        // the unit after this one (same group): (ns, ntq, nqi)
+        int ns = s + kNG, ntq = tq, nqi = qi;
+        while (ns >= J.nr) {
+          ns -= J.nr;
+          if (++ntq == T) { ntq = 0; ++nqi; }
+        }
+        const bool has_next = u + kNG < U;
+        int g1d = INT_MAX, g1i = -1, g2d = INT_MAX, g2i = -1;  // running exact 2-NN over chunks
+        for (int c = 0; c < cpr; ++c) {
+          const uint32_t ck = sbase + SmemPlan::kCol + (s * cpr + c) * kColBytes;
+          int R[16];
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {
-              const uint32_t buf = g * kNB + mp % kNB;
-              PROF_B(); mbar_wait(tfull(buf), (mp / kNB) & 1); PROF_E(0);
-              tc_fence_after();
-              PROF_B();
-#if TID_X128
-              scan_coarse_x128(taddr_q + buf * kPiece, sbase + SmemPlan::kCol + sl * kColBytes + h * kPiece * 4, A1,
-                               A2, B1, B2);
-#else
-              scan_coarse<kCPW>(taddr_q + buf * kPiece,
-                                sbase + SmemPlan::kCol + sl * kColBytes + (h * kPiece + cq * kCPW) * 4, A1, A2, B1, B2);
-#endif
-              PROF_E(1);
-              PROF_B();
-              tc_fence_before();
-              __syncwarp();
-              if (lane == 0) mbar_arrive(tempty(buf));  // accumulator free as soon as it is scanned
-              PROF_E(5);
-              ++mp;
-            }
-            if (kSplit > 1) {  // the kSplit warps of this lane quarter merge their states
-              uint4* x = reinterpret_cast<uint4*>(xch_smem) + (fin * 2 + (xc & 1)) * 32 * (kSplit - 1);
-              if (cq > 0) x[(cq - 1) * 32 + lane] = make_uint4(A1, A2, B1, B2);
-              named_bar(pair_bar, 32 * kSplit);
-              if (cq == 0) {
+          for (int b = 0; b < 16; ++b) R[b] = INT_MAX;
+          int T1 = INT_MAX, T2 = INT_MAX;
+#pragma unroll 1
+          for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
+            const uint32_t buf = g * kNB + (mp & 1);
+            PROF_B(); mbar_wait(tfull(buf), (mp >> 1) & 1); PROF_E(0);
+            tc_fence_after();
+            // x64 loads; the buffer is released as soon as its last load has landed
 #pragma unroll
-                for (int o = 0; o < kSplit - 1; ++o) {
-                  const uint4 r = x[o * 32 + lane];
-                  merge_top2_s16x2(A1, A2, r.x, r.y);
-                  merge_top2_s16x2(B1, B2, r.z, r.w);
-                }
-              }
-              ++xc;
-            }
-          }
-          if (use_coarse && cq == 0) {
-            const int sl = s;
-            PROF_B();
-            int u1, u2;
-            finish_coarse(A1, A2, B1, B2, u1, u2);
-            // bounds: N_R - 2S of the 1st / 2nd neighbour lies in [256 u, 256 u + 255]
-            const int64_t d1lo = static_cast<int64_t>(nqv) + 256 * static_cast<int64_t>(u1);
-            const int64_t d2lo = static_cast<int64_t>(nqv) + 256 * static_cast<int64_t>(u2);
-            const int64_t den2 = p.den2, num2 = p.num2;
-            // u == 0x7FFF only for padding columns (sentinel N_R); real keys are <= 32512
-            const bool fail_sure = (u2 >= 0x7FFF) || den2 * d1lo >= num2 * (d2lo + 255);
-            const bool pass_sure = !fail_sure && den2 * (d1lo + 255) < num2 * d2lo;
-            pass = valid && pass_sure;
-            uint32_t undecided = __ballot_sync(0xffffffffu, valid && !pass_sure && !fail_sure);
-            PROF_E(2);
-            if (undecided) {
-              PROF_B();
-              const uint32_t qt = sbase + SmemPlan::kQ + ((qctr + t) % kQStages) * kQTileBytes;
-              const uint32_t rt = sbase + SmemPlan::kR + sl * kRTileBytes;
-              const uint32_t ck = sbase + SmemPlan::kCol + sl * kColBytes;
-              while (undecided) {
-                const int l = __ffs(undecided) - 1;
-                undecided &= undecided - 1;
-                int k1, k2;
-                exact_row_from_smem(qt, quarter * 32 + l, rt, ck, lane, k1, k2);
-                if (lane == l) {
-                  const int64_t d1 = static_cast<int64_t>(nqv) + (k1 >> 8);
-                  const int64_t d2 = static_cast<int64_t>(nqv) + (k2 >> 8);
-                  pass = (k2 >> 8) < kSentinelNorm && den2 * d1 < num2 * d2;
-                }
-              }
-              PROF_E(3);
-            }
-          } else if (!use_coarse) {
-            for (int c = 0; c < cpr; ++c) {
-              const int sl = s * cpr + c;
-              mbar_wait(rfull(sl), slot_use[sl] & 1);
-              int a1 = INT_MAX, a2 = INT_MAX, b1 = INT_MAX, b2 = INT_MAX;
-#pragma unroll
-              for (int h = 0; h < 2; ++h) {
-                const uint32_t buf = g * kNB + mp % kNB;
-                mbar_wait(tfull(buf), (mp / kNB) & 1);
-                tc_fence_after();
-                scan_exact<kCPW>(taddr_q + buf * kPiece,
-                                 sbase + SmemPlan::kCol + sl * kColBytes + (h * kPiece + cq * kCPW) * 4, a1, a2, b1, b2);
+            for (int h = 0; h < kPiece / 64; ++h) {
+              tmem_ld64(taddr_q + buf * kPiece + h * 64, v);
+              tmem_wait_ld();
+              reg_fence64(v);
+              if (h == kPiece / 64 - 1) {
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(tempty(buf));
                 ++mp;
               }
-              int k1 = min(a1, b1);
-              int k2 = min(max(a1, b1), min(a2, b2));
-              if (kSplit > 1) {
-                uint4* x = reinterpret_cast<uint4*>(xch_smem) + (fin * 2 + (xc & 1)) * 32 * (kSplit - 1);
-                if (cq > 0) x[(cq - 1) * 32 + lane] = make_uint4(static_cast<uint32_t>(k1), static_cast<uint32_t>(k2), 0, 0);
-                named_bar(pair_bar, 32 * kSplit);
-                if (cq == 0) {
-#pragma unroll
-                  for (int o = 0; o < kSplit - 1; ++o) {
-                    const uint4 r = x[o * 32 + lane];
-                    const int p1 = static_cast<int>(r.x), p2 = static_cast<int>(r.y);
-                    const int m2 = min(max(k1, p1), min(k2, p2));
-                    k1 = min(k1, p1);
-                    k2 = m2;
-                  }
-                }
-                ++xc;
-              }
-              const int c1d = k1 >> 8, c1i = (k1 & 255) + c * kBN;
-              const int c2d = k2 >> 8, c2i = (k2 & 255) + c * kBN;
-              // merge into the running 2-NN; earlier chunks win ties (lower index)
-              if (c1d < g1d) {
-                if (c2d < g1d) { g2d = c2d; g2i = c2i; } else { g2d = g1d; g2i = g1i; }
-                g1d = c1d; g1i = c1i;
-              } else if (c1d < g2d) {
-                g2d = c1d; g2i = c1i;
-              }
-            }
-            // ratio test in exact integers: den^2 * d1 < num^2 * d2
-            const bool real1 = g1d < kSentinelNorm, real2 = g2d < kSentinelNorm;
-            const int64_t d1 = static_cast<int64_t>(nqv) + g1d;
-            const int64_t d2 = static_cast<int64_t>(nqv) + g2d;
-            pass = valid && real2 &&
-                   static_cast<uint64_t>(p.den2) * static_cast<uint64_t>(d1) <
-                       static_cast<uint64_t>(p.num2) * static_cast<uint64_t>(d2);
-            if (cq == 0 && p.nn_out != nullptr && row < p.n_rows) {
-              int4 o;
-              o.x = (valid && real1) ? static_cast<int>(d1) : -1; o.y = (valid && real1) ? g1i : -1;
-              o.z = (valid && real2) ? static_cast<int>(d2) : -1; o.w = (valid && real2) ? g2i : -1;
-              reinterpret_cast<int4*>(p.nn_out)[static_cast<int64_t>(qi) * p.n_rows + row] = o;
+              PROF_B();
+              scan32_regs(v, ck + (pp * kPiece + h * 64) * 4, R, T1, T2);
+              scan32_regs(v + 32, ck + (pp * kPiece + h * 64 + 32) * 4, R, T1, T2);
+              PROF_E(1);
             }
           }
-          const uint32_t bal = __ballot_sync(0xffffffffu, pass);
-          if (lane == 0 && cq == 0) {
-            uint32_t& acc = cnt_smem[fin * kMaxSlots + s];
-            acc += __popc(bal);
-            // flush when this group holds no further unit of this (query, reference) pair
-            if (tq == T - 1 || u + J.nr >= U || J.nr % kNG != 0) {
-              if (acc) {
-                const int64_t ci = (p.mode == kModeVerify)
-                                       ? qi : static_cast<int64_t>(qi) * p.ldc + p.col0 + J.ref_first + s;
-                atomicAdd(p.counts + ci, acc);
-              }
-              acc = 0;
-            }
+          PROF_B();
+          int k1, k2;
+          finish_partition(R, T1, T2, k1, k2);
+          const int c1d = k1 >> 8, c1i = (k1 & 255) + c * kBN;
+          const int c2d = k2 >> 8, c2i = (k2 & 255) + c * kBN;
+          if (kSimple || c == 0) {
+            g1d = c1d; g1i = c1i; g2d = c2d; g2i = c2i;
+          } else if (c1d < g1d) {  // merge into the running 2-NN; earlier chunks win ties (lower index)
+            if (c2d < g1d) { g2d = c2d; g2i = c2i; } else { g2d = g1d; g2i = g1i; }
+            g1d = c1d; g1i = c1i;
+          } else if (c1d < g2d) {
+            g2d = c1d; g2i = c1i;
           }
+          PROF_E(2);
         }
-        if (s == J.nr - 1) {  // this warp is done with query tile t (fallback reads it)
-          const uint32_t gq = qctr + t;
-          // a warp with no unit in tile t must not arrive before tile t has landed, or its
-          // arrival would count towards the stage's previous phase
-          if (!touched) mbar_wait(qfull(gq % kQStages), (gq / kQStages) & 1);
-          touched = false;
-          __syncwarp();
-          if (lane == 0) mbar_arrive(qempty(gq % kQStages));
+        // ratio test in exact integers: den^2 * d1 < num^2 * d2
+        const bool real1 = g1d < kSentinelNorm, real2 = g2d < kSentinelNorm;
+        bool pass;
+        if (ratio32) {
+          const uint32_t d1 = static_cast<uint32_t>(nqv + g1d), d2 = static_cast<uint32_t>(nqv + g2d);
+          pass = p.den2 * d1 < p.num2 * d2;
+        } else {
+          const uint64_t d1 = static_cast<uint64_t>(static_cast<int64_t>(nqv) + g1d);
+          const uint64_t d2 = static_cast<uint64_t>(static_cast<int64_t>(nqv) + g2d);
+          pass = static_cast<uint64_t>(p.den2) * d1 < static_cast<uint64_t>(p.num2) * d2;
         }
-        if (++ug == kNG) ug = 0;
-        if (++s == J.nr) {
-          s = 0; ++t;
-          if (++tq == T) { tq = 0; ++qi; }
+        pass = pass && valid && real2;
+        cnt += __popc(__ballot_sync(0xffffffffu, pass));
+        if (!kSimple && p.nn_out != nullptr && row < p.n_rows) {
+          int4 o;
+          o.x = (valid && real1) ? nqv + g1d : -1; o.y = (valid && real1) ? g1i : -1;
+          o.z = (valid && real2) ? nqv + g2d : -1; o.w = (valid && real2) ? g2i : -1;
+          reinterpret_cast<int4*>(p.nn_out)[static_cast<int64_t>(qi) * p.n_rows + row] = o;
+        }
+        // flush the count when the group's next unit is another (query, reference) pair
+        if (!has_next || ns != s || nqi != qi) {
+          if (lane == 0 && cnt) {
+            const int64_t ci = (p.mode == kModeVerify) ? qi : static_cast<int64_t>(qi) * p.ldc + p.col0 + J.ref_first + s;
+            atomicAdd(p.counts + ci, cnt);
+          }
+          cnt = 0;
+        }
+        u += kNG; s = ns; tq = ntq;
+        if (nqi != qi && has_next) {
+          qi = nqi;
+          nvalid = min(p.n_valid ? p.n_valid[qi] : p.n_rows, p.n_rows);
+          nq_row = p.nq + static_cast<int64_t>(qi) * nq_ld + row_in_tile;
         }
       }
       __syncwarp();
       if (lane == 0)
         for (int sl = 0; sl < nslots; ++sl) mbar_arrive(rempty(sl));
-      for (int sl = 0; sl < nslots; ++sl) ++slot_use[sl];
-      qctr += J.nq * T;
+      slot_par ^= (1u << nslots) - 1u;
     }
   }
 
@@ -781,12 +585,19 @@ extern "C" int tid_debug_read_prof(void* host, size_t bytes) {
 }
 #endif
 
+
 cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap, int grid,
                          cudaStream_t s) {
-  cudaError_t e = cudaFuncSetAttribute(match_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+  cudaError_t e = cudaFuncSetAttribute(match_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(SmemPlan::kAlloc));
   if (e != cudaSuccess) return e;
-  match_kernel<<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, p);
+  e = cudaFuncSetAttribute(match_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           static_cast<int>(SmemPlan::kAlloc));
+  if (e != cudaSuccess) return e;
+  if (p.cpr == 1 && p.nn_out == nullptr)
+    match_kernel<true><<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, p);
+  else
+    match_kernel<false><<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, p);
   return cudaGetLastError();
 }
 

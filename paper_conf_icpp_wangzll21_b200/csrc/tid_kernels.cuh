@@ -4,7 +4,8 @@
 //   ref_prep_kernel    a1: zero padded reference rows, squared norms N_R -> packed column keys
 //   query_prep_kernel  a2: squared norms N_Q per query row
 //   match_kernel       a3+a4+a5: TMA -> tcgen05.mma.kind::i8 (u8 x u8 -> s32, TMEM) ->
-//                      exact top-2 epilogue in registers -> integer ratio test -> count
+//                      exact two-partition top-2 epilogue in registers -> integer ratio
+//                      test -> count
 //   topk_kernel        a6: per-(query, segment) top-k of the count matrix
 //   merge_kernel       a6/a9: merge ranked candidate lists (segments or shards)
 //
@@ -23,19 +24,19 @@ constexpr int kBN = 256;           // reference keypoints per chunk (MMA N, TMEM
 constexpr int kQStages = 4;        // query-tile ring
 constexpr int kMaxSlots = 4;       // resident reference chunks per CTA
 #ifndef TID_NG
-#define TID_NG 2
+#define TID_NG 3
 #endif
-constexpr int kNG = TID_NG;                    // epilogue groups (2 or 4), 4 warps each
-constexpr int kPiece = 128;                    // accumulator columns per MMA piece (MMA N)
-constexpr int kTmemBufs = 512 / kPiece;        // 4 TMEM buffers of 128 columns
-constexpr int kNB = kTmemBufs / kNG;           // buffers per epilogue group
-#ifndef TID_SPLIT
-#define TID_SPLIT 1
+#ifndef TID_PIECE
+#define TID_PIECE 64
 #endif
-constexpr int kSplit = TID_SPLIT;              // epilogue warps per (group, TMEM lane quarter)
-constexpr int kCPW = kPiece / kSplit;          // accumulator columns of each piece scanned per warp
-constexpr int kEpiWarps = 4 * kNG * kSplit;
-constexpr int kNumThreads = 32 * (5 + kEpiWarps);  // w0 TMA, w1..w4 MMA, w5.. epilogue
+constexpr int kNG = TID_NG;                    // epilogue groups of 4 warps (one per TMEM lane quarter)
+constexpr int kPiece = TID_PIECE;              // accumulator columns per MMA piece (MMA N)
+constexpr int kNB = 2;                         // TMEM buffers per group (double buffered)
+constexpr int kTmemBufs = kNG * kNB;           // 6 buffers of 64 columns (384 of the 512 allocated)
+static_assert(kTmemBufs * kPiece <= 512, "TMEM has 512 columns");
+constexpr int kPiecesPerChunk = kBN / kPiece;  // 4 pieces per 256-column reference chunk
+constexpr int kEpiWarps = 4 * kNG;             // 12 epilogue warps, 3 per SMSP
+constexpr int kNumThreads = 32 * (1 + kNG + kEpiWarps);  // w0 TMA, w1..w3 MMA (one per group), w4.. epilogue
 constexpr uint32_t kQTileBytes = kBM * kDim;   // 16 KiB
 constexpr uint32_t kRTileBytes = kBN * kDim;   // 32 KiB
 constexpr int kColInts = kBN;                  // per chunk: 256 packed column keys
@@ -46,8 +47,7 @@ constexpr int32_t kSentinelNorm = (1 << 23) - 1;  // > 128*255^2: padded columns
 //   colkey[i] = N_R[i] * 256 + i   (i = index within the chunk).
 // The epilogue forms key = colkey - 512 * S = 256 * (N_R - 2 q.r) + i with one IMAD, which
 // orders exactly like (d_ji, i) for a fixed query row (Alg. 1 step 4 + lowest-index
-// tie-break).  Its top 16 bits (arithmetic) are floor((N_R - 2 q.r) / 256): the coarse key
-// of the search fast path, packed two per register with one PRMT.
+// tie-break); keys are unique within a chunk, so the two smallest keys give (d1, i1, d2, i2).
 
 enum : int { kModeSearch = 0, kModeVerify = 1 };
 
@@ -71,7 +71,6 @@ struct MatchParams {
   int64_t col0;
   int32_t* nn_out;           // verify: [num_q][n_rows][4] or null
   uint32_t num2, den2;       // ratio^2 = num2/den2
-  int32_t coarse;            // 1: 16-bit packed top-2 with exact fallback (search, cpr == 1)
 };
 
 struct RefPrepParams {

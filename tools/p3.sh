@@ -1,0 +1,4 @@
+# ncu full capture of the match kernel on a 20k-reference search (1 GPU)
+mkdir -p gpurun_out
+TAG=${1:-p3}
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:match_kernel -s 1 -c 1 -o gpurun_out/${TAG}_match python tools/run_search.py 20000 256 1 > gpurun_out/${TAG}_ncu.log 2>&1
