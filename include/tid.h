@@ -59,7 +59,9 @@ typedef struct {
   uint32_t ratio_num;          /* ratio threshold num/den, each 1..65535 (0.8 = 4/5)   */
   uint32_t ratio_den;
   uint64_t hbm_budget_bytes;   /* reference descriptor bytes kept resident in HBM (level-1 cache,
-                                  §6.1); 0 = auto (free HBM minus 8 GiB workspace)      */
+                                  §6.1); 0 = auto (free HBM minus 8 GiB workspace).
+                                  Each resident reference additionally holds ref_kp*32 bytes of
+                                  norm-term digits and ceil(ref_kp/256) KiB of column terms.      */
   uint64_t host_budget_bytes;  /* pinned host tier capacity in bytes (level-2 cache); 0 = none    */
   int64_t  id_base;            /* global id of this rank's first reference (shard offset)         */
   int32_t  rank;               /* this process's rank; 0 when world_size == 1                     */

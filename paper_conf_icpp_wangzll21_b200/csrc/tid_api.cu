@@ -154,6 +154,22 @@ tid_status make_map(CUtensorMap* map, const void* base, int64_t count, int64_t r
   return TID_OK;
 }
 
+// u8 norm-term digits [count][rows][32] -> 3-D map with box {32 B, 256, 1}, SWIZZLE_32B.
+tid_status make_xmap(CUtensorMap* map, const void* base, int64_t count, int64_t rows) {
+  PFN_encodeTiled_t fn = encode_fn();
+  if (!fn) return fail(TID_ECUDA, "cuTensorMapEncodeTiled entry point unavailable");
+  cuuint64_t dims[3] = {static_cast<cuuint64_t>(kXDim), static_cast<cuuint64_t>(rows),
+                        static_cast<cuuint64_t>(std::max<int64_t>(count, 1))};
+  cuuint64_t strides[2] = {static_cast<cuuint64_t>(kXDim), static_cast<cuuint64_t>(rows * kXDim)};
+  cuuint32_t box[3] = {static_cast<cuuint32_t>(kXDim), static_cast<cuuint32_t>(kBN), 1};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, 3, const_cast<void*>(base), dims, strides, box, estr,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(TID_ECUDA, "cuTensorMapEncodeTiled (norm digits) failed (%d)", static_cast<int>(r));
+  return TID_OK;
+}
+
 bool is_device_ptr(const void* p) {
   if (!p) return false;
   cudaPointerAttributes a;
@@ -172,7 +188,8 @@ inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 struct Segment {
   bool on_host = false;
   uint8_t* desc = nullptr;    // [cap][m][128]: device (HBM) or pinned host
-  int32_t* colkey = nullptr;  // device, HBM segments only: [cap][cpr][256] packed column keys
+  int32_t* colkey = nullptr;  // device, HBM segments only: [cap][cpr][256] column terms W (search)
+  uint8_t* extra = nullptr;   // device, HBM segments only: [cap][m][32] norm-term digits (search MMA)
   int64_t cap = 0, count = 0, first = 0;
   std::vector<int32_t> kp;    // keypoint count per reference (0 = deleted / empty)
 };
@@ -185,6 +202,7 @@ struct tid_index {
   int num_sms = 148;
   int cpr = 1;                    // chunks per reference = ceil(ref_kp / 256)
   int64_t ref_bytes = 0;          // bytes per stored reference
+  int64_t hbm_ref_bytes = 0;      // HBM bytes per resident reference (descriptors + norm digits + column terms)
   uint64_t hbm_budget = 0, host_budget = 0;
   std::vector<Segment> segs;      // id order; HBM and host segments may interleave (FIFO policy)
   int64_t n_hbm = 0, n_host = 0;  // references held in each tier
@@ -197,7 +215,8 @@ struct tid_index {
   // workspaces
   DevBuf ws_q, ws_nq, ws_nvalid, ws_counts, ws_cand, ws_keys, ws_gather, ws_ids, ws_cnts, ws_r, ws_colkey, ws_nn,
       ws_kp, ws_mr;
-  DevBuf stage_desc[2], stage_colkey[2], stage_kp[2];
+  DevBuf stage_desc[2], stage_colkey[2], stage_kp[2], stage_extra[2];
+  DevBuf ws_qs;                   // shifted queries q' = q ^ 0x80 (search)
   int64_t host_chunk = 0;
   tid_tuning tune{};
   ncclComm_t comm = nullptr;
@@ -255,15 +274,20 @@ void plan_search(const tid_index* idx, int64_t n_refs, int64_t B, int T, int* G_
   *qpj_out = qpj;
 }
 
-tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const uint8_t* rbase, int64_t map_count,
-                               int64_t ref_map_base, const int32_t* colkey, int64_t n_refs, int64_t B, int32_t n,
+tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const uint8_t* rbase, const uint8_t* xbase,
+                               int64_t map_count, int64_t ref_map_base, const int32_t* colkey, int64_t n_refs, int64_t B,
+                               int32_t n,
                                int T, const int32_t* nvalid, uint32_t* counts, int64_t ldc, int64_t col0,
                                cudaStream_t s) {
   if (n_refs <= 0) return TID_OK;
-  CUtensorMap rmap;
+  CUtensorMap rmap, xmap;
   TRY(make_map(&rmap, rbase, map_count, idx->cfg.ref_kp, kBN));
+  TRY(make_xmap(&xmap, xbase, map_count, idx->cfg.ref_kp));
   MatchParams p{};
   p.mode = kModeSearch;
+  p.qs = idx->ws_qs.as<uint8_t>();
+  p.rdesc = rbase;
+  p.m = idx->cfg.ref_kp;
   int G, qpj;
   plan_search(idx, n_refs, B, T, &G, &qpj);
   p.refs_per_job = G;
@@ -301,7 +325,7 @@ tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const ui
     ++idx->prof_used;
     CU(cudaEventRecord(e0, s));
   }
-  cudaError_t e = launch_match(p, qmap, rmap, grid, s);
+  cudaError_t e = launch_match(p, qmap, rmap, &xmap, grid, s);
   if (e != cudaSuccess) return fail(TID_ECUDA, "match kernel launch: %s", cudaGetErrorString(e));
   if (idx->prof) {
     CU(cudaEventRecord(e1, s));
@@ -317,15 +341,16 @@ tid_status run_counts(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, 
   const int T = static_cast<int>(ceil_div(n, kBM));
   const int64_t R = idx->n_hbm + idx->n_host;
   TRY(idx->ws_nq.ensure(static_cast<size_t>(B) * T * kBM * 4, "query norms"));
-  launch_query_prep(dq, B, n, T, idx->ws_nq.as<int32_t>(), s);
+  TRY(idx->ws_qs.ensure(static_cast<size_t>(B) * n * kDim, "shifted queries"));
+  launch_query_prep(dq, B, n, T, idx->ws_nq.as<int32_t>(), idx->ws_qs.as<uint8_t>(), s);
   count_kernel(idx);
   CU(cudaMemsetAsync(counts, 0, static_cast<size_t>(B) * R * 4, s));
   CUtensorMap qmap;
-  TRY(make_map(&qmap, dq, B, n, kBM));
+  TRY(make_map(&qmap, idx->ws_qs.p, B, n, kBM));
   // level 1: HBM-resident segments
   for (const Segment& sg : idx->segs)
     if (!sg.on_host && sg.count > 0)
-      TRY(launch_search_range(idx, qmap, sg.desc, sg.cap, 0, sg.colkey, sg.count, B, n, T, nvalid, counts, R, sg.first,
+      TRY(launch_search_range(idx, qmap, sg.desc, sg.extra, sg.cap, 0, sg.colkey, sg.count, B, n, T, nvalid, counts, R, sg.first,
                               s));
   // level 2: pinned host tier, streamed through two HBM staging buffers on the copy stream
   if (idx->n_host > 0) {
@@ -335,6 +360,7 @@ tid_status run_counts(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, 
       TRY(idx->stage_desc[b].ensure(static_cast<size_t>(chunk * rb), "host-tier staging"));
       TRY(idx->stage_colkey[b].ensure(static_cast<size_t>(chunk) * idx->cpr * kColBytes, "staging keys"));
       TRY(idx->stage_kp[b].ensure(static_cast<size_t>(chunk) * 4, "staging kp"));
+      TRY(idx->stage_extra[b].ensure(static_cast<size_t>(chunk) * idx->cfg.ref_kp * kXDim, "staging norm digits"));
     }
     // the copy stream must not overwrite staging buffers still read by a previous call
     CU(cudaEventRecord(idx->ev_free[0], s));
@@ -367,12 +393,14 @@ tid_status run_counts(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, 
       rp.src = nullptr;
       rp.kp = idx->stage_kp[b].as<int32_t>();
       rp.colkey = idx->stage_colkey[b].as<int32_t>();
+      rp.extra = idx->stage_extra[b].as<uint8_t>();
       rp.count = pc.cnt;
       rp.m = idx->cfg.ref_kp;
       rp.cpr = idx->cpr;
       launch_ref_prep(rp, s);
       count_kernel(idx);
-      TRY(launch_search_range(idx, qmap, idx->stage_desc[b].as<uint8_t>(), chunk, 0, rp.colkey, pc.cnt, B, n, T,
+      TRY(launch_search_range(idx, qmap, idx->stage_desc[b].as<uint8_t>(), rp.extra, chunk, 0, rp.colkey, pc.cnt, B,
+                              n, T,
                               nvalid, counts, R, pc.sg->first + pc.off, s));
       CU(cudaEventRecord(idx->ev_free[b], s));
     }
@@ -396,12 +424,15 @@ tid_status alloc_segment(tid_index* idx, bool on_host, int64_t cap, Segment* out
   } else {
     cudaError_t e1 = cudaMalloc(&sg.desc, static_cast<size_t>(cap * rb));
     cudaError_t e2 = e1 == cudaSuccess ? cudaMalloc(&sg.colkey, static_cast<size_t>(cap) * idx->cpr * kColBytes) : e1;
-    if (e1 != cudaSuccess || e2 != cudaSuccess) {
+    cudaError_t e3 =
+        e2 == cudaSuccess ? cudaMalloc(&sg.extra, static_cast<size_t>(cap) * idx->cfg.ref_kp * kXDim) : e2;
+    if (e1 != cudaSuccess || e2 != cudaSuccess || e3 != cudaSuccess) {
       cudaGetLastError();
       if (sg.desc) cudaFree(sg.desc);
+      if (sg.colkey) cudaFree(sg.colkey);
       return fail(TID_ENOMEM, "HBM arena allocation of %lld references failed", static_cast<long long>(cap));
     }
-    idx->hbm_alloc += cap * rb + cap * idx->cpr * kColBytes;
+    idx->hbm_alloc += cap * idx->hbm_ref_bytes;
   }
   *out = std::move(sg);
   return TID_OK;
@@ -414,10 +445,12 @@ void free_segment(tid_index* idx, Segment& sg) {
   } else {
     if (sg.desc) cudaFree(sg.desc);
     if (sg.colkey) cudaFree(sg.colkey);
-    idx->hbm_alloc -= sg.cap * idx->ref_bytes + sg.cap * idx->cpr * kColBytes;
+    if (sg.extra) cudaFree(sg.extra);
+    idx->hbm_alloc -= sg.cap * idx->hbm_ref_bytes;
   }
   sg.desc = nullptr;
   sg.colkey = nullptr;
+  sg.extra = nullptr;
 }
 
 // Ingest `take` references (host or device `src`, kp_host per reference) into HBM segment sg at
@@ -432,6 +465,7 @@ tid_status ingest_hbm(tid_index* idx, Segment& sg, int64_t pos, const uint8_t* s
   rp.cpr = idx->cpr;
   rp.count = take;
   rp.colkey = sg.colkey + pos * idx->cpr * kColInts;
+  rp.extra = sg.extra + pos * idx->cfg.ref_kp * kXDim;
   if (src_dev) {
     rp.src = src;
   } else {
@@ -567,10 +601,15 @@ tid_status tid_index_create(const tid_config* cfg, tid_index** out) {
   idx->num_sms = prop.multiProcessorCount;
   idx->cpr = static_cast<int>(ceil_div(cfg->ref_kp, kBN));
   idx->ref_bytes = static_cast<int64_t>(cfg->ref_kp) * kDim;
+  idx->hbm_ref_bytes = idx->ref_bytes + static_cast<int64_t>(cfg->ref_kp) * kXDim + static_cast<int64_t>(idx->cpr) * kColBytes;
   size_t free_b = 0, total_b = 0;
   cudaMemGetInfo(&free_b, &total_b);
   const uint64_t reserve = 8ull << 30;
-  idx->hbm_budget = cfg->hbm_budget_bytes ? cfg->hbm_budget_bytes : (free_b > reserve ? free_b - reserve : free_b / 2);
+  // the budget counts descriptor bytes; each resident reference also holds its norm digits and
+  // column terms (hbm_ref_bytes - ref_bytes), which the automatic budget leaves room for
+  const uint64_t avail = free_b > reserve ? free_b - reserve : free_b / 2;
+  idx->hbm_budget = cfg->hbm_budget_bytes ? cfg->hbm_budget_bytes
+                                          : avail / static_cast<uint64_t>(idx->hbm_ref_bytes) * idx->ref_bytes;
   idx->host_budget = cfg->host_budget_bytes;
   idx->host_chunk = 16384;
   cudaError_t e = cudaStreamCreateWithFlags(&idx->copy_stream, cudaStreamNonBlocking);
@@ -609,7 +648,8 @@ tid_status tid_index_destroy(tid_index* idx) {
   DevBuf* bufs[] = {&idx->ws_q, &idx->ws_nq, &idx->ws_nvalid, &idx->ws_counts, &idx->ws_cand, &idx->ws_keys,
                     &idx->ws_gather, &idx->ws_ids, &idx->ws_cnts, &idx->ws_r, &idx->ws_colkey, &idx->ws_nn,
                     &idx->ws_kp, &idx->ws_mr, &idx->stage_desc[0], &idx->stage_desc[1], &idx->stage_colkey[0],
-                    &idx->stage_colkey[1], &idx->stage_kp[0], &idx->stage_kp[1]};
+                    &idx->stage_colkey[1], &idx->stage_kp[0], &idx->stage_kp[1], &idx->stage_extra[0],
+                    &idx->stage_extra[1], &idx->ws_qs};
   for (DevBuf* b : bufs) b->release();
   for (auto& pr : idx->prof_ev) { cudaEventDestroy(pr.first); cudaEventDestroy(pr.second); }
   for (int b = 0; b < 2; ++b) {
@@ -735,6 +775,7 @@ tid_status tid_delete_references(tid_index* idx, const int64_t* local_ids, int64
       CU(cudaMemcpy(idx->ws_kp.p, &zero, 4, cudaMemcpyHostToDevice));
       rp.kp = idx->ws_kp.as<int32_t>();
       rp.colkey = sg->colkey + off * idx->cpr * kColInts;
+      rp.extra = sg->extra + off * idx->cfg.ref_kp * kXDim;
       rp.count = 1;
       rp.m = idx->cfg.ref_kp;
       rp.cpr = idx->cpr;
@@ -980,7 +1021,7 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
   launch_ref_prep(rp, s);
   count_kernel(idx);
   TRY(idx->ws_nq.ensure(static_cast<size_t>(P) * T * kBM * 4, "query norms"));
-  launch_query_prep(dq, P, n, T, idx->ws_nq.as<int32_t>(), s);
+  launch_query_prep(dq, P, n, T, idx->ws_nq.as<int32_t>(), nullptr, s);
   count_kernel(idx);
   const bool dev_counts = is_device_ptr(counts_out);
   TRY(idx->ws_counts.ensure(static_cast<size_t>(P) * 4, "pair counts"));
@@ -1035,7 +1076,7 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
     ++idx->prof_used;
     CU(cudaEventRecord(e0, s));
   }
-  cudaError_t e = launch_match(p, qmap, rmap, grid, s);
+  cudaError_t e = launch_match(p, qmap, rmap, nullptr, grid, s);
   if (e != cudaSuccess) return fail(TID_ECUDA, "match kernel launch: %s", cudaGetErrorString(e));
   if (idx->prof) {
     CU(cudaEventRecord(e1, s));

@@ -85,12 +85,27 @@ __device__ __forceinline__ uint64_t smem_desc_sw128(uint32_t addr) {
   return d;
 }
 
-// Instruction descriptor: kind::i8, A = u8, B = u8, D = s32, K-major A/B, M = 128, N = 128.
-constexpr uint32_t kIdescI8 = (2u << 4)                       // D format S32
-                              | (0u << 7) | (0u << 10)        // A, B unsigned 8-bit
-                              | (0u << 15) | (0u << 16)       // A, B K-major
-                              | (uint32_t(kPiece >> 3) << 17) // N >> 3
-                              | (uint32_t(kBM >> 4) << 24);   // M >> 4
+// K-major, SWIZZLE_32B descriptor (32-byte rows, 8-row groups 256 B apart): the norm-term tiles.
+__device__ __forceinline__ uint64_t smem_desc_sw32(uint32_t addr) {
+  uint64_t d = 0;
+  d |= static_cast<uint64_t>((addr & 0x3FFFF) >> 4);
+  d |= static_cast<uint64_t>(1) << 16;
+  d |= static_cast<uint64_t>(256 >> 4) << 32;           // SBO = 256 B
+  d |= static_cast<uint64_t>(1) << 46;
+  d |= static_cast<uint64_t>(6) << 61;                  // layout: SWIZZLE_32B
+  return d;
+}
+
+// Instruction descriptor: kind::i8, D = s32, K-major A/B, M = 128, N = kPiece; A/B signedness.
+constexpr uint32_t idesc_i8(bool a_signed, bool b_signed) {
+  return (2u << 4)                                      // D format S32
+         | (uint32_t(a_signed) << 7) | (uint32_t(b_signed) << 10)
+         | (0u << 15) | (0u << 16)                      // A, B K-major
+         | (uint32_t(kPiece >> 3) << 17)                // N >> 3
+         | (uint32_t(kBM >> 4) << 24);                  // M >> 4
+}
+constexpr uint32_t kIdescI8 = idesc_i8(false, false);   // verify: u8 x u8
+constexpr uint32_t kIdescFold = idesc_i8(true, false);  // search: q' (s8) x r (u8)
 
 // Issued by the whole (converged) MMA warp: elect.sync picks one lane, so the descriptors stay in
 // uniform registers and ptxas emits a bare UTCIMMA (no per-lane broadcast loop).
@@ -105,6 +120,7 @@ __device__ __forceinline__ void mma_i8(uint32_t tmem_d, uint64_t adesc, uint64_t
 }
 // One accumulator piece: D = A * B over K = 128 bytes as four K = 32 MMAs (advancing both
 // SWIZZLE_128B descriptors by 32 B = 2 units) + commit to `bar`, from a single elected lane.
+template <uint32_t kIdesc>
 __device__ __forceinline__ void mma_piece(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t bar) {
   asm volatile(
       "{\n\t.reg .pred e, f, t;\n\t.reg .b64 a1, a2, a3, b1, b2, b3;\n\t"
@@ -117,11 +133,27 @@ __device__ __forceinline__ void mma_piece(uint32_t tmem_d, uint64_t adesc, uint6
       "@e tcgen05.mma.cta_group::1.kind::i8 [%0], a1, b1, %3, t;\n\t"
       "@e tcgen05.mma.cta_group::1.kind::i8 [%0], a2, b2, %3, t;\n\t"
       "@e tcgen05.mma.cta_group::1.kind::i8 [%0], a3, b3, %3, t;\n\t"
-#ifdef TID_FAKE_FOLD
-      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], a3, b3, %3, t;\n\t"
-#endif
       "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%4];\n\t}" ::"r"(tmem_d),
-      "l"(adesc), "l"(bdesc), "r"(kIdescI8), "r"(bar)
+      "l"(adesc), "l"(bdesc), "r"(kIdesc), "r"(bar)
+      : "memory");
+}
+// Search piece: the four q'.r K-steps, then the norm-term K-step (u8 x u8: D += a . digits(E)).
+__device__ __forceinline__ void mma_piece_fold(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint64_t axdesc,
+                                               uint64_t bxdesc, uint32_t bar) {
+  asm volatile(
+      "{\n\t.reg .pred e, f, t;\n\t.reg .b64 a1, a2, a3, b1, b2, b3;\n\t"
+      "setp.ne.b32 f, 0, 0;\n\t"
+      "setp.eq.b32 t, 0, 0;\n\t"
+      "add.s64 a1, %1, 2;\n\tadd.s64 a2, %1, 4;\n\tadd.s64 a3, %1, 6;\n\t"
+      "add.s64 b1, %2, 2;\n\tadd.s64 b2, %2, 4;\n\tadd.s64 b3, %2, 6;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %5, f;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], a1, b1, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], a2, b2, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], a3, b3, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], %3, %4, %6, t;\n\t"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%7];\n\t}" ::"r"(tmem_d),
+      "l"(adesc), "l"(bdesc), "l"(axdesc), "l"(bxdesc), "r"(kIdescFold), "r"(kIdescI8), "r"(bar)
       : "memory");
 }
 
@@ -209,7 +241,9 @@ static_assert(kNB == 2 && kNumThreads <= 512, "at most 16 warps: >= 128 register
 struct SmemPlan {
   static constexpr uint32_t kR = 0;                                        // kMaxSlots x 32 KiB
   static constexpr uint32_t kQ = kR + kMaxSlots * kRTileBytes;             // kQStages x 16 KiB
-  static constexpr uint32_t kCol = kQ + kQStages * kQTileBytes;            // kMaxSlots x 1 KiB
+  static constexpr uint32_t kX = kQ + kQStages * kQTileBytes;              // kMaxSlots x 8 KiB norm-term tiles
+  static constexpr uint32_t kAx = kX + kMaxSlots * kXTileBytes;            // 4 KiB constant norm-term operand
+  static constexpr uint32_t kCol = kAx + kBM * kXDim;                      // kMaxSlots x 1 KiB
   static constexpr uint32_t kBar = kCol + kMaxSlots * kColBytes;           // mbarriers
   static constexpr uint32_t kQFull = kBar;
   static constexpr uint32_t kQEmpty = kQFull + 8 * kQStages;
@@ -270,15 +304,11 @@ __device__ __forceinline__ void scan32_regs(const uint32_t* v, uint32_t ck_addr,
   int k[32];
 #pragma unroll
   for (int i = 0; i < 32; i += 4) {
-#ifdef TID_FAKE_FOLD  // timing experiment only: keys straight from TMEM (wrong results)
-    k[i] = v[i]; k[i + 1] = v[i + 1]; k[i + 2] = v[i + 2]; k[i + 3] = v[i + 3];
-#else
     const int4 c4 = lds128(ck_addr + i * 4);
     k[i] = c4.x - 512 * static_cast<int>(v[i]);
     k[i + 1] = c4.y - 512 * static_cast<int>(v[i + 1]);
     k[i + 2] = c4.z - 512 * static_cast<int>(v[i + 2]);
     k[i + 3] = c4.w - 512 * static_cast<int>(v[i + 3]);
-#endif
   }
   const int x = min16(k), y = min16(k + 16);
 #pragma unroll
@@ -304,6 +334,85 @@ __device__ __forceinline__ void finish_partition(const int (&R)[16], int T1, int
   k2 = min3i(T2, sr, sc);
 }
 
+// Search path: the same two-partition scan on the folded values X (TMEM, no column keys), for
+// the two LARGEST X.  `lim` = real columns among these 32 (padding is masked to INT_MIN).
+__device__ __forceinline__ int max3i(int a, int b, int c) { return __vimax3_s32(a, b, c); }
+__device__ __forceinline__ int max16(const int* k) {
+  const int a = max3i(k[0], k[1], k[2]), b = max3i(k[3], k[4], k[5]), c = max3i(k[6], k[7], k[8]);
+  const int d = max3i(k[9], k[10], k[11]), e = max3i(k[12], k[13], k[14]);
+  return max(max3i(a, b, c), max3i(d, e, k[15]));
+}
+__device__ __forceinline__ void scan32_fold(const uint32_t* v, int lim, int (&R)[16], int& T1, int& T2) {
+  int k[32];
+  if (lim >= 32) {
+#pragma unroll
+    for (int i = 0; i < 32; ++i) k[i] = static_cast<int>(v[i]);
+  } else {
+#pragma unroll
+    for (int i = 0; i < 32; ++i) k[i] = i < lim ? static_cast<int>(v[i]) : INT_MIN;
+  }
+  const int x = max16(k), y = max16(k + 16);
+#pragma unroll
+  for (int b = 0; b < 16; ++b) R[b] = max3i(R[b], k[b], k[b + 16]);
+  const int hi = max(x, y), lo = min(x, y);
+  T2 = max3i(T2, min(T1, hi), lo);
+  T1 = max(T1, hi);
+}
+__device__ __forceinline__ void finish_fold(const int (&R)[16], int T1, int T2, int& x1, int& x2) {
+  int rm[4], cm[4];
+#pragma unroll
+  for (int a = 0; a < 4; ++a) {
+    rm[a] = max(max3i(R[4 * a], R[4 * a + 1], R[4 * a + 2]), R[4 * a + 3]);
+    cm[a] = max(max3i(R[a], R[a + 4], R[a + 8]), R[a + 12]);
+  }
+  const int sr = max3i(min(max(rm[0], rm[1]), max(rm[2], rm[3])), min(rm[0], rm[1]), min(rm[2], rm[3]));
+  const int sc = max3i(min(max(cm[0], cm[1]), max(cm[2], cm[3])), min(cm[0], cm[1]), min(cm[2], cm[3]));
+  x1 = T1;
+  x2 = max3i(T2, sr, sc);
+}
+
+__device__ __forceinline__ uint32_t dp4a_su(uint32_t a_s8, uint32_t b_u8, uint32_t c) {
+  uint32_t d;
+  asm("dp4a.s32.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a_s8), "r"(b_u8), "r"(c));
+  return d;
+}
+
+// Exact 2-NN distances (d1 <= d2) of one query row against one reference, straight from global
+// memory (the rare rows whose ratio decision the folded +-1 leaves open).  Whole warp; the
+// result is valid in every lane.  d = N_Q - 2 q'.r - W (column term W, < 0 marks padding).
+__device__ __forceinline__ void exact_row_global(const MatchParams& p, int qi, int row, int64_t ref, int32_t nqv,
+                                                 int lane, int cpr, int& d1, int& d2) {
+  const uint4* qrow = reinterpret_cast<const uint4*>(p.qs + (static_cast<int64_t>(qi) * p.n_rows + row) * kDim);
+  uint4 q[8];
+#pragma unroll
+  for (int w = 0; w < 8; ++w) q[w] = qrow[w];
+  int a1 = INT_MAX, a2 = INT_MAX;
+  for (int col = lane; col < cpr * kBN; col += 32) {
+    const int32_t W = p.colkey[ref * cpr * kColInts + col];
+    if (col >= p.m || W < 0) continue;
+    const uint4* rr = reinterpret_cast<const uint4*>(p.rdesc + ((p.ref_map_base + ref) * p.m + col) * kDim);
+    uint32_t dot = 0;
+#pragma unroll
+    for (int w = 0; w < 8; ++w) {
+      const uint4 x = rr[w];
+      dot = dp4a_su(q[w].x, x.x, dot); dot = dp4a_su(q[w].y, x.y, dot);
+      dot = dp4a_su(q[w].z, x.z, dot); dot = dp4a_su(q[w].w, x.w, dot);
+    }
+    const int d = nqv - 2 * static_cast<int>(dot) - W;
+    a2 = min(a2, max(a1, d));
+    a1 = min(a1, d);
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const int b1 = __shfl_xor_sync(0xffffffffu, a1, o), b2 = __shfl_xor_sync(0xffffffffu, a2, o);
+    const int m2 = min(max(a1, b1), min(a2, b2));
+    a1 = min(a1, b1);
+    a2 = m2;
+  }
+  d1 = a1;
+  d2 = a2;
+}
+
 // ------------------------------------------------------------------ fused match kernel
 // One persistent CTA per SM.  A job = (up to 4 references resident in SMEM) x (range of query
 // tiles streamed through a 4-stage ring).  Unit u = (query tile t, reference s), s fastest,
@@ -312,17 +421,17 @@ __device__ __forceinline__ void finish_partition(const int (&R)[16], int T1, int
 // a unit is computed as 4 MMA pieces of 64 columns; group g owns TMEM buffers 2g, 2g+1 and its
 // own MMA warp, so the MMA of the next piece overlaps the scan of the current one, and the 4
 // groups (4 epilogue warps per SMSP) hide each other's TMEM-load and barrier latency.
-// kSimple: one 256-column chunk per reference and no (d1, i1, d2, i2) output (the search
-// path), which frees the registers of the cross-chunk merge.
-template <bool kSimple>
+// kFold: the search path (folded norms, no column keys in the scan, counts only);
+// otherwise the verify path (packed column keys, exact (d1, i1, d2, i2)).
+template <bool kFold>
 __global__ void __launch_bounds__(kNumThreads, 1)
     match_kernel(const __grid_constant__ CUtensorMap qmap, const __grid_constant__ CUtensorMap rmap,
-                 const MatchParams p) {
+                 const __grid_constant__ CUtensorMap xmap, const MatchParams p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const uint32_t sbase = smem_u32(smem);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int T = p.tiles_per_q, cpr = kSimple ? 1 : p.cpr;
+  const int T = p.tiles_per_q, cpr = p.cpr;
 
   auto qfull = [&](int i) { return sbase + SmemPlan::kQFull + 8 * i; };
   auto qempty = [&](int i) { return sbase + SmemPlan::kQEmpty + 8 * i; };
@@ -332,9 +441,15 @@ __global__ void __launch_bounds__(kNumThreads, 1)
   auto tempty = [&](int i) { return sbase + SmemPlan::kTEmpty + 8 * i; };
   uint32_t* tmem_ptr_smem = reinterpret_cast<uint32_t*>(smem + SmemPlan::kTmemPtr);
 
+  if (kFold) {  // constant norm-term operand: every row (255 x 15, 1, 255 x 15, 1); both 16-B halves equal
+    uint32_t* ax = reinterpret_cast<uint32_t*>(smem + SmemPlan::kAx);
+    for (int i = threadIdx.x; i < kBM * kXDim / 4; i += blockDim.x) ax[i] = (i & 3) == 3 ? 0x01FFFFFFu : 0xFFFFFFFFu;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> tensor-core reads
+  }
   if (threadIdx.x == 0) {
     prefetch_tmap(&qmap);
     prefetch_tmap(&rmap);
+    if (kFold) prefetch_tmap(&xmap);
     // query stages are read only by the tensor core: freed by the 4 MMA warps' commits
     for (int i = 0; i < kQStages; ++i) { mbar_init(qfull(i), 1); mbar_init(qempty(i), kNG); }
     // reference slots: MMA operands + column keys read by every epilogue warp
@@ -364,11 +479,14 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         const int nslots = J.nr * cpr;
         for (int sl = 0; sl < nslots; ++sl) {
           PROF_B(); mbar_wait_sleep(rempty(sl), (slot_par >> sl & 1u) ^ 1); PROF_E(0);
-          mbar_expect_tx(rfull(sl), kRTileBytes + kColBytes);
+          mbar_expect_tx(rfull(sl), kRTileBytes + kColBytes + (kFold ? kXTileBytes : 0));
           const int s = sl / cpr, c = sl % cpr;
           const int64_t ref = J.ref_first + s;
           tma_load_3d(sbase + SmemPlan::kR + sl * kRTileBytes, &rmap, rfull(sl), 0, c * kBN,
                       static_cast<int>(p.ref_map_base + ref));
+          if (kFold)
+            tma_load_3d(sbase + SmemPlan::kX + sl * kXTileBytes, &xmap, rfull(sl), 0, c * kBN,
+                        static_cast<int>(p.ref_map_base + ref));
           bulk_load(sbase + SmemPlan::kCol + sl * kColBytes, p.colkey + (ref * cpr + c) * kColInts, kColBytes,
                     rfull(sl));
           slot_par ^= 1u << sl;
@@ -418,8 +536,14 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               const uint32_t buf = mw * kNB + (pc & 1);
               PROF_B(); mbar_wait(tempty(buf), ((pc >> 1) & 1) ^ 1); PROF_E(0);
               tc_fence_after();
-              // rows 64pp.. of the chunk: 8 SWIZZLE_128B core groups of 1024 B each
-              mma_piece(tmem_base + buf * kPiece, ad, bd0 + pp * (kPiece * kDim >> 4), tfull(buf));
+              // rows kPiece*pp.. of the chunk: SWIZZLE_128B core groups of 8 rows x 128 B
+              const uint64_t bd = bd0 + pp * (kPiece * kDim >> 4);
+              if (kFold)  // + norm-term K-step: rows kPiece*pp.. of the 32-B-wide tile
+                mma_piece_fold(tmem_base + buf * kPiece, ad, bd, smem_desc_sw32(sbase + SmemPlan::kAx),
+                               smem_desc_sw32(sbase + SmemPlan::kX + sl * kXTileBytes) + pp * (kPiece * kXDim >> 4),
+                               tfull(buf));
+              else
+                mma_piece<kIdescI8>(tmem_base + buf * kPiece, ad, bd, tfull(buf));
               ++pc;
             }
           }
@@ -484,6 +608,77 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           if (++ntq == T) { ntq = 0; ++nqi; }
         }
         const bool has_next = u + kNG < U;
+        bool pass = false;
+        if constexpr (kFold) {
+          int G1 = INT_MIN, G2 = INT_MIN;  // two largest folded values X over the reference
+          for (int c = 0; c < cpr; ++c) {
+            const uint32_t ck = sbase + SmemPlan::kCol + (s * cpr + c) * kColBytes;
+            int kpc;  // real columns of this chunk: the last column term is -1 - kpc when padded
+            asm volatile("ld.shared.s32 %0, [%1];" : "=r"(kpc) : "r"(ck + (kBN - 1) * 4));
+            kpc = kpc < 0 ? -1 - kpc : kBN;
+            int R[16];
+#pragma unroll
+            for (int b = 0; b < 16; ++b) R[b] = INT_MIN;
+            int T1 = INT_MIN, T2 = INT_MIN;
+#pragma unroll 1
+            for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
+              const uint32_t buf = g * kNB + (mp & 1);
+              PROF_B(); mbar_wait(tfull(buf), (mp >> 1) & 1); PROF_E(0);
+              tc_fence_after();
+#pragma unroll
+              for (int h = 0; h < kPiece / 64; ++h) {
+                tmem_ld64(taddr_q + buf * kPiece + h * 64, v);
+                tmem_wait_ld();
+                reg_fence64(v);
+                if (h == kPiece / 64 - 1) {  // the piece is in registers: buffer free
+                  tc_fence_before();
+                  __syncwarp();
+                  if (lane == 0) mbar_arrive(tempty(buf));
+                  ++mp;
+                }
+                PROF_B();
+                const int base = pp * kPiece + h * 64;
+                scan32_fold(v, kpc - base, R, T1, T2);
+                scan32_fold(v + 32, kpc - base - 32, R, T1, T2);
+                PROF_E(1);
+              }
+            }
+            PROF_B();
+            int x1, x2;
+            finish_fold(R, T1, T2, x1, x2);
+            G2 = max3i(min(G1, x1), G2, x2);
+            G1 = max(G1, x1);
+            PROF_E(2);
+          }
+          // d = N_Q - 2X - p, p in {0, 1}: decide the ratio test from the bounds
+          const bool real2 = G2 > INT_MIN;
+          bool undecided = false;
+          if (valid && real2) {
+            const int hi1 = nqv - 2 * G1, hi2 = nqv - 2 * G2;
+            const int lo1 = max(hi1 - 1, 0), lo2 = max(hi2 - 1, 0);
+            bool pass_sure, fail_sure;
+            if (ratio32) {
+              pass_sure = p.den2 * static_cast<uint32_t>(hi1) < p.num2 * static_cast<uint32_t>(lo2);
+              fail_sure = p.den2 * static_cast<uint32_t>(lo1) >= p.num2 * static_cast<uint32_t>(hi2);
+            } else {
+              pass_sure = uint64_t(p.den2) * uint64_t(hi1) < uint64_t(p.num2) * uint64_t(lo2);
+              fail_sure = uint64_t(p.den2) * uint64_t(lo1) >= uint64_t(p.num2) * uint64_t(hi2);
+            }
+            pass = pass_sure;
+            undecided = !pass_sure && !fail_sure;
+          }
+          uint32_t und = __ballot_sync(0xffffffffu, undecided);
+          while (und) {  // rare: recompute the row exactly
+            const int l = __ffs(und) - 1;
+            und &= und - 1;
+            const int rl = __shfl_sync(0xffffffffu, row, l);
+            const int nl = __shfl_sync(0xffffffffu, nqv, l);
+            int d1, d2;
+            exact_row_global(p, qi, rl, J.ref_first + s, nl, lane, cpr, d1, d2);
+            if (lane == l)
+              pass = d2 != INT_MAX && uint64_t(p.den2) * uint64_t(d1) < uint64_t(p.num2) * uint64_t(d2);
+          }
+        } else {
         int g1d = INT_MAX, g1i = -1, g2d = INT_MAX, g2i = -1;  // running exact 2-NN over chunks
         for (int c = 0; c < cpr; ++c) {
           const uint32_t ck = sbase + SmemPlan::kCol + (s * cpr + c) * kColBytes;
@@ -519,7 +714,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           finish_partition(R, T1, T2, k1, k2);
           const int c1d = k1 >> 8, c1i = (k1 & 255) + c * kBN;
           const int c2d = k2 >> 8, c2i = (k2 & 255) + c * kBN;
-          if (kSimple || c == 0) {
+          if (c == 0) {
             g1d = c1d; g1i = c1i; g2d = c2d; g2i = c2i;
           } else if (c1d < g1d) {  // merge into the running 2-NN; earlier chunks win ties (lower index)
             if (c2d < g1d) { g2d = c2d; g2i = c2i; } else { g2d = g1d; g2i = g1i; }
@@ -531,7 +726,6 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         }
         // ratio test in exact integers: den^2 * d1 < num^2 * d2
         const bool real1 = g1d < kSentinelNorm, real2 = g2d < kSentinelNorm;
-        bool pass;
         if (ratio32) {
           const uint32_t d1 = static_cast<uint32_t>(nqv + g1d), d2 = static_cast<uint32_t>(nqv + g2d);
           pass = p.den2 * d1 < p.num2 * d2;
@@ -541,13 +735,14 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           pass = static_cast<uint64_t>(p.den2) * d1 < static_cast<uint64_t>(p.num2) * d2;
         }
         pass = pass && valid && real2;
-        cnt += __popc(__ballot_sync(0xffffffffu, pass));
-        if (!kSimple && p.nn_out != nullptr && row < p.n_rows) {
+        if (p.nn_out != nullptr && row < p.n_rows) {
           int4 o;
           o.x = (valid && real1) ? nqv + g1d : -1; o.y = (valid && real1) ? g1i : -1;
           o.z = (valid && real2) ? nqv + g2d : -1; o.w = (valid && real2) ? g2i : -1;
           reinterpret_cast<int4*>(p.nn_out)[static_cast<int64_t>(qi) * p.n_rows + row] = o;
         }
+        }
+        cnt += __popc(__ballot_sync(0xffffffffu, pass));
         // flush the count when the group's next unit is another (query, reference) pair
         if (!has_next || ns != s || nqi != qi) {
           if (lane == 0 && cnt) {
@@ -586,18 +781,18 @@ extern "C" int tid_debug_read_prof(void* host, size_t bytes) {
 #endif
 
 
-cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap, int grid,
-                         cudaStream_t s) {
+cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap,
+                         const CUtensorMap* xmap, int grid, cudaStream_t s) {
   cudaError_t e = cudaFuncSetAttribute(match_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(SmemPlan::kAlloc));
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(match_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                            static_cast<int>(SmemPlan::kAlloc));
   if (e != cudaSuccess) return e;
-  if (p.cpr == 1 && p.nn_out == nullptr)
-    match_kernel<true><<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, p);
+  if (xmap)
+    match_kernel<true><<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, *xmap, p);
   else
-    match_kernel<false><<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, p);
+    match_kernel<false><<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, rmap, p);
   return cudaGetLastError();
 }
 
@@ -614,28 +809,59 @@ __global__ void ref_prep_kernel(RefPrepParams p) {
   const int i = static_cast<int>(gid % cols);
   int kp = p.kp ? p.kp[r] : p.m;
   kp = max(0, min(kp, p.m));
-  int32_t norm = kSentinelNorm;
+  const int c = i / kBN, ii = i & (kBN - 1);
+  int32_t norm = kSentinelNorm;  // N_R = sum r^2 (Alg. 1 step 1)
+  int32_t sum = 0;               // sum r (search column term W = 256 sum r - N_R)
+  const bool real = i < kp;
   if (i < p.m) {
     uint4* dst = p.desc ? reinterpret_cast<uint4*>(p.desc + (r * p.m + i) * kDim) : nullptr;
-    if (i < kp) {
+    if (real) {
       const uint4* src = p.src ? reinterpret_cast<const uint4*>(p.src + (r * p.m + i) * kDim) : dst;
-      uint32_t acc = 0;
+      uint32_t acc = 0, s1 = 0;
 #pragma unroll
       for (int w = 0; w < kDim / 16; ++w) {
         const uint4 x = src[w];
         acc = __dp4a(x.x, x.x, acc); acc = __dp4a(x.y, x.y, acc);
         acc = __dp4a(x.z, x.z, acc); acc = __dp4a(x.w, x.w, acc);
+        s1 = __dp4a(x.x, 0x01010101u, s1); s1 = __dp4a(x.y, 0x01010101u, s1);
+        s1 = __dp4a(x.z, 0x01010101u, s1); s1 = __dp4a(x.w, 0x01010101u, s1);
         if (p.src && dst) dst[w] = x;
       }
       norm = static_cast<int32_t>(acc);
+      sum = static_cast<int32_t>(s1);
     } else if (dst) {
 #pragma unroll
       for (int w = 0; w < kDim / 16; ++w) dst[w] = make_uint4(0, 0, 0, 0);
     }
+    if (p.extra) {
+      // u8 digits b of E = floor(W / 2) against the constant operand a = (255 x 15, 1, 255 x 15, 1):
+      // E = 255 * (sum of the 30 "255" digits) + b15 + b31  (capacity 1,951,260 >= max E = 1,048,576)
+      uint32_t d[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+      if (real) {
+        const uint32_t E = static_cast<uint32_t>(256 * sum - norm) >> 1;
+        uint32_t hi = E / 255;
+        const uint32_t lo = E - hi * 255;
+        uint8_t* db = reinterpret_cast<uint8_t*>(d);
+        for (int t = 0; t < kXDim && hi; ++t) {
+          if (t == 15 || t == 31) continue;
+          const uint32_t v = hi < 255 ? hi : 255;
+          db[t] = static_cast<uint8_t>(v);
+          hi -= v;
+        }
+        db[15] = static_cast<uint8_t>(lo);
+      }
+      uint4* xd = reinterpret_cast<uint4*>(p.extra + (r * p.m + i) * kXDim);
+      xd[0] = make_uint4(d[0], d[1], d[2], d[3]);
+      xd[1] = make_uint4(d[4], d[5], d[6], d[7]);
+    }
   }
-  const int c = i / kBN, ii = i & (kBN - 1);
   int32_t* ck = p.colkey + (r * p.cpr + c) * kColInts;
-  ck[ii] = norm * 256 + ii;
+  if (p.extra) {
+    const int kpc = max(0, min(kp - c * kBN, kBN));  // real columns in this chunk
+    ck[ii] = real ? 256 * sum - norm : -1 - kpc;
+  } else {
+    ck[ii] = norm * 256 + ii;
+  }
 }
 
 void launch_ref_prep(const RefPrepParams& p, cudaStream_t s) {
@@ -645,8 +871,10 @@ void launch_ref_prep(const RefPrepParams& p, cudaStream_t s) {
 }
 
 // ------------------------------------------------------------------ a2: query prep
+// N_Q per row (Alg. 1 step 2) and, for the search path, the shifted copy q' = q ^ 0x80
+// (= q - 128 as s8), one 16-byte word per thread-iteration.
 __global__ void query_prep_kernel(const uint8_t* __restrict__ q, int64_t B, int32_t n, int32_t rows_pad,
-                                  int32_t* __restrict__ nq) {
+                                  int32_t* __restrict__ nq, uint8_t* __restrict__ qs) {
   const int64_t gid = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
   if (gid >= B * rows_pad) return;
   const int64_t b = gid / rows_pad;
@@ -654,21 +882,24 @@ __global__ void query_prep_kernel(const uint8_t* __restrict__ q, int64_t B, int3
   uint32_t acc = 0;
   if (row < n) {
     const uint4* src = reinterpret_cast<const uint4*>(q + (b * n + row) * kDim);
+    uint4* dst = qs ? reinterpret_cast<uint4*>(qs + (b * n + row) * kDim) : nullptr;
 #pragma unroll
     for (int w = 0; w < kDim / 16; ++w) {
       const uint4 x = src[w];
       acc = __dp4a(x.x, x.x, acc); acc = __dp4a(x.y, x.y, acc);
       acc = __dp4a(x.z, x.z, acc); acc = __dp4a(x.w, x.w, acc);
+      if (dst) dst[w] = make_uint4(x.x ^ 0x80808080u, x.y ^ 0x80808080u, x.z ^ 0x80808080u, x.w ^ 0x80808080u);
     }
   }
   nq[gid] = static_cast<int32_t>(acc);
 }
 
-void launch_query_prep(const uint8_t* q, int64_t B, int32_t n, int32_t tiles_per_q, int32_t* nq, cudaStream_t s) {
+void launch_query_prep(const uint8_t* q, int64_t B, int32_t n, int32_t tiles_per_q, int32_t* nq, uint8_t* qs,
+                       cudaStream_t s) {
   const int32_t rows_pad = tiles_per_q * kBM;
   const int64_t total = B * rows_pad;
   if (total == 0) return;
-  query_prep_kernel<<<static_cast<unsigned>((total + 255) / 256), 256, 0, s>>>(q, B, n, rows_pad, nq);
+  query_prep_kernel<<<static_cast<unsigned>((total + 255) / 256), 256, 0, s>>>(q, B, n, rows_pad, nq, qs);
 }
 
 // ------------------------------------------------------------------ a6: top-k of the count matrix

@@ -21,7 +21,7 @@ namespace tid {
 constexpr int kDim = 128;          // SIFT descriptor length, bytes per keypoint row
 constexpr int kBM = 128;           // query keypoints per MMA tile (TMEM lanes)
 constexpr int kBN = 256;           // reference keypoints per chunk (MMA N, TMEM columns)
-constexpr int kQStages = 4;        // query-tile ring
+constexpr int kQStages = 3;        // query-tile ring
 constexpr int kMaxSlots = 4;       // resident reference chunks per CTA
 #ifndef TID_NG
 #define TID_NG 3
@@ -42,8 +42,19 @@ constexpr uint32_t kRTileBytes = kBN * kDim;   // 32 KiB
 constexpr int kColInts = kBN;                  // per chunk: 256 packed column keys
 constexpr uint32_t kColBytes = kColInts * 4;   // 1 KiB per chunk
 constexpr int32_t kSentinelNorm = (1 << 23) - 1;  // > 128*255^2: padded columns never win
+constexpr int kXDim = 32;                      // bytes of the per-column norm-term operand (one MMA K-step)
+constexpr uint32_t kXTileBytes = kBN * kXDim;  // 8 KiB per 256-column chunk
 
-// Packed column key, per 256-column chunk (global layout [ref][chunk][256] int32):
+// Search path ("folded" norms).  With q' = q - 128 (s8) and r (u8),
+//   S3 = sum_t q'_t r_t = S - 128 sum_t r_t,  W = sum_t r_t (256 - r_t) = 256 sum r - N_R >= 0,
+//   d(q, r) = N_Q + N_R - 2S = N_Q - (2 S3 + W).
+// A fifth MMA K-step adds E = floor(W / 2) (u8 digits of E against a constant u8 operand), so
+// TMEM holds X = S3 + E and  d = N_Q - 2X - p,  p = W mod 2 in {0, 1}: the two LARGEST X of a
+// row are its two nearest columns (ties broken by p), and d1, d2 are known to within 1.  Rows
+// whose ratio decision the +-1 can flip are recomputed exactly (rare).  Column term array for
+// search: W (>= 0) for real columns, -1 - kp(chunk) for padded ones.
+//
+// Packed column key (verify path), per 256-column chunk (global layout [ref][chunk][256] int32):
 //   colkey[i] = N_R[i] * 256 + i   (i = index within the chunk).
 // The epilogue forms key = colkey - 512 * S = 256 * (N_R - 2 q.r) + i with one IMAD, which
 // orders exactly like (d_ji, i) for a fixed query row (Alg. 1 step 4 + lowest-index
@@ -71,13 +82,18 @@ struct MatchParams {
   int64_t col0;
   int32_t* nn_out;           // verify: [num_q][n_rows][4] or null
   uint32_t num2, den2;       // ratio^2 = num2/den2
+  // search (folded norms): exact fallback operands in global memory
+  const uint8_t* qs;         // [num_q][n_rows][128] shifted queries q' = q ^ 0x80
+  const uint8_t* rdesc;      // reference descriptors of the tensor map, [*][m][128] raw u8
+  int32_t m;                 // stored rows per reference
 };
 
 struct RefPrepParams {
   uint8_t* desc;             // [count][m][128] destination (null = read-only, keys only)
   const uint8_t* src;        // optional source to copy from (null = in place)
   const int32_t* kp;         // [count] or null (= m)
-  int32_t* colkey;           // [count][cpr][256]
+  int32_t* colkey;           // [count][cpr][256]: packed keys (verify) or column terms (search)
+  uint8_t* extra;            // search only: [count][m][32] u8 digits of floor(W / 2) (null = verify keys)
   int64_t count;
   int32_t m;
   int32_t cpr;
@@ -85,9 +101,9 @@ struct RefPrepParams {
 
 void launch_ref_prep(const RefPrepParams& p, cudaStream_t s);
 void launch_query_prep(const uint8_t* q, int64_t B, int32_t n, int32_t tiles_per_q, int32_t* nq,
-                       cudaStream_t s);
+                       uint8_t* qs, cudaStream_t s);
 cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap,
-                         int grid, cudaStream_t s);
+                         const CUtensorMap* xmap, int grid, cudaStream_t s);
 void launch_topk(const uint32_t* counts, int64_t B, int64_t R, int64_t ldc, int64_t id_base, int32_t k,
                  int32_t segs, const uint8_t* dead, uint64_t* cand_out, cudaStream_t s);
 void launch_merge(const uint64_t* cand, int32_t L, int64_t B, int32_t k, int64_t list_stride_b,

@@ -201,9 +201,10 @@ def test_device_tensors_and_stream(tid):
 
 @pytest.mark.parametrize("hi", [3, 24, 256])
 def test_search_fast_path_fallback(tid, rng, hi):
-    """Search fast path (16-bit packed keys + exact fallback): low-range data makes most rows
-    undecidable (exact re-scan), full-range data almost none; both must equal the oracle and
-    the exact-only path bit for bit."""
+    """Search path (folded norms: d known to +-1 from the MMA, exact global-memory recompute of
+    the rows whose ratio decision that leaves open): low-range data makes many rows undecided,
+    full-range data almost none; both must equal the oracle bit for bit.  `exact_only` is an
+    accepted no-op tuning flag (kept for ABI stability) and must not change anything."""
     R, m, n, B = 24, 256, 300, 2
     refs = rng.integers(0, hi, (R, m, 128), dtype=np.uint8)
     qs = rng.integers(0, hi, (B, n, 128), dtype=np.uint8)
@@ -220,8 +221,8 @@ def test_search_fast_path_fallback(tid, rng, hi):
 
 def test_search_boundary_ratios(tid):
     """Rows whose ratio sits exactly on / next to the 0.8 boundary at large distances (the
-    coarse bounds straddle, forcing the exact fallback): q = 0, two reference keypoints with
-    ||r||^2 = 16 s^2 and 25 s^2 (+/- 1)."""
+    folded +-1 bounds straddle it, forcing the exact recompute): q = 0, two reference keypoints
+    with ||r||^2 = 16 s^2 and 25 s^2 (+/- 1)."""
     m, n = 256, 8
     R = np.zeros((1, m, 128), np.uint8)
     # d1 = 16*s^2 via sixteen entries of s; d2 = 25*s^2 via twenty-five entries of s (+ tweak)
