@@ -157,6 +157,34 @@ __device__ __forceinline__ void mma_piece_fold(uint32_t tmem_d, uint64_t adesc, 
       : "memory");
 }
 
+// SMEM (matrix descriptor) -> TMEM: 128 rows x 32 B into 128 lanes x 8 columns (single thread).
+__device__ __forceinline__ void tmem_cp_128x256b(uint32_t taddr, uint64_t sdesc) {
+  asm volatile("tcgen05.cp.cta_group::1.128x256b [%0], %1;" ::"r"(taddr), "l"(sdesc) : "memory");
+}
+__device__ __forceinline__ void commit_one(uint32_t bar) {  // single-thread form
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
+}
+// Search piece with A in TMEM: four q'.r K-steps (A = 8 TMEM columns per K-step), then the norm-term
+// K-step (A = constant operand in TMEM).  Only B is read from shared memory.
+__device__ __forceinline__ void mma_piece_fold_ts(uint32_t tmem_d, uint32_t a_tmem, uint64_t bdesc, uint32_t ax_tmem,
+                                                  uint64_t bxdesc, uint32_t bar) {
+  asm volatile(
+      "{\n\t.reg .pred e, f, t;\n\t.reg .b32 a1, a2, a3;\n\t.reg .b64 b1, b2, b3;\n\t"
+      "setp.ne.b32 f, 0, 0;\n\t"
+      "setp.eq.b32 t, 0, 0;\n\t"
+      "add.u32 a1, %1, 8;\n\tadd.u32 a2, %1, 16;\n\tadd.u32 a3, %1, 24;\n\t"
+      "add.s64 b1, %2, 2;\n\tadd.s64 b2, %2, 4;\n\tadd.s64 b3, %2, 6;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %5, f;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [a1], b1, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [a2], b2, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [a3], b3, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [%3], %4, %6, t;\n\t"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%7];\n\t}" ::"r"(tmem_d),
+      "r"(a_tmem), "l"(bdesc), "r"(ax_tmem), "l"(bxdesc), "r"(kIdescFold), "r"(kIdescI8), "r"(bar)
+      : "memory");
+}
+
 __device__ __forceinline__ void mma_commit(uint32_t bar) {
   asm volatile(
       "{\n\t.reg .pred e;\n\t"
@@ -231,6 +259,14 @@ __device__ unsigned long long g_prof[148 * 32 * 8];
 #define PROF_FLUSH()
 #endif
 
+// TMEM columns: accumulators [0, 384); search-path A operands: kTQ query tiles of 32 columns
+// (128 rows x 128 B, K packed 4 bytes per column) and the constant norm-term operand (8 columns).
+constexpr int kTQ = 3;
+constexpr int kQCols = kDim / 4;
+constexpr int kTQBase = kTmemBufs * kPiece;
+constexpr int kAxCol = kTQBase + kTQ * kQCols;
+static_assert(kAxCol + kXDim / 4 <= 512, "TMEM budget");
+
 constexpr int kProducerWarp = 0;               // warp 0: TMA producer
 constexpr int kFirstMmaWarp = 1;               // warps 1..3: MMA issuer of group mw (SMSPs 1, 2, 3)
 constexpr int kFirstEpiWarp = 1 + kNG;         // warps 4..15: epilogue, group (w-4)/4, lane quarter w%4
@@ -251,7 +287,10 @@ struct SmemPlan {
   static constexpr uint32_t kREmpty = kRFull + 8 * kMaxSlots;
   static constexpr uint32_t kTFull = kREmpty + 8 * kMaxSlots;
   static constexpr uint32_t kTEmpty = kTFull + 8 * kTmemBufs;
-  static constexpr uint32_t kTmemPtr = kTEmpty + 8 * kTmemBufs;
+  static constexpr uint32_t kTQFull = kTEmpty + 8 * kTmemBufs;           // query tiles staged in TMEM (search)
+  static constexpr uint32_t kTQEmpty = kTQFull + 8 * kTQ;
+  static constexpr uint32_t kAxFull = kTQEmpty + 8 * kTQ;
+  static constexpr uint32_t kTmemPtr = kAxFull + 8;
   static constexpr uint32_t kEnd = kTmemPtr + 16;
   static constexpr uint32_t kAlloc = kEnd + 1024;                          // + alignment slack
 };
@@ -342,15 +381,11 @@ __device__ __forceinline__ int max16(const int* k) {
   const int d = max3i(k[9], k[10], k[11]), e = max3i(k[12], k[13], k[14]);
   return max(max3i(a, b, c), max3i(d, e, k[15]));
 }
+template <bool kMask>
 __device__ __forceinline__ void scan32_fold(const uint32_t* v, int lim, int (&R)[16], int& T1, int& T2) {
   int k[32];
-  if (lim >= 32) {
 #pragma unroll
-    for (int i = 0; i < 32; ++i) k[i] = static_cast<int>(v[i]);
-  } else {
-#pragma unroll
-    for (int i = 0; i < 32; ++i) k[i] = i < lim ? static_cast<int>(v[i]) : INT_MIN;
-  }
+  for (int i = 0; i < 32; ++i) k[i] = (!kMask || i < lim) ? static_cast<int>(v[i]) : INT_MIN;
   const int x = max16(k), y = max16(k + 16);
 #pragma unroll
   for (int b = 0; b < 16; ++b) R[b] = max3i(R[b], k[b], k[b + 16]);
@@ -439,6 +474,9 @@ __global__ void __launch_bounds__(kNumThreads, 1)
   auto rempty = [&](int i) { return sbase + SmemPlan::kREmpty + 8 * i; };
   auto tfull = [&](int i) { return sbase + SmemPlan::kTFull + 8 * i; };
   auto tempty = [&](int i) { return sbase + SmemPlan::kTEmpty + 8 * i; };
+  auto tqfull = [&](int i) { return sbase + SmemPlan::kTQFull + 8 * i; };
+  auto tqempty = [&](int i) { return sbase + SmemPlan::kTQEmpty + 8 * i; };
+  const uint32_t axfull = sbase + SmemPlan::kAxFull;
   uint32_t* tmem_ptr_smem = reinterpret_cast<uint32_t*>(smem + SmemPlan::kTmemPtr);
 
   if (kFold) {  // constant norm-term operand: every row (255 x 15, 1, 255 x 15, 1); both 16-B halves equal
@@ -450,8 +488,11 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     prefetch_tmap(&qmap);
     prefetch_tmap(&rmap);
     if (kFold) prefetch_tmap(&xmap);
-    // query stages are read only by the tensor core: freed by the 4 MMA warps' commits
-    for (int i = 0; i < kQStages; ++i) { mbar_init(qfull(i), 1); mbar_init(qempty(i), kNG); }
+    // query stages: search copies each tile to TMEM (freed by that copy); verify feeds the MMAs from
+    // shared memory (freed by the kNG MMA warps' commits)
+    for (int i = 0; i < kQStages; ++i) { mbar_init(qfull(i), 1); mbar_init(qempty(i), kFold ? 1 : kNG); }
+    for (int i = 0; i < kTQ; ++i) { mbar_init(tqfull(i), 1); mbar_init(tqempty(i), kNG); }
+    mbar_init(axfull, 1);
     // reference slots: MMA operands + column keys read by every epilogue warp
     for (int i = 0; i < kMaxSlots; ++i) { mbar_init(rfull(i), 1); mbar_init(rempty(i), kNG + kEpiWarps); }
     for (int i = 0; i < kTmemBufs; ++i) { mbar_init(tfull(i), 1); mbar_init(tempty(i), 4); }
@@ -472,6 +513,11 @@ __global__ void __launch_bounds__(kNumThreads, 1)
   if (warp == kProducerWarp) {
     // ===================== TMA producer =====================
     if (lane == 0) {
+      if (kFold) {  // constant norm-term operand -> TMEM, once
+        tc_fence_after();
+        tmem_cp_128x256b(tmem_base + kAxCol, smem_desc_sw32(sbase + SmemPlan::kAx));
+        commit_one(axfull);
+      }
       uint32_t qctr = 0;
       uint32_t slot_par = 0;  // bit sl = phase parity of reference slot sl
       for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
@@ -492,11 +538,36 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           slot_par ^= 1u << sl;
         }
         const int ntiles = J.nq * T;
+        if (kFold) {
+          // TMA tile t+1 into shared memory while tile t is copied to its TMEM slot (the MMAs read A
+          // from TMEM, so each query tile crosses the shared-memory port once, not once per piece)
+          auto issue = [&](int t) {
+            const uint32_t gq = qctr + t, st = gq % kQStages;
+            PROF_B(); mbar_wait_sleep(qempty(st), ((gq / kQStages) & 1) ^ 1); PROF_E(1);
+            mbar_expect_tx(qfull(st), kQTileBytes);
+            tma_load_3d(sbase + SmemPlan::kQ + st * kQTileBytes, &qmap, qfull(st), 0, (t % T) * kBM, J.q_first + t / T);
+          };
+          if (ntiles > 0) issue(0);
+          for (int t = 0; t < ntiles; ++t) {
+            if (t + 1 < ntiles) issue(t + 1);
+            const uint32_t gq = qctr + t, st = gq % kQStages, sl = gq % kTQ;
+            mbar_wait(qfull(st), (gq / kQStages) & 1);
+            mbar_wait_sleep(tqempty(sl), ((gq / kTQ) & 1) ^ 1);
+            tc_fence_after();
+            const uint64_t sd = smem_desc_sw128(sbase + SmemPlan::kQ + st * kQTileBytes);
+#pragma unroll
+            for (int k = 0; k < kDim / kXDim; ++k) tmem_cp_128x256b(tmem_base + kTQBase + sl * kQCols + 8 * k, sd + 2 * k);
+            commit_one(tqfull(sl));
+            commit_one(qempty(st));
+          }
+          qctr += ntiles;
+        } else {
         for (int t = 0; t < ntiles; ++t, ++qctr) {
           const int st = qctr % kQStages;
           PROF_B(); mbar_wait_sleep(qempty(st), ((qctr / kQStages) & 1) ^ 1); PROF_E(1);
           mbar_expect_tx(qfull(st), kQTileBytes);
           tma_load_3d(sbase + SmemPlan::kQ + st * kQTileBytes, &qmap, qfull(st), 0, (t % T) * kBM, J.q_first + t / T);
+        }
         }
       }
     }
@@ -508,6 +579,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     // query tile (waiting for tiles it never used, so the stage phases stay in order).
     const int mw = warp - kFirstMmaWarp;
     uint32_t qctr = 0, pc = 0;
+    if (kFold) mbar_wait(axfull, 0);  // constant norm-term operand in TMEM
     uint32_t slot_par = 0;  // bit sl = phase parity of reference slot sl
     for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
       const Job J = decode_job(p, j);
@@ -519,11 +591,15 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         if (g == mw) {
           while (waited <= t) {
             const uint32_t gq = qctr + waited;
-            PROF_B(); mbar_wait(qfull(gq % kQStages), (gq / kQStages) & 1); PROF_E(1);
+            PROF_B();
+            if (kFold) mbar_wait(tqfull(gq % kTQ), (gq / kTQ) & 1);
+            else mbar_wait(qfull(gq % kQStages), (gq / kQStages) & 1);
+            PROF_E(1);
             ++waited;
           }
           const uint32_t st = (qctr + t) % kQStages;
           const uint64_t ad = smem_desc_sw128(sbase + SmemPlan::kQ + st * kQTileBytes);
+          const uint32_t at = tmem_base + kTQBase + ((qctr + t) % kTQ) * kQCols;  // search: A in TMEM
           for (int c = 0; c < cpr; ++c) {
             const int sl = s * cpr + c;
             if (!(ready_mask >> sl & 1u)) {
@@ -539,9 +615,9 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               // rows kPiece*pp.. of the chunk: SWIZZLE_128B core groups of 8 rows x 128 B
               const uint64_t bd = bd0 + pp * (kPiece * kDim >> 4);
               if (kFold)  // + norm-term K-step: rows kPiece*pp.. of the 32-B-wide tile
-                mma_piece_fold(tmem_base + buf * kPiece, ad, bd, smem_desc_sw32(sbase + SmemPlan::kAx),
-                               smem_desc_sw32(sbase + SmemPlan::kX + sl * kXTileBytes) + pp * (kPiece * kXDim >> 4),
-                               tfull(buf));
+                mma_piece_fold_ts(tmem_base + buf * kPiece, at, bd, tmem_base + kAxCol,
+                                  smem_desc_sw32(sbase + SmemPlan::kX + sl * kXTileBytes) + pp * (kPiece * kXDim >> 4),
+                                  tfull(buf));
               else
                 mma_piece<kIdescI8>(tmem_base + buf * kPiece, ad, bd, tfull(buf));
               ++pc;
@@ -549,12 +625,13 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           }
         }
         if (s == J.nr - 1) {  // this warp's release of query tile t (covers all its prior MMAs)
+          const uint32_t gq = qctr + t;
           if (waited <= t) {  // never touched tile t: still wait for it so the phase order holds
-            const uint32_t gq = qctr + t;
-            mbar_wait(qfull(gq % kQStages), (gq / kQStages) & 1);
+            if (kFold) mbar_wait(tqfull(gq % kTQ), (gq / kTQ) & 1);
+            else mbar_wait(qfull(gq % kQStages), (gq / kQStages) & 1);
             waited = t + 1;
           }
-          mma_commit(qempty((qctr + t) % kQStages));
+          mma_commit(kFold ? tqempty(gq % kTQ) : qempty(gq % kQStages));
         }
         if (++g == kNG) g = 0;
         if (++s == J.nr) { s = 0; ++t; }
@@ -638,8 +715,13 @@ __global__ void __launch_bounds__(kNumThreads, 1)
                 }
                 PROF_B();
                 const int base = pp * kPiece + h * 64;
-                scan32_fold(v, kpc - base, R, T1, T2);
-                scan32_fold(v + 32, kpc - base - 32, R, T1, T2);
+                if (kpc >= kBN) {  // full chunk (the common case): no masking
+                  scan32_fold<false>(v, 32, R, T1, T2);
+                  scan32_fold<false>(v + 32, 32, R, T1, T2);
+                } else {
+                  scan32_fold<true>(v, kpc - base, R, T1, T2);
+                  scan32_fold<true>(v + 32, kpc - base - 32, R, T1, T2);
+                }
                 PROF_E(1);
               }
             }
