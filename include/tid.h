@@ -163,6 +163,29 @@ tid_status tid_merge_topk(tid_index* idx, const int64_t* ids_in, const int32_t* 
                           int32_t G, int64_t B, int32_t k, int64_t* ids_out, int32_t* counts_out,
                           void* stream);
 
+/*
+ * Float-descriptor path (the paper's RootSIFT + FP16 configuration,
+ * §4.2, §5.1, Algorithm 2).  Uses the index only for its
+ * device, ratio and workspace; references are passed per call (not stored).
+ *
+ * tid_f16_prepare: u8 SIFT [rows][128] (host or device) -> fp16 bits [rows][128] (host or device):
+ *   rootsift != 0: x / sum(x), element-wise sqrt (RootSIFT; all-zero rows stay 0);
+ *   then multiply by `scale` (> 0; the paper's fp16 scale factor, 2^-7 in practice, P:504-507,
+ *   P:527-530) and round to nearest even.  Computed in fp32 on the GPU.
+ *
+ * tid_f16_search_counts: good-match counts of B fp16 queries [B][n][128] against R fp16 references
+ *   [R][m][128] (host or device; n <= query_kp_max, 2 <= m <= 256) -> counts_out uint32 [B][R].
+ *   The product q.r runs on tcgen05.mma.kind::f16 with fp32 accumulation; d = N_Q + N_R - 2 q.r in
+ *   fp32 (N in fp32 from the fp16 values); 2-NN per query row; ratio test
+ *   den^2 * d1 < num^2 * d2 compared in fp64.  Counts equal the exact float64 definition
+ *   on the same fp16 values except where fp32 rounding moves a ratio across the threshold
+ *   (acceptance: within +-1 for >= 99.9% of pairs; exact for u8 SIFT x 2^-k).
+ */
+tid_status tid_f16_prepare(tid_index* idx, const uint8_t* sift, int64_t rows, int32_t rootsift, float scale,
+                           uint16_t* out, void* stream);
+tid_status tid_f16_search_counts(tid_index* idx, const uint16_t* q, int32_t n, int64_t B, const uint16_t* r,
+                                 int32_t m, int64_t R, uint32_t* counts_out, void* stream);
+
 /* 128-byte ncclUniqueId for rank 0 to broadcast before tid_index_create. */
 tid_status tid_nccl_unique_id(void* out128);
 
@@ -195,9 +218,9 @@ tid_status tid_get_stats(tid_index* idx, tid_stats* out); /* synchronises record
 
 /* Tuning knobs (0 = automatic).  refs_per_job: references resident per CTA job (1..4);
  * grid: persistent CTAs for the match kernel; host_chunk_refs: references per
- * host-tier staging buffer; exact_only: disable the search fast path (16-bit packed
- * top-2 with exact fallback) and scan every element with exact 32-bit keys.  Results
- * are identical either way. */
+ * host-tier staging buffer; exact_only: accepted for ABI stability and ignored (every
+ * scan is exact; the search path recomputes the rare +-1-undecided rows exactly).
+ * Results never depend on these knobs. */
 typedef struct {
   int32_t refs_per_job;
   int32_t grid;

@@ -26,7 +26,7 @@ STATUS = {0: "TID_OK", -1: "TID_EINVAL", -2: "TID_ENOMEM", -3: "TID_ECUDA", -4: 
 EXPORTS = ("tid_index_create", "tid_index_destroy", "tid_add_references", "tid_search", "tid_search_counts",
            "tid_verify", "tid_merge_topk", "tid_nccl_unique_id", "tid_get_info", "tid_profile", "tid_get_stats",
            "tid_set_tuning", "tid_delete_references", "tid_update_references", "tid_index_save", "tid_index_load",
-           "tid_last_error")
+           "tid_f16_prepare", "tid_f16_search_counts", "tid_last_error")
 
 
 class TidError(RuntimeError):
@@ -89,6 +89,8 @@ def load_library(path: str = LIB_PATH):
     lib.tid_update_references.argtypes = [vp, vp, vp, vp, i64]
     lib.tid_index_save.argtypes = [vp, ctypes.c_char_p]
     lib.tid_index_load.argtypes = [vp, ctypes.c_char_p, P(i64)]
+    lib.tid_f16_prepare.argtypes = [vp, vp, i64, i32, ctypes.c_float, vp, vp]
+    lib.tid_f16_search_counts.argtypes = [vp, vp, i32, i64, vp, i32, i64, vp, vp]
     lib.tid_last_error.restype = ctypes.c_char_p
     for name in EXPORTS[:-1]:
         getattr(lib, name).restype = ctypes.c_int
@@ -225,6 +227,34 @@ class Index:
             out = np.empty((B, R), np.uint32)
         op, k3 = _ptr(out)
         _check(self._lib.tid_search_counts(self._h, qp, nqp, n, B, op, _stream(queries, out)))
+        return out
+
+    # ---- f1: float-descriptor path (RootSIFT / scaled SIFT in fp16, tcgen05 kind::f16)
+    def f16_prepare(self, sift, rootsift: bool = True, scale: float = 1.0, out=None):
+        """u8 SIFT [..., 128] -> fp16 [..., 128] (RootSIFT if asked, times `scale`), on the GPU.
+        Returns a numpy float16 array unless ``out`` (float16 numpy / torch, host or device) is given."""
+        shp = _shape(sift)
+        assert shp[-1] == 128
+        rows = int(np.prod(shp[:-1]))
+        sp, k1 = _ptr(sift, np.uint8)
+        if out is None:
+            out = np.empty(shp, np.float16)
+        op, k2 = _ptr(out)
+        _check(self._lib.tid_f16_prepare(self._h, sp, rows, 1 if rootsift else 0, float(scale), op,
+                                         _stream(sift, out)))
+        return out
+
+    def f16_search_counts(self, q16, r16, out=None):
+        """fp16 queries [B][n][128] x fp16 references [R][m][128] -> counts uint32 [B][R]."""
+        B, n, d = _shape(q16)
+        R, m, d2 = _shape(r16)
+        assert d == 128 and d2 == 128
+        qp, k1 = _ptr(q16, np.float16)
+        rp, k2 = _ptr(r16, np.float16)
+        if out is None:
+            out = np.empty((B, R), np.uint32)
+        op, k3 = _ptr(out)
+        _check(self._lib.tid_f16_search_counts(self._h, qp, n, B, rp, m, R, op, _stream(q16, out)))
         return out
 
     def verify(self, q, r, n_q=None, m_r=None, want_nn: bool = True, out=None):

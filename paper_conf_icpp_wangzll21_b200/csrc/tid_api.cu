@@ -170,6 +170,24 @@ tid_status make_xmap(CUtensorMap* map, const void* base, int64_t count, int64_t 
   return TID_OK;
 }
 
+// fp16 tensor [count][rows][128] -> 3-D map with box {64 elements = 128 B, box_rows, 1}, SWIZZLE_128B
+// (a row's two K-halves are loaded as two tiles).
+tid_status make_map_f16(CUtensorMap* map, const void* base, int64_t count, int64_t rows, int box_rows) {
+  PFN_encodeTiled_t fn = encode_fn();
+  if (!fn) return fail(TID_ECUDA, "cuTensorMapEncodeTiled entry point unavailable");
+  if (reinterpret_cast<uintptr_t>(base) % 16) return fail(TID_EINVAL, "fp16 buffer must be 16-byte aligned");
+  cuuint64_t dims[3] = {static_cast<cuuint64_t>(kDim), static_cast<cuuint64_t>(rows),
+                        static_cast<cuuint64_t>(std::max<int64_t>(count, 1))};
+  cuuint64_t strides[2] = {static_cast<cuuint64_t>(kDim * 2), static_cast<cuuint64_t>(rows * kDim * 2)};
+  cuuint32_t box[3] = {64, static_cast<cuuint32_t>(box_rows), 1};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_UINT16, 3, const_cast<void*>(base), dims, strides, box, estr,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(TID_ECUDA, "cuTensorMapEncodeTiled (fp16) failed (%d)", static_cast<int>(r));
+  return TID_OK;
+}
+
 bool is_device_ptr(const void* p) {
   if (!p) return false;
   cudaPointerAttributes a;
@@ -217,6 +235,7 @@ struct tid_index {
       ws_kp, ws_mr;
   DevBuf stage_desc[2], stage_colkey[2], stage_kp[2], stage_extra[2];
   DevBuf ws_qs;                   // shifted queries q' = q ^ 0x80 (search)
+  DevBuf ws_f16q, ws_f16r, ws_f16nq, ws_f16nr, ws_f16in;  // f1 float path
   int64_t host_chunk = 0;
   tid_tuning tune{};
   ncclComm_t comm = nullptr;
@@ -649,7 +668,8 @@ tid_status tid_index_destroy(tid_index* idx) {
                     &idx->ws_gather, &idx->ws_ids, &idx->ws_cnts, &idx->ws_r, &idx->ws_colkey, &idx->ws_nn,
                     &idx->ws_kp, &idx->ws_mr, &idx->stage_desc[0], &idx->stage_desc[1], &idx->stage_colkey[0],
                     &idx->stage_colkey[1], &idx->stage_kp[0], &idx->stage_kp[1], &idx->stage_extra[0],
-                    &idx->stage_extra[1], &idx->ws_qs};
+                    &idx->stage_extra[1], &idx->ws_qs, &idx->ws_f16q, &idx->ws_f16r, &idx->ws_f16nq,
+                    &idx->ws_f16nr, &idx->ws_f16in};
   for (DevBuf* b : bufs) b->release();
   for (auto& pr : idx->prof_ev) { cudaEventDestroy(pr.first); cudaEventDestroy(pr.second); }
   for (int b = 0; b < 2; ++b) {
@@ -1114,6 +1134,85 @@ tid_status tid_merge_topk(tid_index* idx, const int64_t* ids_in, const int32_t* 
   TRY(copy_out(idx, ids_out, dids, static_cast<size_t>(B) * k * 8, s, &host_out));
   TRY(copy_out(idx, counts_out, dcnt, static_cast<size_t>(B) * k * 4, s, &host_out));
   if (host_out) CU(cudaStreamSynchronize(s));
+  return TID_OK;
+}
+
+// ---------------------------------------------------------------- f1: float-descriptor path
+tid_status tid_f16_prepare(tid_index* idx, const uint8_t* sift, int64_t rows, int32_t rootsift, float scale,
+                           uint16_t* out, void* stream) {
+  if (!idx || !sift || !out) return fail(TID_EINVAL, "null argument");
+  if (rows < 0) return fail(TID_EINVAL, "rows < 0");
+  if (!(scale > 0.0f)) return fail(TID_EINVAL, "scale must be > 0");
+  if (rows == 0) return TID_OK;
+  TRY(set_device(idx));
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const size_t in_b = static_cast<size_t>(rows) * kDim, out_b = in_b * 2;
+  const uint8_t* din = sift;
+  if (!is_device_ptr(sift)) {
+    TRY(idx->ws_f16in.ensure(in_b, "f16 prepare input"));
+    TRY(copy_in(idx, idx->ws_f16in.p, sift, in_b, s));
+    din = idx->ws_f16in.as<uint8_t>();
+  }
+  const bool dev_out = is_device_ptr(out);
+  void* dout = out;
+  if (!dev_out) {
+    TRY(idx->ws_f16r.ensure(out_b, "f16 prepare output"));
+    dout = idx->ws_f16r.p;
+  }
+  CU(launch_f16_prepare(din, rows, rootsift, scale, dout, s));
+  count_kernel(idx);
+  if (!dev_out) {
+    bool host_out = false;
+    TRY(copy_out(idx, out, dout, out_b, s, &host_out));
+    CU(cudaStreamSynchronize(s));
+  }
+  return TID_OK;
+}
+
+tid_status tid_f16_search_counts(tid_index* idx, const uint16_t* q, int32_t n, int64_t B, const uint16_t* r,
+                                 int32_t m, int64_t R, uint32_t* counts_out, void* stream) {
+  if (!idx || !q || !r || !counts_out) return fail(TID_EINVAL, "null argument");
+  if (n < 1 || n > idx->cfg.query_kp_max) return fail(TID_EINVAL, "n=%d outside 1..query_kp_max", n);
+  if (m < 2 || m > kBN) return fail(TID_EINVAL, "m=%d outside 2..256 (float path)", m);
+  if (B < 1 || R < 1) return fail(TID_EINVAL, "B and R must be >= 1");
+  if (B > (1LL << 30) || R > (1LL << 31) - 1) return fail(TID_EINVAL, "B or R too large");
+  TRY(set_device(idx));
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const int T = static_cast<int>(ceil_div(n, kBM));
+  const size_t qb = static_cast<size_t>(B) * n * kDim * 2, rb = static_cast<size_t>(R) * m * kDim * 2;
+  const uint16_t* dq = q;
+  const uint16_t* dr = r;
+  if (!is_device_ptr(q)) {
+    TRY(idx->ws_f16q.ensure(qb, "f16 queries"));
+    TRY(copy_in(idx, idx->ws_f16q.p, q, qb, s));
+    dq = idx->ws_f16q.as<uint16_t>();
+  }
+  if (!is_device_ptr(r)) {
+    TRY(idx->ws_f16r.ensure(rb, "f16 references"));
+    TRY(copy_in(idx, idx->ws_f16r.p, r, rb, s));
+    dr = idx->ws_f16r.as<uint16_t>();
+  }
+  TRY(idx->ws_f16nq.ensure(static_cast<size_t>(B) * T * kBM * 4, "f16 query norms"));
+  TRY(idx->ws_f16nr.ensure(static_cast<size_t>(R) * kBN * 4, "f16 reference norms"));
+  CU(launch_f16_norms(dq, B, n, T * kBM, 0.0f, idx->ws_f16nq.as<float>(), s));
+  CU(launch_f16_norms(dr, R, m, kBN, __builtin_inff(), idx->ws_f16nr.as<float>(), s));
+  count_kernel(idx, 2);
+  const bool dev_counts = is_device_ptr(counts_out);
+  TRY(idx->ws_counts.ensure(static_cast<size_t>(B) * R * 4, "count matrix"));
+  uint32_t* counts = dev_counts ? counts_out : idx->ws_counts.as<uint32_t>();
+  CU(cudaMemsetAsync(counts, 0, static_cast<size_t>(B) * R * 4, s));
+  CUtensorMap qmap, rmap;
+  TRY(make_map_f16(&qmap, dq, B, n, kBM));
+  TRY(make_map_f16(&rmap, dr, R, m, kBN));
+  CU(launch_f16_match(qmap, rmap, idx->ws_f16nr.as<float>(), idx->ws_f16nq.as<float>(), static_cast<int32_t>(B), n,
+                      T, R, idx->cfg.ratio_num * idx->cfg.ratio_num, idx->cfg.ratio_den * idx->cfg.ratio_den, counts,
+                      idx->num_sms, s));
+  count_kernel(idx);
+  if (!dev_counts) {
+    bool host_out = false;
+    TRY(copy_out(idx, counts_out, counts, static_cast<size_t>(B) * R * 4, s, &host_out));
+    CU(cudaStreamSynchronize(s));
+  }
   return TID_OK;
 }
 

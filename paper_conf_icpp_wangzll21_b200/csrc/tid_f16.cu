@@ -1,0 +1,336 @@
+// tid_f16.cu — SURVEY §8 row f1: the paper's float-descriptor path on sm_100a.
+//
+//   prepare : SIFT u8 -> [RootSIFT (L1-normalise, element-wise sqrt; §5.1)] -> x * scale
+//             (the fp16 scale factor, 2^-7 in practice; §4.2) -> fp16 (RNE).
+//   match   : TMA -> tcgen05.mma.kind::f16 (fp16 x fp16 -> fp32 in TMEM; the paper's HGEMM, Alg. 2
+//             step 1 P:648) -> epilogue d = N_Q + N_R - 2 q.r in fp32 (Alg. 1 / Eq. 1; for RootSIFT
+//             N = 1 and this is Alg. 2's sqrt(2 + A) ordering) -> exact two-partition top-2
+//             of d (non-negative fp32 orders like its bit pattern) -> ratio test den^2 d1 < num^2 d2
+//             (compared in fp64) -> count per (query, reference).
+//
+// One CTA per job = (reference r, range of queries); warp 0 TMA producer, warp 1 MMA issuer,
+// warps 2..5 epilogue (one per TMEM lane quarter).  The reference tile (256 keypoints x 128 fp16 =
+// 64 KiB, two SWIZZLE_128B K-halves) stays in shared memory for the job; query tiles (128 x 128
+// fp16) stream through a 2-stage ring; the accumulator (128 x 256 fp32) is double-buffered in TMEM.
+// Not the tuned path (the integer kernel is): this row is about the method's float variant.
+#include "tid_kernels.cuh"
+
+#include <cuda_fp16.h>
+
+#include <climits>
+
+namespace tid {
+namespace f16 {
+
+constexpr int kThreads = 32 * 6;
+constexpr int kHalfBytes = 128;                     // one SWIZZLE_128B row = 64 fp16
+constexpr uint32_t kRHalf = kBN * kHalfBytes;       // 32 KiB: 256 reference rows x 64 fp16
+constexpr uint32_t kQHalf = kBM * kHalfBytes;       // 16 KiB: 128 query rows x 64 fp16
+constexpr int kStages = 2;
+
+struct Plan {
+  static constexpr uint32_t kR = 0;                            // 2 halves
+  static constexpr uint32_t kQ = kR + 2 * kRHalf;              // kStages x 2 halves
+  static constexpr uint32_t kNR = kQ + kStages * 2 * kQHalf;   // 256 fp32 reference norms
+  static constexpr uint32_t kBar = kNR + kBN * 4;
+  static constexpr uint32_t kQFull = kBar, kQEmpty = kBar + 8 * kStages;
+  static constexpr uint32_t kRFull = kQEmpty + 8 * kStages, kREmpty = kRFull + 8;
+  static constexpr uint32_t kTFull = kREmpty + 8, kTEmpty = kTFull + 16;
+  static constexpr uint32_t kTmemPtr = kTEmpty + 16;
+  static constexpr uint32_t kAlloc = kTmemPtr + 16 + 1024;
+};
+
+__device__ __forceinline__ uint32_t su32(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
+__device__ __forceinline__ void bar_init(uint32_t b, uint32_t c) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(b), "r"(c) : "memory");
+}
+__device__ __forceinline__ void bar_expect(uint32_t b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(b), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bar_arrive(uint32_t b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(b) : "memory");
+}
+__device__ __forceinline__ void bar_wait(uint32_t b, uint32_t par) {
+  asm volatile(
+      "{\n\t.reg .pred P1;\n\tW:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+      "@P1 bra D;\n\tbra W;\n\tD:\n\t}" ::"r"(b), "r"(par) : "memory");
+}
+__device__ __forceinline__ void tma3(uint32_t dst, const CUtensorMap* m, uint32_t bar, int c0, int c1, int c2) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5}], [%2];"
+      ::"r"(dst), "l"(reinterpret_cast<uint64_t>(m)), "r"(bar), "r"(c0), "r"(c1), "r"(c2) : "memory");
+}
+__device__ __forceinline__ void bulk(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
+}
+__device__ __forceinline__ uint64_t desc128(uint32_t addr) {
+  return static_cast<uint64_t>((addr & 0x3FFFF) >> 4) | (uint64_t(1) << 16) | (uint64_t(1024 >> 4) << 32) |
+         (uint64_t(1) << 46) | (uint64_t(2) << 61);
+}
+// kind::f16: D = F32 (bits 4-5 = 1), A = B = F16 (0), K-major, N = 256, M = 128.
+constexpr uint32_t kIdesc = (1u << 4) | (uint32_t(kBN >> 3) << 17) | (uint32_t(kBM >> 4) << 24);
+
+// D (+)= Q . R^T over K = 128 fp16: per K-half (one SWIZZLE_128B tile) four K = 16 steps of 32 B.
+__device__ __forceinline__ void mma_unit(uint32_t d, uint64_t a0, uint64_t a1, uint64_t b0, uint64_t b1, uint32_t bar) {
+  asm volatile(
+      "{\n\t.reg .pred e, f, t;\n\t"
+      "setp.ne.b32 f, 0, 0;\n\tsetp.eq.b32 t, 0, 0;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %3, %5, f;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %7, %8, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %9, %10, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %11, %12, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %2, %4, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %13, %14, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %15, %16, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %17, %18, %5, t;\n\t"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%6];\n\t}"
+      ::"r"(d), "l"(a0), "l"(a1), "l"(b0), "l"(b1), "r"(kIdesc), "r"(bar),
+        "l"(a0 + 2), "l"(b0 + 2), "l"(a0 + 4), "l"(b0 + 4), "l"(a0 + 6), "l"(b0 + 6),
+        "l"(a1 + 2), "l"(b1 + 2), "l"(a1 + 4), "l"(b1 + 4), "l"(a1 + 6), "l"(b1 + 6)
+      : "memory");
+}
+__device__ __forceinline__ void commit(uint32_t bar) {
+  asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+               "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(bar)
+               : "memory");
+}
+#define F16_OUT32(v)                                                                                           \
+  "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]), "=r"(v[8]),    \
+      "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]), "=r"(v[16]),    \
+      "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]), "=r"(v[24]),   \
+      "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+__device__ __forceinline__ void ld32(uint32_t taddr, uint32_t (&v)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
+      "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : F16_OUT32(v) : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+  for (int i = 0; i < 32; ++i) asm volatile("" : "+r"(v[i]));
+}
+
+__device__ __forceinline__ int mn3(int a, int b, int c) { return __vimin3_s32(a, b, c); }
+
+__global__ void __launch_bounds__(kThreads, 1)
+    match_f16_kernel(const __grid_constant__ CUtensorMap qmap, const __grid_constant__ CUtensorMap rmap,
+                     const float* __restrict__ nr_all, const float* __restrict__ nq_all, int32_t B, int32_t n,
+                     int32_t T, int64_t R, int32_t q_per_job, uint32_t num2, uint32_t den2,
+                     uint32_t* __restrict__ counts) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const uint32_t sb = su32(smem);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  auto qfull = [&](int i) { return sb + Plan::kQFull + 8 * i; };
+  auto qempty = [&](int i) { return sb + Plan::kQEmpty + 8 * i; };
+  const uint32_t rfull = sb + Plan::kRFull, rempty = sb + Plan::kREmpty;
+  auto tfull = [&](int i) { return sb + Plan::kTFull + 8 * i; };
+  auto tempty = [&](int i) { return sb + Plan::kTEmpty + 8 * i; };
+  uint32_t* tptr = reinterpret_cast<uint32_t*>(smem + Plan::kTmemPtr);
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kStages; ++i) { bar_init(qfull(i), 1); bar_init(qempty(i), 1); }
+    bar_init(rfull, 1);
+    bar_init(rempty, 1 + 4);
+    for (int i = 0; i < 2; ++i) { bar_init(tfull(i), 1); bar_init(tempty(i), 4); }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(su32(tptr)) : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = *tptr;
+  const int64_t qchunks = (B + q_per_job - 1) / q_per_job;
+  const int64_t n_jobs = R * qchunks;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      uint32_t qc = 0, rc = 0;
+      for (int64_t j = blockIdx.x; j < n_jobs; j += gridDim.x, ++rc) {
+        const int64_t r = j / qchunks;
+        const int q0 = static_cast<int>(j % qchunks) * q_per_job, nq = min(q_per_job, B - q0);
+        bar_wait(rempty, (rc & 1) ^ 1);
+        bar_expect(rfull, 2 * kRHalf + kBN * 4);
+        tma3(sb + Plan::kR, &rmap, rfull, 0, 0, static_cast<int>(r));
+        tma3(sb + Plan::kR + kRHalf, &rmap, rfull, 64, 0, static_cast<int>(r));
+        bulk(sb + Plan::kNR, nr_all + r * kBN, kBN * 4, rfull);
+        for (int t = 0; t < nq * T; ++t, ++qc) {
+          const int st = qc % kStages;
+          bar_wait(qempty(st), ((qc / kStages) & 1) ^ 1);
+          bar_expect(qfull(st), 2 * kQHalf);
+          const uint32_t dst = sb + Plan::kQ + st * 2 * kQHalf;
+          tma3(dst, &qmap, qfull(st), 0, (t % T) * kBM, q0 + t / T);
+          tma3(dst + kQHalf, &qmap, qfull(st), 64, (t % T) * kBM, q0 + t / T);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    uint32_t qc = 0, rc = 0, uc = 0;
+    for (int64_t j = blockIdx.x; j < n_jobs; j += gridDim.x, ++rc) {
+      const int q0 = static_cast<int>(j % qchunks) * q_per_job, nq = min(q_per_job, B - q0);
+      bar_wait(rfull, rc & 1);
+      const uint64_t b0 = desc128(sb + Plan::kR), b1 = desc128(sb + Plan::kR + kRHalf);
+      for (int t = 0; t < nq * T; ++t, ++qc, ++uc) {
+        const int st = qc % kStages, buf = uc & 1;
+        bar_wait(qfull(st), (qc / kStages) & 1);
+        bar_wait(tempty(buf), ((uc >> 1) & 1) ^ 1);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        const uint32_t qa = sb + Plan::kQ + st * 2 * kQHalf;
+        mma_unit(tmem + buf * kBN, desc128(qa), desc128(qa + kQHalf), b0, b1, tfull(buf));
+        commit(qempty(st));
+      }
+      commit(rempty);
+    }
+  } else {
+    const int quarter = warp & 3;
+    const uint32_t tq = tmem + (static_cast<uint32_t>(quarter * 32) << 16);
+    const float* nr_s = reinterpret_cast<const float*>(smem + Plan::kNR);
+    uint32_t rc = 0, uc = 0;
+    for (int64_t j = blockIdx.x; j < n_jobs; j += gridDim.x, ++rc) {
+      const int64_t r = j / qchunks;
+      const int q0 = static_cast<int>(j % qchunks) * q_per_job, nq = min(q_per_job, B - q0);
+      bar_wait(rfull, rc & 1);
+      uint32_t cnt = 0;
+      for (int t = 0; t < nq * T; ++t, ++uc) {
+        const int buf = uc & 1, qi = q0 + t / T, row = (t % T) * kBM + quarter * 32 + lane;
+        const bool valid = row < n;
+        const float nqv = nq_all[static_cast<int64_t>(qi) * T * kBM + row];
+        bar_wait(tfull(buf), (uc >> 1) & 1);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        // two-partition exact top-2 (see tid_kernels.cu) over the bit patterns of d >= 0
+        int Rm[16];
+#pragma unroll
+        for (int b = 0; b < 16; ++b) Rm[b] = INT_MAX;
+        int T1 = INT_MAX, T2 = INT_MAX;
+#pragma unroll 1
+        for (int c = 0; c < kBN / 32; ++c) {
+          uint32_t v[32];
+          ld32(tq + buf * kBN + c * 32, v);
+          int k[32];
+#pragma unroll
+          for (int i = 0; i < 32; ++i) {
+            const float d = fmaxf(fmaf(-2.0f, __uint_as_float(v[i]), nr_s[c * 32 + i]) + nqv, 0.0f);
+            k[i] = __float_as_int(d);
+          }
+          const int x = min(mn3(mn3(k[0], k[1], k[2]), mn3(k[3], k[4], k[5]), mn3(k[6], k[7], k[8])),
+                            mn3(mn3(k[9], k[10], k[11]), mn3(k[12], k[13], k[14]), k[15]));
+          const int y = min(mn3(mn3(k[16], k[17], k[18]), mn3(k[19], k[20], k[21]), mn3(k[22], k[23], k[24])),
+                            mn3(mn3(k[25], k[26], k[27]), mn3(k[28], k[29], k[30]), k[31]));
+#pragma unroll
+          for (int b = 0; b < 16; ++b) Rm[b] = mn3(Rm[b], k[b], k[b + 16]);
+          const int lo = min(x, y), hi = max(x, y);
+          T2 = mn3(T2, max(T1, lo), hi);
+          T1 = min(T1, lo);
+        }
+        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+        __syncwarp();
+        if (lane == 0) bar_arrive(tempty(buf));
+        int rm[4], cm[4];
+#pragma unroll
+        for (int a = 0; a < 4; ++a) {
+          rm[a] = min(mn3(Rm[4 * a], Rm[4 * a + 1], Rm[4 * a + 2]), Rm[4 * a + 3]);
+          cm[a] = min(mn3(Rm[a], Rm[a + 4], Rm[a + 8]), Rm[a + 12]);
+        }
+        const int sr = mn3(max(min(rm[0], rm[1]), min(rm[2], rm[3])), max(rm[0], rm[1]), max(rm[2], rm[3]));
+        const int sc = mn3(max(min(cm[0], cm[1]), min(cm[2], cm[3])), max(cm[0], cm[1]), max(cm[2], cm[3]));
+        const float d1 = __int_as_float(T1), d2 = __int_as_float(mn3(T2, sr, sc));
+        // ratio test in fp64 on the fp32 distances; padded columns are +inf
+        const bool pass = valid && isfinite(d2) && double(den2) * double(d1) < double(num2) * double(d2);
+        cnt += __popc(__ballot_sync(0xffffffffu, pass));
+        if (t % T == T - 1) {
+          if (lane == 0 && cnt) atomicAdd(counts + static_cast<int64_t>(qi) * R + r, cnt);
+          cnt = 0;
+        }
+      }
+      __syncwarp();
+      if (lane == 0) bar_arrive(rempty);
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  if (warp == 1) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem) : "memory");
+  }
+}
+
+// Squared norms in fp32 of fp16 rows: out[item][row] for rows < valid, `pad` beyond (items of
+// `rows` rows, padded to `rows_pad`).
+__global__ void norms_kernel(const __half* __restrict__ x, int64_t items, int32_t rows, int32_t rows_pad,
+                             float pad, float* __restrict__ out) {
+  const int64_t g = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (g >= items * rows_pad) return;
+  const int64_t it = g / rows_pad;
+  const int row = static_cast<int>(g % rows_pad);
+  float acc = pad;
+  if (row < rows) {
+    const __half2* p = reinterpret_cast<const __half2*>(x + (it * rows + row) * kDim);
+    acc = 0.0f;
+#pragma unroll 8
+    for (int i = 0; i < kDim / 2; ++i) {
+      const float2 f = __half22float2(p[i]);
+      acc = fmaf(f.x, f.x, acc);
+      acc = fmaf(f.y, f.y, acc);
+    }
+  }
+  out[g] = acc;
+}
+
+// SIFT u8 -> [RootSIFT] -> * scale -> fp16 (round to nearest even).  One thread per row.
+__global__ void prepare_kernel(const uint8_t* __restrict__ sift, int64_t rows, int32_t rootsift, float scale,
+                               __half* __restrict__ out) {
+  const int64_t r = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (r >= rows) return;
+  const uint8_t* s = sift + r * kDim;
+  float sum = 0.0f;
+  if (rootsift)
+    for (int i = 0; i < kDim; ++i) sum += static_cast<float>(s[i]);
+  for (int i = 0; i < kDim; ++i) {
+    float v = static_cast<float>(s[i]);
+    if (rootsift) v = sum > 0.0f ? sqrtf(v / sum) : 0.0f;
+    out[r * kDim + i] = __float2half_rn(v * scale);
+  }
+}
+
+}  // namespace f16
+
+size_t f16_smem_bytes() { return f16::Plan::kAlloc; }
+
+cudaError_t launch_f16_prepare(const uint8_t* sift, int64_t rows, int32_t rootsift, float scale, void* out,
+                               cudaStream_t s) {
+  if (rows <= 0) return cudaSuccess;
+  f16::prepare_kernel<<<static_cast<unsigned>((rows + 127) / 128), 128, 0, s>>>(sift, rows, rootsift, scale,
+                                                                                 static_cast<__half*>(out));
+  return cudaGetLastError();
+}
+
+cudaError_t launch_f16_norms(const void* x, int64_t items, int32_t rows, int32_t rows_pad, float pad, float* out,
+                             cudaStream_t s) {
+  const int64_t total = items * rows_pad;
+  if (total <= 0) return cudaSuccess;
+  f16::norms_kernel<<<static_cast<unsigned>((total + 255) / 256), 256, 0, s>>>(static_cast<const __half*>(x), items,
+                                                                               rows, rows_pad, pad, out);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_f16_match(const CUtensorMap& qmap, const CUtensorMap& rmap, const float* nr, const float* nq,
+                             int32_t B, int32_t n, int32_t T, int64_t R, uint32_t num2, uint32_t den2,
+                             uint32_t* counts, int num_sms, cudaStream_t s) {
+  cudaError_t e = cudaFuncSetAttribute(f16::match_f16_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(f16::Plan::kAlloc));
+  if (e != cudaSuccess) return e;
+  // queries per job: enough jobs to fill the SMs, otherwise all queries reuse the resident reference
+  int32_t qpj = B;
+  while (R * ((B + qpj - 1) / qpj) < 2LL * num_sms && qpj > 1) qpj = (qpj + 1) / 2;
+  const int64_t jobs = R * ((B + qpj - 1) / qpj);
+  const int grid = static_cast<int>(jobs < num_sms ? jobs : num_sms);
+  f16::match_f16_kernel<<<grid, f16::kThreads, f16::Plan::kAlloc, s>>>(qmap, rmap, nr, nq, B, n, T, R, qpj, num2,
+                                                                        den2, counts);
+  return cudaGetLastError();
+}
+
+}  // namespace tid

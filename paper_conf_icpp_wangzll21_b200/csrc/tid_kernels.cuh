@@ -112,4 +112,14 @@ void launch_merge(const uint64_t* cand, int32_t L, int64_t B, int32_t k, int64_t
 void launch_pack_lists(const int64_t* ids, const int32_t* counts, int64_t n, uint64_t* keys, cudaStream_t s);
 size_t match_smem_bytes();
 
+// f1 float path (tid_f16.cu)
+size_t f16_smem_bytes();
+cudaError_t launch_f16_prepare(const uint8_t* sift, int64_t rows, int32_t rootsift, float scale, void* out,
+                               cudaStream_t s);
+cudaError_t launch_f16_norms(const void* x, int64_t items, int32_t rows, int32_t rows_pad, float pad, float* out,
+                             cudaStream_t s);
+cudaError_t launch_f16_match(const CUtensorMap& qmap, const CUtensorMap& rmap, const float* nr, const float* nq,
+                             int32_t B, int32_t n, int32_t T, int64_t R, uint32_t num2, uint32_t den2,
+                             uint32_t* counts, int num_sms, cudaStream_t s);
+
 }  // namespace tid

@@ -98,8 +98,35 @@ def verify_case(P=4096, n=1000, m=1000, reps=10):
     print(json.dumps(out), flush=True)
 
 
+def f16_case(B=64, n=1000, R=20000, m=256, reps=5):
+    """Row f1: RootSIFT fp16 search counts (tcgen05 kind::f16) vs the integer path on the same
+    workload; Eq. 2 compression error of RootSIFT in fp16 on a small sample (oracle)."""
+    import torch
+    import oracle
+    refs, _ = tidgen.refs(0, R, m)
+    qs, tg = tidgen.queries(0, B, n, R_total=R, m=m)
+    idx = tid.Index(ref_kp=m, query_kp_max=n)
+    dq, dr = torch.from_numpy(qs).cuda(), torch.from_numpy(refs).cuda()
+    q16 = torch.empty(qs.shape, dtype=torch.float16, device="cuda")
+    r16 = torch.empty(refs.shape, dtype=torch.float16, device="cuda")
+    idx.f16_prepare(dq, True, 1.0, out=q16)
+    idx.f16_prepare(dr, True, 1.0, out=r16)
+    out = torch.empty((B, R), dtype=torch.int32, device="cuda")
+    ts = timed(lambda: idx.f16_search_counts(q16, r16, out=out), reps)
+    top1 = float(np.mean(out.argmax(1).cpu().numpy() == tg))
+    rq, rr = oracle.rootsift(qs[0, :200]), oracle.rootsift(refs[0])
+    err = oracle.compression_error(rq, rr, oracle.to_fp16(rq), oracle.to_fp16(rr))
+    res = {"case": "f1 RootSIFT fp16", "queries": B, "query_kp": n, "refs": R, "ref_kp": m,
+           "p50_ms": statistics.median(ts), "comparisons_per_s": B * R / (statistics.median(ts) / 1e3),
+           "planted_top1": top1, "eq2_compression_error_sample": err}
+    idx.close()
+    print(json.dumps(res), flush=True)
+
+
 def main():
-    what = sys.argv[1:] or ["c1", "c3", "c2", "sweep"]
+    what = sys.argv[1:] or ["c1", "c3", "c2", "sweep", "f16"]
+    if "f16" in what:
+        f16_case()
     if "c1" in what:
         search_case("C1", 1, 256, 64, 256, 5, reps=100)
     if "c3" in what:
