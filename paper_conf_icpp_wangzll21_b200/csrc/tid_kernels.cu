@@ -268,10 +268,10 @@ constexpr int kAxCol = kTQBase + kTQ * kQCols;
 static_assert(kAxCol + kXDim / 4 <= 512, "TMEM budget");
 
 constexpr int kProducerWarp = 0;               // warp 0: TMA producer
-constexpr int kFirstMmaWarp = 1;               // warps 1..3: MMA issuer of group mw (SMSPs 1, 2, 3)
-constexpr int kFirstEpiWarp = 1 + kNG;         // warps 4..15: epilogue, group (w-4)/4, lane quarter w%4
+constexpr int kFirstMmaWarp = 1;               // warps 1..kNG: MMA issuer of group mw
+constexpr int kFirstEpiWarp = 1 + kNG;         // then 4 warps per group; lane quarter w % 4
 // (any 4 consecutive warps cover the 4 TMEM lane quarters w % 4)
-static_assert(kNB == 2 && kNumThreads <= 512, "at most 16 warps: >= 128 registers per thread");
+static_assert(kNumThreads <= 512, "at most 16 warps: >= 128 registers per thread");
 
 // ------------------------------------------------------------------ shared memory plan
 struct SmemPlan {
@@ -578,7 +578,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     // 64-column buffers (whole warp, one elected lane).  Every warp commits the release of every
     // query tile (waiting for tiles it never used, so the stage phases stay in order).
     const int mw = warp - kFirstMmaWarp;
-    uint32_t qctr = 0, pc = 0;
+    uint32_t qctr = 0, pb = 0, pph = 0;  // next buffer of this group and its phase
     if (kFold) mbar_wait(axfull, 0);  // constant norm-term operand in TMEM
     uint32_t slot_par = 0;  // bit sl = phase parity of reference slot sl
     for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
@@ -609,18 +609,21 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             const uint64_t bd0 = smem_desc_sw128(sbase + SmemPlan::kR + sl * kRTileBytes);
 #pragma unroll 1
             for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
-              const uint32_t buf = mw * kNB + (pc & 1);
-              PROF_B(); mbar_wait(tempty(buf), ((pc >> 1) & 1) ^ 1); PROF_E(0);
+              const uint32_t buf = mw * kNB + pb;
+              PROF_B(); mbar_wait(tempty(buf), pph ^ 1); PROF_E(0);
               tc_fence_after();
               // rows kPiece*pp.. of the chunk: SWIZZLE_128B core groups of 8 rows x 128 B
               const uint64_t bd = bd0 + pp * (kPiece * kDim >> 4);
+#ifdef TID_NOMMA  // timing experiment only: no MMAs (the commit still signals the buffer)
+              if (kFold) mma_commit(tfull(buf)); else
+#endif
               if (kFold)  // + norm-term K-step: rows kPiece*pp.. of the 32-B-wide tile
                 mma_piece_fold_ts(tmem_base + buf * kPiece, at, bd, tmem_base + kAxCol,
                                   smem_desc_sw32(sbase + SmemPlan::kX + sl * kXTileBytes) + pp * (kPiece * kXDim >> 4),
                                   tfull(buf));
               else
                 mma_piece<kIdescI8>(tmem_base + buf * kPiece, ad, bd, tfull(buf));
-              ++pc;
+              if (++pb == kNB) { pb = 0; pph ^= 1; }
             }
           }
         }
@@ -655,7 +658,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     const int row_in_tile = quarter * 32 + lane;
     const int nq_ld = T * kBM;
     const bool ratio32 = p.num2 <= 511u && p.den2 <= 511u;  // den^2 * d fits 32 bits (d <= 8,323,200)
-    uint32_t mp = 0;                      // pieces consumed by this warp (buffer + phase)
+    uint32_t eb = 0, eph = 0;             // next buffer of this group to consume and its phase
     uint32_t slot_par = 0;                // bit sl = phase parity of reference slot sl
     uint32_t v[64];
 
@@ -678,12 +681,6 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         const int row = tq * kBM + row_in_tile;
         const bool valid = row < nvalid;
         const int32_t nqv = valid ? nq_row[tq * kBM] : 0;
-        // the unit after this one (same group): (ns, ntq, nqi)
-        int ns = s + kNG, ntq = tq, nqi = qi;
-        while (ns >= J.nr) {
-          ns -= J.nr;
-          if (++ntq == T) { ntq = 0; ++nqi; }
-        }
         const bool has_next = u + kNG < U;
         bool pass = false;
         if constexpr (kFold) {
@@ -699,31 +696,27 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             int T1 = INT_MIN, T2 = INT_MIN;
 #pragma unroll 1
             for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
-              const uint32_t buf = g * kNB + (mp & 1);
-              PROF_B(); mbar_wait(tfull(buf), (mp >> 1) & 1); PROF_E(0);
+              const uint32_t buf = g * kNB + eb;
+              PROF_B(); mbar_wait(tfull(buf), eph); PROF_E(0);
               tc_fence_after();
-#pragma unroll
-              for (int h = 0; h < kPiece / 64; ++h) {
-                tmem_ld64(taddr_q + buf * kPiece + h * 64, v);
-                tmem_wait_ld();
-                reg_fence64(v);
-                if (h == kPiece / 64 - 1) {  // the piece is in registers: buffer free
-                  tc_fence_before();
-                  __syncwarp();
-                  if (lane == 0) mbar_arrive(tempty(buf));
-                  ++mp;
-                }
-                PROF_B();
-                const int base = pp * kPiece + h * 64;
-                if (kpc >= kBN) {  // full chunk (the common case): no masking
-                  scan32_fold<false>(v, 32, R, T1, T2);
-                  scan32_fold<false>(v + 32, 32, R, T1, T2);
-                } else {
-                  scan32_fold<true>(v, kpc - base, R, T1, T2);
-                  scan32_fold<true>(v + 32, kpc - base - 32, R, T1, T2);
-                }
-                PROF_E(1);
+              tmem_ld64(taddr_q + buf * kPiece, v);
+              tmem_wait_ld();
+              reg_fence64(v);
+              tc_fence_before();  // the piece is in registers: buffer free
+              __syncwarp();
+              if (lane == 0) mbar_arrive(tempty(buf));
+              if (++eb == kNB) { eb = 0; eph ^= 1; }
+              PROF_B();
+              if (kpc >= kBN) {  // full chunk (the common case): no masking
+#ifndef TID_NOSCAN
+                scan32_fold<false>(v, 32, R, T1, T2);
+                scan32_fold<false>(v + 32, 32, R, T1, T2);
+#endif
+              } else {
+                scan32_fold<true>(v, kpc - pp * kPiece, R, T1, T2);
+                scan32_fold<true>(v + 32, kpc - pp * kPiece - 32, R, T1, T2);
               }
+              PROF_E(1);
             }
             PROF_B();
             int x1, x2;
@@ -770,8 +763,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           int T1 = INT_MAX, T2 = INT_MAX;
 #pragma unroll 1
           for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
-            const uint32_t buf = g * kNB + (mp & 1);
-            PROF_B(); mbar_wait(tfull(buf), (mp >> 1) & 1); PROF_E(0);
+            const uint32_t buf = g * kNB + eb;
+            PROF_B(); mbar_wait(tfull(buf), eph); PROF_E(0);
             tc_fence_after();
             // x64 loads; the buffer is released as soon as its last load has landed
 #pragma unroll
@@ -783,7 +776,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(tempty(buf));
-                ++mp;
+                if (++eb == kNB) { eb = 0; eph ^= 1; }
               }
               PROF_B();
               scan32_regs(v, ck + (pp * kPiece + h * 64) * 4, R, T1, T2);
@@ -825,6 +818,12 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         }
         }
         cnt += __popc(__ballot_sync(0xffffffffu, pass));
+        // the unit after this one (same group): (ns, ntq, nqi)
+        int ns = s + kNG, ntq = tq, nqi = qi;
+        while (ns >= J.nr) {
+          ns -= J.nr;
+          if (++ntq == T) { ntq = 0; ++nqi; }
+        }
         // flush the count when the group's next unit is another (query, reference) pair
         if (!has_next || ns != s || nqi != qi) {
           if (lane == 0 && cnt) {

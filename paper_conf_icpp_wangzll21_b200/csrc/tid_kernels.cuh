@@ -26,12 +26,15 @@ constexpr int kMaxSlots = 4;       // resident reference chunks per CTA
 #ifndef TID_NG
 #define TID_NG 3
 #endif
+#ifndef TID_NB
+#define TID_NB 2
+#endif
 #ifndef TID_PIECE
 #define TID_PIECE 64
 #endif
 constexpr int kNG = TID_NG;                    // epilogue groups of 4 warps (one per TMEM lane quarter)
 constexpr int kPiece = TID_PIECE;              // accumulator columns per MMA piece (MMA N)
-constexpr int kNB = 2;                         // TMEM buffers per group (double buffered)
+constexpr int kNB = TID_NB;                    // TMEM buffers per group
 constexpr int kTmemBufs = kNG * kNB;           // 6 buffers of 64 columns (384 of the 512 allocated)
 static_assert(kTmemBufs * kPiece <= 512, "TMEM has 512 columns");
 constexpr int kPiecesPerChunk = kBN / kPiece;  // 4 pieces per 256-column reference chunk
