@@ -699,7 +699,9 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               const uint32_t buf = g * kNB + eb;
               PROF_B(); mbar_wait(tfull(buf), eph); PROF_E(0);
               tc_fence_after();
+#ifndef TID_NOLOAD  // timing experiment only: scan stale registers (wrong results)
               tmem_ld64(taddr_q + buf * kPiece, v);
+#endif
               tmem_wait_ld();
               reg_fence64(v);
               tc_fence_before();  // the piece is in registers: buffer free
