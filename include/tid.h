@@ -175,9 +175,11 @@ tid_status tid_merge_topk(tid_index* idx, const int64_t* ids_in, const int32_t* 
  *
  * tid_f16_search_counts: good-match counts of B fp16 queries [B][n][128] against R fp16 references
  *   [R][m][128] (host or device; n <= query_kp_max, 2 <= m <= 256) -> counts_out uint32 [B][R].
- *   The product q.r runs on tcgen05.mma.kind::f16 with fp32 accumulation; d = N_Q + N_R - 2 q.r in
- *   fp32 (N in fp32 from the fp16 values); 2-NN per query row; ratio test
- *   den^2 * d1 < num^2 * d2 compared in fp64.  Counts equal the exact float64 definition
+ *   The product q.r runs on tcgen05.mma.kind::f16 with fp32 accumulation; a ninth K-step adds
+ *   C - N_R / 2 (N_R in fp32 from the fp16 values, split into three fp16 terms; C = power of two
+ *   >= max N_R / 2), so d = N_Q + 2C - 2 X with X = C + q.r - N_R / 2 >= 0 read straight from the
+ *   accumulator; 2-NN per query row; ratio test den^2 * d1 < num^2 * d2 with d computed and
+ *   compared in fp64 from the fp32 X.  Counts equal the exact float64 definition
  *   on the same fp16 values except where fp32 rounding moves a ratio across the threshold
  *   (acceptance: within +-1 for >= 99.9% of pairs; exact for u8 SIFT x 2^-k).
  */

@@ -1193,19 +1193,25 @@ tid_status tid_f16_search_counts(tid_index* idx, const uint16_t* q, int32_t n, i
     dr = idx->ws_f16r.as<uint16_t>();
   }
   TRY(idx->ws_f16nq.ensure(static_cast<size_t>(B) * T * kBM * 4, "f16 query norms"));
-  TRY(idx->ws_f16nr.ensure(static_cast<size_t>(R) * kBN * 4, "f16 reference norms"));
+  // norm-term operand (R x 256 rows x 32 B) + the scalars max N_R (bits) and C
+  const size_t xb = static_cast<size_t>(R) * kBN * 32;
+  TRY(idx->ws_f16nr.ensure(xb + 256, "f16 reference norm terms"));
+  uint8_t* xop = idx->ws_f16nr.as<uint8_t>();
+  uint32_t* nrmax = reinterpret_cast<uint32_t*>(xop + xb);
+  float* cterm = reinterpret_cast<float*>(xop + xb + 128);
   CU(launch_f16_norms(dq, B, n, T * kBM, 0.0f, idx->ws_f16nq.as<float>(), s));
-  CU(launch_f16_norms(dr, R, m, kBN, __builtin_inff(), idx->ws_f16nr.as<float>(), s));
+  CU(launch_f16_xop(dr, R, m, nrmax, xop, cterm, s));
   count_kernel(idx, 2);
   const bool dev_counts = is_device_ptr(counts_out);
   TRY(idx->ws_counts.ensure(static_cast<size_t>(B) * R * 4, "count matrix"));
   uint32_t* counts = dev_counts ? counts_out : idx->ws_counts.as<uint32_t>();
   CU(cudaMemsetAsync(counts, 0, static_cast<size_t>(B) * R * 4, s));
-  CUtensorMap qmap, rmap;
+  CUtensorMap qmap, rmap, xmap;
   TRY(make_map_f16(&qmap, dq, B, n, kBM));
   TRY(make_map_f16(&rmap, dr, R, m, kBN));
-  CU(launch_f16_match(qmap, rmap, idx->ws_f16nr.as<float>(), idx->ws_f16nq.as<float>(), static_cast<int32_t>(B), n,
-                      T, R, idx->cfg.ratio_num * idx->cfg.ratio_num, idx->cfg.ratio_den * idx->cfg.ratio_den, counts,
+  TRY(make_xmap(&xmap, xop, R, kBN));  // 32-B rows, SWIZZLE_32B (same geometry as the u8 norm digits)
+  CU(launch_f16_match(qmap, rmap, xmap, cterm, idx->ws_f16nq.as<float>(), static_cast<int32_t>(B), n, T, R,
+                      idx->cfg.ratio_num * idx->cfg.ratio_num, idx->cfg.ratio_den * idx->cfg.ratio_den, counts,
                       idx->num_sms, s));
   count_kernel(idx);
   if (!dev_counts) {

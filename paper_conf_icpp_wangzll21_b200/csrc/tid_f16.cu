@@ -8,11 +8,19 @@
 //             of d (non-negative fp32 orders like its bit pattern) -> ratio test den^2 d1 < num^2 d2
 //             (compared in fp64) -> count per (query, reference).
 //
+// Folded norms (as in the integer path): a ninth K = 16 step adds, per reference keypoint, the
+// constant C - N_R / 2 (three fp16 terms h1 + h2 + h3 against a constant A operand of ones), so
+// TMEM holds X = C + q.r - N_R / 2 >= 0 and d = N_Q + 2C - 2X.  C is the smallest power of two
+// >= max N_R / 2 of the launch, so X >= 0 and its fp32 bit pattern orders like its value: the
+// epilogue scans raw TMEM words (two largest X = two nearest columns), with no per-element
+// arithmetic.  Padded columns get h1 = -inf.  For u8 SIFT x 2^-k every term is exact.
+//
 // One CTA per job = (reference r, range of queries); warp 0 TMA producer, warp 1 MMA issuer,
-// warps 2..5 epilogue (one per TMEM lane quarter).  The reference tile (256 keypoints x 128 fp16 =
-// 64 KiB, two SWIZZLE_128B K-halves) stays in shared memory for the job; query tiles (128 x 128
-// fp16) stream through a 2-stage ring; the accumulator (128 x 256 fp32) is double-buffered in TMEM.
-// Not the tuned path (the integer kernel is): this row is about the method's float variant.
+// warps 2..9 epilogue: two warps per TMEM lane quarter, 16 lanes each (16x64b loads; a row's
+// columns are split over a thread pair as even / odd columns).  The reference tile (256 keypoints
+// x 128 fp16 = 64 KiB, two SWIZZLE_128B K-halves) and its 8 KiB norm-term tile stay in shared
+// memory for the job; query tiles (128 x 128 fp16) stream through a 2-stage ring; the
+// accumulator (128 x 256 fp32) is double-buffered in TMEM.
 #include "tid_kernels.cuh"
 
 #include <cuda_fp16.h>
@@ -22,17 +30,21 @@
 namespace tid {
 namespace f16 {
 
-constexpr int kThreads = 32 * 6;
+constexpr int kEpi = 8;                             // epilogue warps (2 per TMEM lane quarter)
+constexpr int kThreads = 32 * (2 + kEpi);
 constexpr int kHalfBytes = 128;                     // one SWIZZLE_128B row = 64 fp16
 constexpr uint32_t kRHalf = kBN * kHalfBytes;       // 32 KiB: 256 reference rows x 64 fp16
 constexpr uint32_t kQHalf = kBM * kHalfBytes;       // 16 KiB: 128 query rows x 64 fp16
-constexpr int kStages = 2;
+constexpr int kStages = 4;
+constexpr int kXH = 16;                             // fp16 per norm-term row (one K = 16 step, 32 B)
+constexpr uint32_t kXTile = kBN * kXH * 2;          // 8 KiB: 256 reference rows x 16 fp16
 
 struct Plan {
   static constexpr uint32_t kR = 0;                            // 2 halves
   static constexpr uint32_t kQ = kR + 2 * kRHalf;              // kStages x 2 halves
-  static constexpr uint32_t kNR = kQ + kStages * 2 * kQHalf;   // 256 fp32 reference norms
-  static constexpr uint32_t kBar = kNR + kBN * 4;
+  static constexpr uint32_t kX = kQ + kStages * 2 * kQHalf;    // norm-term tile (SWIZZLE_32B)
+  static constexpr uint32_t kAx = kX + kXTile;                 // constant A operand (ones)
+  static constexpr uint32_t kBar = kAx + kBM * kXH * 2;
   static constexpr uint32_t kQFull = kBar, kQEmpty = kBar + 8 * kStages;
   static constexpr uint32_t kRFull = kQEmpty + 8 * kStages, kREmpty = kRFull + 8;
   static constexpr uint32_t kTFull = kREmpty + 8, kTEmpty = kTFull + 16;
@@ -69,11 +81,18 @@ __device__ __forceinline__ uint64_t desc128(uint32_t addr) {
   return static_cast<uint64_t>((addr & 0x3FFFF) >> 4) | (uint64_t(1) << 16) | (uint64_t(1024 >> 4) << 32) |
          (uint64_t(1) << 46) | (uint64_t(2) << 61);
 }
+// K-major SWIZZLE_32B (32-byte rows, 8-row groups 256 B apart): the norm-term operands.
+__device__ __forceinline__ uint64_t desc32(uint32_t addr) {
+  return static_cast<uint64_t>((addr & 0x3FFFF) >> 4) | (uint64_t(1) << 16) | (uint64_t(256 >> 4) << 32) |
+         (uint64_t(1) << 46) | (uint64_t(6) << 61);
+}
 // kind::f16: D = F32 (bits 4-5 = 1), A = B = F16 (0), K-major, N = 256, M = 128.
 constexpr uint32_t kIdesc = (1u << 4) | (uint32_t(kBN >> 3) << 17) | (uint32_t(kBM >> 4) << 24);
 
-// D (+)= Q . R^T over K = 128 fp16: per K-half (one SWIZZLE_128B tile) four K = 16 steps of 32 B.
-__device__ __forceinline__ void mma_unit(uint32_t d, uint64_t a0, uint64_t a1, uint64_t b0, uint64_t b1, uint32_t bar) {
+// D = Q . R^T over K = 128 fp16 (per K-half, one SWIZZLE_128B tile, four K = 16 steps of 32 B),
+// then D += ones . (h1, h2, h3) (the norm-term step).
+__device__ __forceinline__ void mma_unit(uint32_t d, uint64_t a0, uint64_t a1, uint64_t b0, uint64_t b1, uint64_t ax,
+                                         uint64_t bx, uint32_t bar) {
   asm volatile(
       "{\n\t.reg .pred e, f, t;\n\t"
       "setp.ne.b32 f, 0, 0;\n\tsetp.eq.b32 t, 0, 0;\n\t"
@@ -86,10 +105,11 @@ __device__ __forceinline__ void mma_unit(uint32_t d, uint64_t a0, uint64_t a1, u
       "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %13, %14, %5, t;\n\t"
       "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %15, %16, %5, t;\n\t"
       "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %17, %18, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %19, %20, %5, t;\n\t"
       "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%6];\n\t}"
       ::"r"(d), "l"(a0), "l"(a1), "l"(b0), "l"(b1), "r"(kIdesc), "r"(bar),
         "l"(a0 + 2), "l"(b0 + 2), "l"(a0 + 4), "l"(b0 + 4), "l"(a0 + 6), "l"(b0 + 6),
-        "l"(a1 + 2), "l"(b1 + 2), "l"(a1 + 4), "l"(b1 + 4), "l"(a1 + 6), "l"(b1 + 6)
+        "l"(a1 + 2), "l"(b1 + 2), "l"(a1 + 4), "l"(b1 + 4), "l"(a1 + 6), "l"(b1 + 6), "l"(ax), "l"(bx)
       : "memory");
 }
 __device__ __forceinline__ void commit(uint32_t bar) {
@@ -102,23 +122,70 @@ __device__ __forceinline__ void commit(uint32_t bar) {
       "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]), "=r"(v[16]),    \
       "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]), "=r"(v[24]),   \
       "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
-__device__ __forceinline__ void ld32(uint32_t taddr, uint32_t (&v)[32]) {
+// 16 lanes x 128 columns (16x64b.x64): thread t holds lane (t >> 2) + 8 (t & 1) of the 16 and
+// columns 2 i + ((t >> 1) & 1), i = 0..63 (tools/ld_shape_probe.cu).
+__device__ __forceinline__ void ld16x64(uint32_t taddr, uint32_t (&v)[64]) {
   asm volatile(
-      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
-      "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
-      : F16_OUT32(v) : "r"(taddr));
+      "tcgen05.ld.sync.aligned.16x64b.x64.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
+      "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32,%33,%34,%35,%36,%37,%38,%39,%40,%41,%42,%43,%44,"
+      "%45,%46,%47,%48,%49,%50,%51,%52,%53,%54,%55,%56,%57,%58,%59,%60,%61,%62,%63}, [%64];"
+      : F16_OUT32(v), F16_OUT32((v + 32)) : "r"(taddr));
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 #pragma unroll
-  for (int i = 0; i < 32; ++i) asm volatile("" : "+r"(v[i]));
+  for (int i = 0; i < 64; ++i) asm volatile("" : "+r"(v[i]));
 }
 
-__device__ __forceinline__ int mn3(int a, int b, int c) { return __vimin3_s32(a, b, c); }
+// Two x64 loads (columns [0, 128) and [128, 256) of the same 16 lanes) with one wait.
+__device__ __forceinline__ void ld16x64x2(uint32_t taddr, uint32_t (&v)[64], uint32_t (&w)[64]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.16x64b.x64.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
+      "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32,%33,%34,%35,%36,%37,%38,%39,%40,%41,%42,%43,%44,"
+      "%45,%46,%47,%48,%49,%50,%51,%52,%53,%54,%55,%56,%57,%58,%59,%60,%61,%62,%63}, [%64];"
+      : F16_OUT32(v), F16_OUT32((v + 32)) : "r"(taddr));
+  asm volatile(
+      "tcgen05.ld.sync.aligned.16x64b.x64.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
+      "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32,%33,%34,%35,%36,%37,%38,%39,%40,%41,%42,%43,%44,"
+      "%45,%46,%47,%48,%49,%50,%51,%52,%53,%54,%55,%56,%57,%58,%59,%60,%61,%62,%63}, [%64];"
+      : F16_OUT32(w), F16_OUT32((w + 32)) : "r"(taddr + 128));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+  for (int i = 0; i < 64; ++i) asm volatile("" : "+r"(v[i]), "+r"(w[i]));
+}
+
+// Two-partition top-2 of the largest values (see tid_kernels.cu): P = 16-register halves of a
+// 32-register block, P' = position mod 16; R[b] = P' maxima, T1 >= T2 = two largest P maxima.
+__device__ __forceinline__ int mx3(int a, int b, int c) { return __vimax3_s32(a, b, c); }
+__device__ __forceinline__ int mx16(const uint32_t* k) {
+  const int a = mx3(k[0], k[1], k[2]), b = mx3(k[3], k[4], k[5]), c = mx3(k[6], k[7], k[8]);
+  const int d = mx3(k[9], k[10], k[11]), e = mx3(k[12], k[13], k[14]);
+  return max(mx3(a, b, c), mx3(d, e, static_cast<int>(k[15])));
+}
+__device__ __forceinline__ void scan32(const uint32_t* k, int (&R)[16], int& T1, int& T2) {
+  const int x = mx16(k), y = mx16(k + 16);
+#pragma unroll
+  for (int b = 0; b < 16; ++b) R[b] = mx3(R[b], k[b], k[b + 16]);
+  const int hi = max(x, y), lo = min(x, y);
+  T2 = mx3(T2, min(T1, hi), lo);
+  T1 = max(T1, hi);
+}
+__device__ __forceinline__ void finish(const int (&R)[16], int T1, int T2, int& x1, int& x2) {
+  int rm[4], cm[4];
+#pragma unroll
+  for (int a = 0; a < 4; ++a) {
+    rm[a] = max(mx3(R[4 * a], R[4 * a + 1], R[4 * a + 2]), R[4 * a + 3]);
+    cm[a] = max(mx3(R[a], R[a + 4], R[a + 8]), R[a + 12]);
+  }
+  const int sr = mx3(min(max(rm[0], rm[1]), max(rm[2], rm[3])), min(rm[0], rm[1]), min(rm[2], rm[3]));
+  const int sc = mx3(min(max(cm[0], cm[1]), max(cm[2], cm[3])), min(cm[0], cm[1]), min(cm[2], cm[3]));
+  x1 = T1;
+  x2 = mx3(T2, sr, sc);
+}
 
 __global__ void __launch_bounds__(kThreads, 1)
     match_f16_kernel(const __grid_constant__ CUtensorMap qmap, const __grid_constant__ CUtensorMap rmap,
-                     const float* __restrict__ nr_all, const float* __restrict__ nq_all, int32_t B, int32_t n,
-                     int32_t T, int64_t R, int32_t q_per_job, uint32_t num2, uint32_t den2,
-                     uint32_t* __restrict__ counts) {
+                     const __grid_constant__ CUtensorMap xmap, const float* __restrict__ cterm,
+                     const float* __restrict__ nq_all, int32_t B, int32_t n, int32_t T, int64_t R, int32_t q_per_job,
+                     uint32_t num2, uint32_t den2, uint32_t* __restrict__ counts) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const uint32_t sb = su32(smem);
@@ -129,11 +196,21 @@ __global__ void __launch_bounds__(kThreads, 1)
   auto tfull = [&](int i) { return sb + Plan::kTFull + 8 * i; };
   auto tempty = [&](int i) { return sb + Plan::kTEmpty + 8 * i; };
   uint32_t* tptr = reinterpret_cast<uint32_t*>(smem + Plan::kTmemPtr);
+  {  // constant A operand of the norm-term step: every row (1, 1, 1, 0 x 5) in both 16-B halves,
+     // so the SWIZZLE_32B layout does not matter
+    uint32_t* ax = reinterpret_cast<uint32_t*>(smem + Plan::kAx);
+    const uint32_t one2 = 0x3C003C00u, one0 = 0x00003C00u;  // fp16 pairs (1, 1), (1, 0)
+    for (int i = threadIdx.x; i < kBM * kXH / 2; i += blockDim.x) {
+      const int w = i & 3;  // 32-bit word within a 16-B half
+      ax[i] = w == 0 ? one2 : (w == 1 ? one0 : 0u);
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
   if (threadIdx.x == 0) {
     for (int i = 0; i < kStages; ++i) { bar_init(qfull(i), 1); bar_init(qempty(i), 1); }
     bar_init(rfull, 1);
-    bar_init(rempty, 1 + 4);
-    for (int i = 0; i < 2; ++i) { bar_init(tfull(i), 1); bar_init(tempty(i), 4); }
+    bar_init(rempty, 1 + kEpi);
+    for (int i = 0; i < 2; ++i) { bar_init(tfull(i), 1); bar_init(tempty(i), kEpi); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 1) {
@@ -154,10 +231,10 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int64_t r = j / qchunks;
         const int q0 = static_cast<int>(j % qchunks) * q_per_job, nq = min(q_per_job, B - q0);
         bar_wait(rempty, (rc & 1) ^ 1);
-        bar_expect(rfull, 2 * kRHalf + kBN * 4);
+        bar_expect(rfull, 2 * kRHalf + kXTile);
         tma3(sb + Plan::kR, &rmap, rfull, 0, 0, static_cast<int>(r));
         tma3(sb + Plan::kR + kRHalf, &rmap, rfull, 64, 0, static_cast<int>(r));
-        bulk(sb + Plan::kNR, nr_all + r * kBN, kBN * 4, rfull);
+        tma3(sb + Plan::kX, &xmap, rfull, 0, 0, static_cast<int>(r));
         for (int t = 0; t < nq * T; ++t, ++qc) {
           const int st = qc % kStages;
           bar_wait(qempty(st), ((qc / kStages) & 1) ^ 1);
@@ -170,6 +247,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
   } else if (warp == 1) {
     uint32_t qc = 0, rc = 0, uc = 0;
+    const uint64_t ax = desc32(sb + Plan::kAx), bx = desc32(sb + Plan::kX);
     for (int64_t j = blockIdx.x; j < n_jobs; j += gridDim.x, ++rc) {
       const int q0 = static_cast<int>(j % qchunks) * q_per_job, nq = min(q_per_job, B - q0);
       bar_wait(rfull, rc & 1);
@@ -180,70 +258,68 @@ __global__ void __launch_bounds__(kThreads, 1)
         bar_wait(tempty(buf), ((uc >> 1) & 1) ^ 1);
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         const uint32_t qa = sb + Plan::kQ + st * 2 * kQHalf;
-        mma_unit(tmem + buf * kBN, desc128(qa), desc128(qa + kQHalf), b0, b1, tfull(buf));
+#ifdef TID_NOMMA  // timing experiment only
+        commit(tfull(buf));
+#else
+        mma_unit(tmem + buf * kBN, desc128(qa), desc128(qa + kQHalf), b0, b1, ax, bx, tfull(buf));
+#endif
         commit(qempty(st));
       }
       commit(rempty);
     }
   } else {
-    const int quarter = warp & 3;
-    const uint32_t tq = tmem + (static_cast<uint32_t>(quarter * 32) << 16);
-    const float* nr_s = reinterpret_cast<const float*>(smem + Plan::kNR);
+    // warps 2..9: lane quarter warp % 4, 16-lane half (warp - 2) / 4
+    const int quarter = warp & 3, half = (warp - 2) >> 2;
+    const uint32_t tq = tmem + (static_cast<uint32_t>(quarter * 32 + 16 * half) << 16);
+    const int row_in_tile = quarter * 32 + 16 * half + (lane >> 2) + 8 * (lane & 1);
+    const double c2 = 2.0 * static_cast<double>(*cterm);
     uint32_t rc = 0, uc = 0;
+    uint32_t v[64], w[64];
     for (int64_t j = blockIdx.x; j < n_jobs; j += gridDim.x, ++rc) {
       const int64_t r = j / qchunks;
       const int q0 = static_cast<int>(j % qchunks) * q_per_job, nq = min(q_per_job, B - q0);
       bar_wait(rfull, rc & 1);
       uint32_t cnt = 0;
+      int qi = q0, tt = 0;  // query and tile of unit t (no divisions per unit)
       for (int t = 0; t < nq * T; ++t, ++uc) {
-        const int buf = uc & 1, qi = q0 + t / T, row = (t % T) * kBM + quarter * 32 + lane;
+        const int buf = uc & 1, row = tt * kBM + row_in_tile;
         const bool valid = row < n;
         const float nqv = nq_all[static_cast<int64_t>(qi) * T * kBM + row];
         bar_wait(tfull(buf), (uc >> 1) & 1);
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        // two-partition exact top-2 (see tid_kernels.cu) over the bit patterns of d >= 0
         int Rm[16];
 #pragma unroll
-        for (int b = 0; b < 16; ++b) Rm[b] = INT_MAX;
-        int T1 = INT_MAX, T2 = INT_MAX;
-#pragma unroll 1
-        for (int c = 0; c < kBN / 32; ++c) {
-          uint32_t v[32];
-          ld32(tq + buf * kBN + c * 32, v);
-          int k[32];
-#pragma unroll
-          for (int i = 0; i < 32; ++i) {
-            const float d = fmaxf(fmaf(-2.0f, __uint_as_float(v[i]), nr_s[c * 32 + i]) + nqv, 0.0f);
-            k[i] = __float_as_int(d);
-          }
-          const int x = min(mn3(mn3(k[0], k[1], k[2]), mn3(k[3], k[4], k[5]), mn3(k[6], k[7], k[8])),
-                            mn3(mn3(k[9], k[10], k[11]), mn3(k[12], k[13], k[14]), k[15]));
-          const int y = min(mn3(mn3(k[16], k[17], k[18]), mn3(k[19], k[20], k[21]), mn3(k[22], k[23], k[24])),
-                            mn3(mn3(k[25], k[26], k[27]), mn3(k[28], k[29], k[30]), k[31]));
-#pragma unroll
-          for (int b = 0; b < 16; ++b) Rm[b] = mn3(Rm[b], k[b], k[b + 16]);
-          const int lo = min(x, y), hi = max(x, y);
-          T2 = mn3(T2, max(T1, lo), hi);
-          T1 = min(T1, lo);
-        }
+        for (int b = 0; b < 16; ++b) Rm[b] = INT_MIN;
+        int T1 = INT_MIN, T2 = INT_MIN;
+        // both 128-column halves in flight at once; the buffer is free as soon as they landed
+        ld16x64x2(tq + buf * kBN, v, w);
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         __syncwarp();
         if (lane == 0) bar_arrive(tempty(buf));
-        int rm[4], cm[4];
-#pragma unroll
-        for (int a = 0; a < 4; ++a) {
-          rm[a] = min(mn3(Rm[4 * a], Rm[4 * a + 1], Rm[4 * a + 2]), Rm[4 * a + 3]);
-          cm[a] = min(mn3(Rm[a], Rm[a + 4], Rm[a + 8]), Rm[a + 12]);
+#ifndef TID_NOSCAN  // timing experiment only
+        scan32(v, Rm, T1, T2);
+        scan32(v + 32, Rm, T1, T2);
+        scan32(w, Rm, T1, T2);
+        scan32(w + 32, Rm, T1, T2);
+#endif
+        int x1, x2;
+        finish(Rm, T1, T2, x1, x2);
+        {  // merge with the partner thread holding the row's other columns
+          const int o1 = __shfl_xor_sync(0xffffffffu, x1, 2), o2 = __shfl_xor_sync(0xffffffffu, x2, 2);
+          x2 = mx3(min(x1, o1), x2, o2);
+          x1 = max(x1, o1);
         }
-        const int sr = mn3(max(min(rm[0], rm[1]), min(rm[2], rm[3])), max(rm[0], rm[1]), max(rm[2], rm[3]));
-        const int sc = mn3(max(min(cm[0], cm[1]), min(cm[2], cm[3])), max(cm[0], cm[1]), max(cm[2], cm[3]));
-        const float d1 = __int_as_float(T1), d2 = __int_as_float(mn3(T2, sr, sc));
-        // ratio test in fp64 on the fp32 distances; padded columns are +inf
-        const bool pass = valid && isfinite(d2) && double(den2) * double(d1) < double(num2) * double(d2);
-        cnt += __popc(__ballot_sync(0xffffffffu, pass));
-        if (t % T == T - 1) {
+        // d = N_Q + 2C - 2X (fp64 from the fp32 values; clamped at 0); padded columns have X < 0
+        const double d1 = fmax(double(nqv) + c2 - 2.0 * double(__int_as_float(x1)), 0.0);
+        const double d2 = fmax(double(nqv) + c2 - 2.0 * double(__int_as_float(x2)), 0.0);
+        // ratio test in fp64
+        const bool pass = valid && x2 >= 0 && double(den2) * d1 < double(num2) * d2;
+        cnt += __popc(__ballot_sync(0xffffffffu, pass) & 0x33333333u);  // one thread per row
+        if (++tt == T) {
           if (lane == 0 && cnt) atomicAdd(counts + static_cast<int64_t>(qi) * R + r, cnt);
           cnt = 0;
+          tt = 0;
+          ++qi;
         }
       }
       __syncwarp();
@@ -256,6 +332,62 @@ __global__ void __launch_bounds__(kThreads, 1)
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem) : "memory");
   }
+}
+
+// Largest squared norm of the launch's references (fp32 bits, non-negative: integer max).
+__global__ void nr_max_kernel(const __half* __restrict__ x, int64_t rows, uint32_t* __restrict__ max_bits) {
+  const int64_t g = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+  float acc = 0.0f;
+  if (g < rows) {
+    const __half2* p = reinterpret_cast<const __half2*>(x + g * kDim);
+#pragma unroll 8
+    for (int i = 0; i < kDim / 2; ++i) {
+      const float2 f = __half22float2(p[i]);
+      acc = fmaf(f.x, f.x, acc);
+      acc = fmaf(f.y, f.y, acc);
+    }
+  }
+  for (int o = 16; o > 0; o >>= 1) acc = fmaxf(acc, __shfl_xor_sync(0xffffffffu, acc, o));
+  if ((threadIdx.x & 31) == 0) atomicMax(max_bits, __float_as_uint(acc));
+}
+
+// Norm-term rows [R][256][16] fp16: (h1, h2, h3, 0 ...) with h1 + h2 + h3 = C - N_R / 2 (three
+// fp16 terms of the fp32 value, 33 significant bits), C = smallest power of two >= max N_R / 2;
+// rows >= m: h1 = -inf.  Also writes C.
+__global__ void xop_kernel(const __half* __restrict__ x, int64_t R, int32_t m, const uint32_t* __restrict__ max_bits,
+                           __half* __restrict__ xop, float* __restrict__ cterm) {
+  const int64_t g = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (g >= R * kBN) return;
+  int e;
+  frexpf(0.5f * __uint_as_float(*max_bits), &e);
+  const float C = ldexpf(1.0f, e);  // > max N_R / 2 (or 1 if all norms are 0)
+  if (g == 0) *cterm = C;
+  const int64_t ref = g / kBN;
+  const int row = static_cast<int>(g % kBN);
+  __half h[kXH];
+#pragma unroll
+  for (int i = 0; i < kXH; ++i) h[i] = __float2half_rn(0.0f);
+  if (row < m) {
+    const __half2* p = reinterpret_cast<const __half2*>(x + (ref * m + row) * kDim);
+    float acc = 0.0f;
+#pragma unroll 8
+    for (int i = 0; i < kDim / 2; ++i) {
+      const float2 f = __half22float2(p[i]);
+      acc = fmaf(f.x, f.x, acc);
+      acc = fmaf(f.y, f.y, acc);
+    }
+    const float val = C - 0.5f * acc;
+    h[0] = __float2half_rn(val);
+    const float r1 = val - __half2float(h[0]);
+    h[1] = __float2half_rn(r1);
+    h[2] = __float2half_rn(r1 - __half2float(h[1]));
+  } else {
+    h[0] = __ushort_as_half(0xFC00u);  // -inf
+  }
+  uint4* dst = reinterpret_cast<uint4*>(xop + g * kXH);
+  const uint4* src = reinterpret_cast<const uint4*>(h);
+  dst[0] = src[0];
+  dst[1] = src[1];
 }
 
 // Squared norms in fp32 of fp16 rows: out[item][row] for rows < valid, `pad` beyond (items of
@@ -317,9 +449,21 @@ cudaError_t launch_f16_norms(const void* x, int64_t items, int32_t rows, int32_t
   return cudaGetLastError();
 }
 
-cudaError_t launch_f16_match(const CUtensorMap& qmap, const CUtensorMap& rmap, const float* nr, const float* nq,
-                             int32_t B, int32_t n, int32_t T, int64_t R, uint32_t num2, uint32_t den2,
-                             uint32_t* counts, int num_sms, cudaStream_t s) {
+cudaError_t launch_f16_xop(const void* r, int64_t R, int32_t m, uint32_t* scratch, void* xop, float* cterm,
+                           cudaStream_t s) {
+  cudaError_t e = cudaMemsetAsync(scratch, 0, 4, s);
+  if (e != cudaSuccess) return e;
+  const int64_t rows = R * m;
+  f16::nr_max_kernel<<<static_cast<unsigned>((rows + 255) / 256), 256, 0, s>>>(static_cast<const __half*>(r), rows,
+                                                                              scratch);
+  f16::xop_kernel<<<static_cast<unsigned>((R * kBN + 255) / 256), 256, 0, s>>>(
+      static_cast<const __half*>(r), R, m, scratch, static_cast<__half*>(xop), cterm);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_f16_match(const CUtensorMap& qmap, const CUtensorMap& rmap, const CUtensorMap& xmap,
+                             const float* cterm, const float* nq, int32_t B, int32_t n, int32_t T, int64_t R,
+                             uint32_t num2, uint32_t den2, uint32_t* counts, int num_sms, cudaStream_t s) {
   cudaError_t e = cudaFuncSetAttribute(f16::match_f16_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(f16::Plan::kAlloc));
   if (e != cudaSuccess) return e;
@@ -328,8 +472,8 @@ cudaError_t launch_f16_match(const CUtensorMap& qmap, const CUtensorMap& rmap, c
   while (R * ((B + qpj - 1) / qpj) < 2LL * num_sms && qpj > 1) qpj = (qpj + 1) / 2;
   const int64_t jobs = R * ((B + qpj - 1) / qpj);
   const int grid = static_cast<int>(jobs < num_sms ? jobs : num_sms);
-  f16::match_f16_kernel<<<grid, f16::kThreads, f16::Plan::kAlloc, s>>>(qmap, rmap, nr, nq, B, n, T, R, qpj, num2,
-                                                                        den2, counts);
+  f16::match_f16_kernel<<<grid, f16::kThreads, f16::Plan::kAlloc, s>>>(qmap, rmap, xmap, cterm, nq, B, n, T, R, qpj,
+                                                                        num2, den2, counts);
   return cudaGetLastError();
 }
 
