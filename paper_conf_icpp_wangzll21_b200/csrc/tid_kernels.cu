@@ -578,7 +578,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     // 64-column buffers (whole warp, one elected lane).  Every warp commits the release of every
     // query tile (waiting for tiles it never used, so the stage phases stay in order).
     const int mw = warp - kFirstMmaWarp;
-    uint32_t qctr = 0, pb = 0, pph = 0;  // next buffer of this group and its phase
+    uint32_t qctr = 0;
     if (kFold) mbar_wait(axfull, 0);  // constant norm-term operand in TMEM
     uint32_t slot_par = 0;  // bit sl = phase parity of reference slot sl
     for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
@@ -607,10 +607,10 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               ready_mask |= 1u << sl;
             }
             const uint64_t bd0 = smem_desc_sw128(sbase + SmemPlan::kR + sl * kRTileBytes);
-#pragma unroll 1
-            for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
-              const uint32_t buf = mw * kNB + pb;
-              PROF_B(); mbar_wait(tempty(buf), pph ^ 1); PROF_E(0);
+#pragma unroll
+            for (int pp = 0; pp < kPiecesPerChunk; ++pp) {  // static buffer / phase (see the epilogue)
+              const uint32_t buf = mw * kNB + (pp & 1);
+              PROF_B(); mbar_wait(tempty(buf), ((pp >> 1) & 1) ^ 1); PROF_E(0);
               tc_fence_after();
               // rows kPiece*pp.. of the chunk: SWIZZLE_128B core groups of 8 rows x 128 B
               const uint64_t bd = bd0 + pp * (kPiece * kDim >> 4);
@@ -623,7 +623,6 @@ __global__ void __launch_bounds__(kNumThreads, 1)
                                   tfull(buf));
               else
                 mma_piece<kIdescI8>(tmem_base + buf * kPiece, ad, bd, tfull(buf));
-              if (++pb == kNB) { pb = 0; pph ^= 1; }
             }
           }
         }
@@ -658,7 +657,6 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     const int row_in_tile = quarter * 32 + lane;
     const int nq_ld = T * kBM;
     const bool ratio32 = p.num2 <= 511u && p.den2 <= 511u;  // den^2 * d fits 32 bits (d <= 8,323,200)
-    uint32_t eb = 0, eph = 0;             // next buffer of this group to consume and its phase
     uint32_t slot_par = 0;                // bit sl = phase parity of reference slot sl
     uint32_t v[64];
 
@@ -694,10 +692,13 @@ __global__ void __launch_bounds__(kNumThreads, 1)
 #pragma unroll
             for (int b = 0; b < 16; ++b) R[b] = INT_MIN;
             int T1 = INT_MIN, T2 = INT_MIN;
-#pragma unroll 1
+            // 4 pieces per chunk through the group's 2 buffers: each buffer is used twice per chunk,
+            // so buffer and phase are compile-time functions of pp (fully unrolled)
+            static_assert(kNB == 2 && kPiecesPerChunk == 4, "static buffer / phase schedule");
+#pragma unroll
             for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
-              const uint32_t buf = g * kNB + eb;
-              PROF_B(); mbar_wait(tfull(buf), eph); PROF_E(0);
+              const uint32_t buf = g * kNB + (pp & 1);
+              PROF_B(); mbar_wait(tfull(buf), (pp >> 1) & 1); PROF_E(0);
               tc_fence_after();
 #ifndef TID_NOLOAD  // timing experiment only: scan stale registers (wrong results)
               tmem_ld64(taddr_q + buf * kPiece, v);
@@ -707,7 +708,6 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               tc_fence_before();  // the piece is in registers: buffer free
               __syncwarp();
               if (lane == 0) mbar_arrive(tempty(buf));
-              if (++eb == kNB) { eb = 0; eph ^= 1; }
               PROF_B();
               if (kpc >= kBN) {  // full chunk (the common case): no masking
 #ifndef TID_NOSCAN
@@ -765,8 +765,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           int T1 = INT_MAX, T2 = INT_MAX;
 #pragma unroll 1
           for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
-            const uint32_t buf = g * kNB + eb;
-            PROF_B(); mbar_wait(tfull(buf), eph); PROF_E(0);
+            const uint32_t buf = g * kNB + (pp & 1);
+            PROF_B(); mbar_wait(tfull(buf), (pp >> 1) & 1); PROF_E(0);
             tc_fence_after();
             // x64 loads; the buffer is released as soon as its last load has landed
 #pragma unroll
@@ -778,7 +778,6 @@ __global__ void __launch_bounds__(kNumThreads, 1)
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(tempty(buf));
-                if (++eb == kNB) { eb = 0; eph ^= 1; }
               }
               PROF_B();
               scan32_regs(v, ck + (pp * kPiece + h * 64) * 4, R, T1, T2);
