@@ -763,7 +763,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
 #pragma unroll
           for (int b = 0; b < 16; ++b) R[b] = INT_MAX;
           int T1 = INT_MAX, T2 = INT_MAX;
-#pragma unroll 1
+#pragma unroll
           for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
             const uint32_t buf = g * kNB + (pp & 1);
             PROF_B(); mbar_wait(tfull(buf), (pp >> 1) & 1); PROF_E(0);
