@@ -38,6 +38,16 @@ constexpr uint32_t kQHalf = kBM * kHalfBytes;       // 16 KiB: 128 query rows x 
 constexpr int kStages = 4;
 constexpr int kXH = 16;                             // fp16 per norm-term row (one K = 16 step, 32 B)
 constexpr uint32_t kXTile = kBN * kXH * 2;          // 8 KiB: 256 reference rows x 16 fp16
+#ifndef TID_F16_N
+#define TID_F16_N 128
+#endif
+// MMA pieces of kFN columns through kFNB = 512 / kFN TMEM buffers: with N = 128 the MMA can run
+// 1.5 units ahead of the epilogue instead of one (the A tile is re-read per piece: more shared-
+// memory operand traffic, which the measurement decides)
+constexpr int kFN = TID_F16_N;
+constexpr int kFPieces = kBN / kFN;                 // pieces per unit
+constexpr int kFNB = 512 / kFN;                     // TMEM buffers
+static_assert(kFNB % kFPieces == 0 && (kFNB / kFPieces) == 2, "two units of pieces in flight");
 
 struct Plan {
   static constexpr uint32_t kR = 0;                            // 2 halves
@@ -47,8 +57,8 @@ struct Plan {
   static constexpr uint32_t kBar = kAx + kBM * kXH * 2;
   static constexpr uint32_t kQFull = kBar, kQEmpty = kBar + 8 * kStages;
   static constexpr uint32_t kRFull = kQEmpty + 8 * kStages, kREmpty = kRFull + 8;
-  static constexpr uint32_t kTFull = kREmpty + 8, kTEmpty = kTFull + 16;
-  static constexpr uint32_t kTmemPtr = kTEmpty + 16;
+  static constexpr uint32_t kTFull = kREmpty + 8, kTEmpty = kTFull + 8 * kFNB;
+  static constexpr uint32_t kTmemPtr = kTEmpty + 8 * kFNB;
   static constexpr uint32_t kAlloc = kTmemPtr + 16 + 1024;
 };
 
@@ -87,7 +97,7 @@ __device__ __forceinline__ uint64_t desc32(uint32_t addr) {
          (uint64_t(1) << 46) | (uint64_t(6) << 61);
 }
 // kind::f16: D = F32 (bits 4-5 = 1), A = B = F16 (0), K-major, N = 256, M = 128.
-constexpr uint32_t kIdesc = (1u << 4) | (uint32_t(kBN >> 3) << 17) | (uint32_t(kBM >> 4) << 24);
+constexpr uint32_t kIdesc = (1u << 4) | (uint32_t(kFN >> 3) << 17) | (uint32_t(kBM >> 4) << 24);
 
 // D = Q . R^T over K = 128 fp16 (per K-half, one SWIZZLE_128B tile, four K = 16 steps of 32 B),
 // then D += ones . (h1, h2, h3) (the norm-term step).
@@ -210,7 +220,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     for (int i = 0; i < kStages; ++i) { bar_init(qfull(i), 1); bar_init(qempty(i), 1); }
     bar_init(rfull, 1);
     bar_init(rempty, 1 + kEpi);
-    for (int i = 0; i < 2; ++i) { bar_init(tfull(i), 1); bar_init(tempty(i), kEpi); }
+    for (int i = 0; i < kFNB; ++i) { bar_init(tfull(i), 1); bar_init(tempty(i), kEpi); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 1) {
@@ -253,16 +263,23 @@ __global__ void __launch_bounds__(kThreads, 1)
       bar_wait(rfull, rc & 1);
       const uint64_t b0 = desc128(sb + Plan::kR), b1 = desc128(sb + Plan::kR + kRHalf);
       for (int t = 0; t < nq * T; ++t, ++qc, ++uc) {
-        const int st = qc % kStages, buf = uc & 1;
+        const int st = qc % kStages;
         bar_wait(qfull(st), (qc / kStages) & 1);
-        bar_wait(tempty(buf), ((uc >> 1) & 1) ^ 1);
-        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         const uint32_t qa = sb + Plan::kQ + st * 2 * kQHalf;
+        // unit uc uses buffers kFPieces * (uc & 1) + h, each once per two units (static phases)
+#pragma unroll
+        for (int h = 0; h < kFPieces; ++h) {
+          const int buf = kFPieces * (uc & 1) + h;
+          bar_wait(tempty(buf), ((uc >> 1) & 1) ^ 1);
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 #ifdef TID_NOMMA  // timing experiment only
-        commit(tfull(buf));
+          commit(tfull(buf));
 #else
-        mma_unit(tmem + buf * kBN, desc128(qa), desc128(qa + kQHalf), b0, b1, ax, bx, tfull(buf));
+          // reference rows kFN * h.. : SWIZZLE_128B 8-row groups of 1 KiB / SWIZZLE_32B groups of 256 B
+          mma_unit(tmem + buf * kFN, desc128(qa), desc128(qa + kQHalf), b0 + h * (kFN * 128 >> 4),
+                   b1 + h * (kFN * 128 >> 4), ax, bx + h * (kFN * 32 >> 4), tfull(buf));
 #endif
+        }
         commit(qempty(st));
       }
       commit(rempty);
@@ -274,7 +291,10 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int row_in_tile = quarter * 32 + 16 * half + (lane >> 2) + 8 * (lane & 1);
     const double c2 = 2.0 * static_cast<double>(*cterm);
     uint32_t rc = 0, uc = 0;
-    uint32_t v[64], w[64];
+    uint32_t v[64];
+#if TID_F16_N == 256
+    uint32_t w[64];
+#endif
     for (int64_t j = blockIdx.x; j < n_jobs; j += gridDim.x, ++rc) {
       const int64_t r = j / qchunks;
       const int q0 = static_cast<int>(j % qchunks) * q_per_job, nq = min(q_per_job, B - q0);
@@ -282,15 +302,17 @@ __global__ void __launch_bounds__(kThreads, 1)
       uint32_t cnt = 0;
       int qi = q0, tt = 0;  // query and tile of unit t (no divisions per unit)
       for (int t = 0; t < nq * T; ++t, ++uc) {
-        const int buf = uc & 1, row = tt * kBM + row_in_tile;
+        const int row = tt * kBM + row_in_tile;
         const bool valid = row < n;
         const float nqv = nq_all[static_cast<int64_t>(qi) * T * kBM + row];
-        bar_wait(tfull(buf), (uc >> 1) & 1);
-        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         int Rm[16];
 #pragma unroll
         for (int b = 0; b < 16; ++b) Rm[b] = INT_MIN;
         int T1 = INT_MIN, T2 = INT_MIN;
+#if TID_F16_N == 256
+        const int buf = uc & 1;
+        bar_wait(tfull(buf), (uc >> 1) & 1);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         // both 128-column halves in flight at once; the buffer is free as soon as they landed
         ld16x64x2(tq + buf * kBN, v, w);
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
@@ -301,6 +323,22 @@ __global__ void __launch_bounds__(kThreads, 1)
         scan32(v + 32, Rm, T1, T2);
         scan32(w, Rm, T1, T2);
         scan32(w + 32, Rm, T1, T2);
+#endif
+#else
+#pragma unroll
+        for (int h = 0; h < kFPieces; ++h) {  // one x64 load (128 columns) per piece
+          const int buf = kFPieces * (uc & 1) + h;
+          bar_wait(tfull(buf), (uc >> 1) & 1);
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          ld16x64(tq + buf * kFN, v);
+          asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+          __syncwarp();
+          if (lane == 0) bar_arrive(tempty(buf));
+#ifndef TID_NOSCAN  // timing experiment only
+          scan32(v, Rm, T1, T2);
+          scan32(v + 32, Rm, T1, T2);
+#endif
+        }
 #endif
         int x1, x2;
         finish(Rm, T1, T2, x1, x2);
