@@ -24,4 +24,11 @@ with tid.Index(ref_kp=256) as idx:
     vc, nn = idx.verify(Q, R)
 ec, _ = oracle.verify(Q, R)
 assert np.array_equal(vc.astype(np.int64), ec)
+# f1 float path (kind::f16, folded norms): u8 x 2^-7 is exact, so counts equal the integer oracle
+Rr, _ = tidgen.refs(5, 5, 200)
+Qf, _ = tidgen.queries(5, 2, 300, R_total=5, m=200, n_planted=60)
+with tid.Index(query_kp_max=1024) as idx:
+    q16, r16 = idx.f16_prepare(Qf, False, 2.0 ** -7), idx.f16_prepare(Rr, False, 2.0 ** -7)
+    fc = idx.f16_search_counts(q16, r16)
+assert np.array_equal(fc.astype(np.int64), oracle.search_counts(Qf, Rr))
 print("sanitize run ok")
