@@ -1,0 +1,89 @@
+"""GPU parity at BASELINE.json's full sizes, in the launch configuration bench.py times.
+
+C4 (bench default: 256 queries x 1000 keypoints vs a 125,000-reference x 256-keypoint shard)
+and C3 (64 x 100,000) are too large for the oracle in full, so they are checked
+  * on sampled outputs the oracle computes one by one: the count of every (query, reference)
+    pair in a seeded random sample, plus every planted target, exactly;
+  * by properties that hold at any size: every planted target ranks first; the top-k returned by
+    tid_search equals the (count desc, id asc) ranking of the full GPU count matrix re-sorted
+    on the host; counts never exceed n.
+C2 (4,096 verification pairs, n = m = 1000) is small enough for the oracle in full: bit-exact
+counts and (d1, i1, d2, i2) for all 4.1 M query rows.
+Inputs come from tidgen with bench.py's seed; expected values only from oracle/.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import tidgen
+
+pytestmark = pytest.mark.gpu
+
+SEED = 2021  # bench.py
+
+
+@pytest.fixture(scope="module")
+def tid():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    from paper_conf_icpp_wangzll21_b200 import build
+    build.build()
+    import paper_conf_icpp_wangzll21_b200 as t
+    return t
+
+
+def _sampled_search_check(tid, B, n, R, m, k, n_sample_q, n_sample_r):
+    import torch
+    refs, _ = tidgen.refs(0, R, m, seed=SEED)
+    qs, targets = tidgen.queries(0, B, n, R_total=R, m=m, seed=SEED)
+    dq = torch.from_numpy(qs).cuda()
+    with tid.Index(ref_kp=m, query_kp_max=1024, ratio=(4, 5)) as idx:
+        idx.add_references(refs)
+        counts = idx.search_counts(dq)  # [B][R] u32 on the device
+        ids, cnt = idx.search(dq, k)
+        torch.cuda.synchronize()
+        counts = counts.cpu().numpy().astype(np.int64) if hasattr(counts, "cpu") else counts.astype(np.int64)
+        ids = ids.cpu().numpy() if hasattr(ids, "cpu") else ids
+        cnt = cnt.cpu().numpy() if hasattr(cnt, "cpu") else cnt
+    assert counts.shape == (B, R)
+    assert counts.max() <= n
+    # planted targets rank first for every query
+    np.testing.assert_array_equal(ids[:, 0], targets)
+    # top-k == host ranking of the full GPU count matrix (count desc, id asc)
+    e_ids, e_cnt = oracle.topk(counts, k)
+    np.testing.assert_array_equal(ids, e_ids)
+    np.testing.assert_array_equal(cnt, e_cnt)
+    # sampled pairs, exact vs the oracle computed one by one
+    rng = np.random.default_rng(SEED + B)
+    qsel = np.sort(rng.choice(B, size=n_sample_q, replace=False))
+    for q in qsel:
+        rsel = np.unique(np.concatenate([rng.choice(R, size=n_sample_r, replace=False), [targets[q]], ids[q]]))
+        want = oracle.search_counts(qs[q:q + 1], refs[rsel])[0]
+        np.testing.assert_array_equal(counts[q, rsel], want, err_msg=f"query {q}")
+
+
+def test_c4_fullsize_sampled(tid):
+    """C4 per-GPU shard (bench.py's workload): 256 queries x 125,000 references."""
+    _sampled_search_check(tid, B=256, n=1000, R=125_000, m=256, k=5, n_sample_q=16, n_sample_r=120)
+
+
+def test_c3_fullsize_sampled(tid):
+    """C3: 64 queries x 100,000 references."""
+    _sampled_search_check(tid, B=64, n=1000, R=100_000, m=256, k=5, n_sample_q=8, n_sample_r=120)
+
+
+def test_c2_full_verify_bitexact(tid):
+    """C2: 4,096 pairs (half planted-positive), n = m = 1000: every count and every (d1, i1, d2, i2)."""
+    P, n, m = 4096, 1000, 1000
+    Q, R, pos = tidgen.pairs(P, n, m, seed=SEED)
+    with tid.Index(ref_kp=256, query_kp_max=n) as idx:
+        vc, nn = idx.verify(Q, R)
+    ec, enn = oracle.verify(Q, R)
+    np.testing.assert_array_equal(vc.astype(np.int64), ec)
+    o = enn.copy()
+    big = np.iinfo(np.int64).max
+    o[..., 0][o[..., 0] == big] = -1
+    o[..., 2][o[..., 2] == big] = -1
+    np.testing.assert_array_equal(nn.astype(np.int64), o.astype(np.int64))
+    assert vc[pos].mean() > 100 and vc[~pos].mean() < 5
