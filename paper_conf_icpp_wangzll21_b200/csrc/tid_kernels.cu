@@ -449,13 +449,14 @@ __device__ __forceinline__ void exact_row_global(const MatchParams& p, int qi, i
 }
 
 // ------------------------------------------------------------------ fused match kernel
-// One persistent CTA per SM.  A job = (up to 4 references resident in SMEM) x (range of query
-// tiles streamed through a 4-stage ring).  Unit u = (query tile t, reference s), s fastest,
-// belongs to epilogue group u % 4 (with 4 resident references: group g <-> reference g, so its
-// counts accumulate in a register over the query's tiles).  Each 256-column reference chunk of
-// a unit is computed as 4 MMA pieces of 64 columns; group g owns TMEM buffers 2g, 2g+1 and its
-// own MMA warp, so the MMA of the next piece overlaps the scan of the current one, and the 4
-// groups (4 epilogue warps per SMSP) hide each other's TMEM-load and barrier latency.
+// One persistent CTA per SM.  A job = (up to kNG = 3 references resident in SMEM, fewer chunks'
+// worth for m > 256) x (range of query tiles streamed through a kQStages ring; search: copied
+// once per tile into TMEM).  Unit u = (query tile t, reference s), s fastest, belongs to epilogue
+// group u % kNG (group g <-> reference g, so its counts accumulate in a register over the query's
+// tiles).  Each 256-column reference chunk of a unit is 4 MMA pieces of 64 columns through the
+// group's 2 TMEM buffers (buffer pp & 1, phase pp >> 1: compile-time, fully unrolled); group g has
+// its own MMA warp, so the MMA of the next piece overlaps the scan of the current one, and the 3
+// groups (3 epilogue warps per SMSP) hide each other's TMEM-load and barrier latency.
 // kFold: the search path (folded norms, no column keys in the scan, counts only);
 // otherwise the verify path (packed column keys, exact (d1, i1, d2, i2)).
 template <bool kFold>
@@ -573,8 +574,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     }
   } else if (warp < kFirstEpiWarp) {
     // ===================== MMA issuers: warp mw serves epilogue group mw =====================
-    // Issuing tcgen05.mma costs the issuing SMSP throughput, so the 4 issuers sit on 4 SMSPs.
-    // Warp mw issues the pieces of the units u with u % 4 == mw, in order, into its group's two
+    // Issuing tcgen05.mma costs the issuing SMSP throughput, so the kNG issuers sit on SMSPs 1-3.
+    // Warp mw issues the pieces of the units u with u % kNG == mw, in order, into its group's two
     // 64-column buffers (whole warp, one elected lane).  Every warp commits the release of every
     // query tile (waiting for tiles it never used, so the stage phases stay in order).
     const int mw = warp - kFirstMmaWarp;
