@@ -343,3 +343,32 @@ def test_delete_update_save_load(tid, tmp_path):
     np.testing.assert_array_equal(c2, counts)
     np.testing.assert_array_equal(i2, ids)
     np.testing.assert_array_equal(n2, cnt)
+
+
+# ------------------------------------------------------------------------------ ABI error behaviour
+def test_abi_errors_and_empty_queries(tid):
+    """include/tid.h conventions on a GPU: invalid arguments return TID_EINVAL (raised as TidError
+    with the status) and leave the index usable; an empty query (n_q = 0) matches nothing."""
+    R, m, n = 10, 256, 300
+    refs, _ = tidgen.refs(0, R, m)
+    qs, _ = tidgen.queries(0, 3, n, R_total=R, m=m, n_planted=50)
+    with pytest.raises(tid.TidError) as e:
+        tid.Index(ref_kp=1)  # ref_kp < 2
+    assert e.value.status == tid.TID_EINVAL
+    with tid.Index(ref_kp=m, query_kp_max=512) as idx:
+        idx.add_references(refs)
+        with pytest.raises(tid.TidError) as e:
+            idx.search(qs, R + 1)  # k > number of references
+        assert e.value.status == tid.TID_EINVAL
+        big, _ = tidgen.queries(0, 1, 600, R_total=R, m=m)
+        with pytest.raises(tid.TidError) as e:
+            idx.search(big, 3)  # n > query_kp_max
+        assert e.value.status == tid.TID_EINVAL
+        n_q = np.array([0, n, 7], np.int32)  # still usable after the errors
+        counts = idx.search_counts(qs, n_q=n_q)
+        ids, cnt = idx.search(qs, 3, n_q=n_q)
+    e_ids, e_cnt, e_counts = oracle.search(qs, refs, 3, n_q=n_q)
+    np.testing.assert_array_equal(counts.astype(np.int64), e_counts)
+    np.testing.assert_array_equal(ids, e_ids)
+    np.testing.assert_array_equal(cnt, e_cnt)
+    assert (counts[0] == 0).all()
