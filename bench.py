@@ -112,6 +112,29 @@ def peaks():
                 "source": "fallback (B200_PROFILING.md)"}
 
 
+def pipes_from_profile(traffic):
+    """Tensor / ALU pipe utilisation of the match kernel from the committed ncu summary that the
+    traffic figure comes from (profiles/; one `ncu --set full` launch at this config), or None."""
+    if not traffic or "source" not in traffic:
+        return None
+    path = os.path.join(ROOT, traffic["source"].split()[0])
+    want = {"sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active": "tensor_active",
+            "sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active": "alu_active",
+            "smsp__issue_active.avg.pct_of_peak_sustained_active": "issue_active"}
+    out = {}
+    try:
+        for line in open(path):
+            parts = line.split()
+            if len(parts) >= 2 and parts[0] in want:
+                out[want[parts[0]]] = float(parts[1]) / 100.0
+    except (OSError, ValueError):
+        return None
+    if not out:
+        return None
+    out["source"] = traffic["source"].split()[0]
+    return out
+
+
 # ----------------------------------------------------------------------------- oracle arm
 def time_oracle(qs, refs, seconds: float):
     """Time the CPU oracle (as it stands, OpenMP over all host cores) on a bounded sample:
@@ -318,7 +341,8 @@ def main():
             "algorithmic_ops": "2*n*m*128 per (query, reference) pair; the kernel also runs a 5th (norm-term) "
                                "K-step, +25% tensor work not counted here",
             "binding_note": "the fused epilogue (TMEM loads + two-partition top-2 on the ALU pipe) limits the kernel "
-                            "below the tensor peak; see DESIGN.md section 7"}
+                            "below the tensor peak; see DESIGN.md section 7",
+            "pipes_ncu": pipes_from_profile(traffic)}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
