@@ -963,17 +963,22 @@ tid_status tid_search(tid_index* idx, const uint8_t* queries, const int32_t* n_q
   segs = std::min<int64_t>(segs, 1024);
   TRY(idx->ws_cand.ensure(static_cast<size_t>(B) * segs * k * 8, "top-k candidates"));
   TRY(sync_dead(idx, s));
-  launch_topk(counts, B, R, R, idx->cfg.id_base, k, static_cast<int32_t>(segs),
-              idx->any_dead ? idx->dead_dev.as<uint8_t>() : nullptr, idx->ws_cand.as<uint64_t>(), s);
-  count_kernel(idx);
   TRY(idx->ws_ids.ensure(static_cast<size_t>(B) * k * 8, "ids"));
   TRY(idx->ws_cnts.ensure(static_cast<size_t>(B) * k * 4, "counts"));
   const bool dev_ids = is_device_ptr(ref_ids_out), dev_cnt = is_device_ptr(match_counts_out);
   int64_t* ids = dev_ids ? ref_ids_out : idx->ws_ids.as<int64_t>();
   int32_t* cnts = dev_cnt ? match_counts_out : idx->ws_cnts.as<int32_t>();
+  // one segment on one GPU: the top-k kernel writes the final ranking (no merge launch)
+  const bool direct = idx->comm == nullptr && segs == 1;
+  launch_topk(counts, B, R, R, idx->cfg.id_base, k, static_cast<int32_t>(segs),
+              idx->any_dead ? idx->dead_dev.as<uint8_t>() : nullptr, idx->ws_cand.as<uint64_t>(), s,
+              direct ? ids : nullptr, direct ? cnts : nullptr);
+  count_kernel(idx);
   if (idx->comm == nullptr) {
-    launch_merge(idx->ws_cand.as<uint64_t>(), static_cast<int32_t>(segs), B, k, segs * k, k, nullptr, ids, cnts, s);
-    count_kernel(idx);
+    if (!direct) {
+      launch_merge(idx->ws_cand.as<uint64_t>(), static_cast<int32_t>(segs), B, k, segs * k, k, nullptr, ids, cnts, s);
+      count_kernel(idx);
+    }
   } else {
     // a9: local top-k -> NCCL all-gather over NVLink -> identical merge on every rank
     const int G = idx->cfg.world_size;

@@ -1024,9 +1024,11 @@ __device__ void block_select(const uint64_t* lists, int k, uint64_t* out, uint64
   }
 }
 
-// grid (B, segs), 256 threads, dyn smem = 256*k*8 + 33*8.
+// grid (B, segs), 256 threads, dyn smem = 256*k*8 + 33*8.  With one segment and ids_out set, the
+// block's winners are the final ranking: written as (ids, counts) directly (no merge launch).
 __global__ void topk_kernel(const uint32_t* __restrict__ counts, int64_t R, int64_t ldc, int64_t id_base, int32_t k,
-                            const uint8_t* __restrict__ dead, uint64_t* __restrict__ cand_out) {
+                            const uint8_t* __restrict__ dead, uint64_t* __restrict__ cand_out,
+                            int64_t* __restrict__ ids_out, int32_t* __restrict__ counts_out) {
   extern __shared__ uint64_t tk_smem[];
   uint64_t* lists = tk_smem;
   uint64_t* red = tk_smem + blockDim.x * k;
@@ -1048,19 +1050,28 @@ __global__ void topk_kernel(const uint32_t* __restrict__ counts, int64_t R, int6
     }
   }
   __syncthreads();
-  block_select(lists, k, cand_out + (static_cast<int64_t>(b) * segs + seg) * k, red);
+  uint64_t* out = cand_out + (static_cast<int64_t>(b) * segs + seg) * k;
+  block_select(lists, k, out, red);
+  if (ids_out) {  // segs == 1: final (count desc, id asc) ranking
+    __syncthreads();
+    for (int i = threadIdx.x; i < k; i += blockDim.x) {
+      const uint64_t key = out[i];
+      ids_out[static_cast<int64_t>(b) * k + i] = key ? static_cast<int64_t>(kIdMask - (key & kIdMask)) : -1;
+      counts_out[static_cast<int64_t>(b) * k + i] = static_cast<int32_t>(key >> 40);
+    }
+  }
 }
 
 void launch_topk(const uint32_t* counts, int64_t B, int64_t R, int64_t ldc, int64_t id_base, int32_t k, int32_t segs,
-                 const uint8_t* dead, uint64_t* cand_out, cudaStream_t s) {
+                 const uint8_t* dead, uint64_t* cand_out, cudaStream_t s, int64_t* ids_out, int32_t* counts_out) {
   const size_t smem = (256 * static_cast<size_t>(k) + 33) * 8;
   static size_t attr = 0;
   if (smem > 48 * 1024 && smem > attr) {
     cudaFuncSetAttribute(topk_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
     attr = smem;
   }
-  topk_kernel<<<dim3(static_cast<unsigned>(B), static_cast<unsigned>(segs)), 256, smem, s>>>(counts, R, ldc, id_base,
-                                                                                              k, dead, cand_out);
+  topk_kernel<<<dim3(static_cast<unsigned>(B), static_cast<unsigned>(segs)), 256, smem, s>>>(
+      counts, R, ldc, id_base, k, dead, cand_out, segs == 1 ? ids_out : nullptr, segs == 1 ? counts_out : nullptr);
 }
 
 // ------------------------------------------------------------------ a6/a9: merge ranked lists

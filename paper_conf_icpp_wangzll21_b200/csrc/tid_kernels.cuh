@@ -107,8 +107,10 @@ void launch_query_prep(const uint8_t* q, int64_t B, int32_t n, int32_t tiles_per
                        uint8_t* qs, cudaStream_t s);
 cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap,
                          const CUtensorMap* xmap, int grid, cudaStream_t s);
+// ids_out / counts_out (optional): with segs == 1 the final ranking is written directly
 void launch_topk(const uint32_t* counts, int64_t B, int64_t R, int64_t ldc, int64_t id_base, int32_t k,
-                 int32_t segs, const uint8_t* dead, uint64_t* cand_out, cudaStream_t s);
+                 int32_t segs, const uint8_t* dead, uint64_t* cand_out, cudaStream_t s, int64_t* ids_out = nullptr,
+                 int32_t* counts_out = nullptr);
 void launch_merge(const uint64_t* cand, int32_t L, int64_t B, int32_t k, int64_t list_stride_b,
                   int64_t list_stride_l, uint64_t* keys_out, int64_t* ids_out, int32_t* counts_out,
                   cudaStream_t s);
