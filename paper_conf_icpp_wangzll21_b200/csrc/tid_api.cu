@@ -136,9 +136,47 @@ PFN_encodeTiled_t encode_fn() {
   return fn;
 }
 
+// Encoded maps depend only on (address, geometry), so repeated searches reuse them: a small
+// per-thread cache (encoding costs host microseconds, which bound small-search latency).
+struct MapKey {
+  int kind;
+  const void* base;
+  int64_t count, rows;
+  int box;
+  bool operator==(const MapKey& o) const {
+    return kind == o.kind && base == o.base && count == o.count && rows == o.rows && box == o.box;
+  }
+};
+bool map_cache_get(const MapKey& k, CUtensorMap* map);
+void map_cache_put(const MapKey& k, const CUtensorMap& map);
+struct MapCache {
+  static constexpr int kN = 16;
+  MapKey key[kN];
+  CUtensorMap map[kN];
+  int used = 0, next = 0;
+};
+thread_local MapCache g_maps;
+bool map_cache_get(const MapKey& k, CUtensorMap* map) {
+  for (int i = 0; i < g_maps.used; ++i)
+    if (g_maps.key[i] == k) {
+      *map = g_maps.map[i];
+      return true;
+    }
+  return false;
+}
+void map_cache_put(const MapKey& k, const CUtensorMap& map) {
+  const int i = g_maps.next;
+  g_maps.key[i] = k;
+  g_maps.map[i] = map;
+  g_maps.next = (i + 1) % MapCache::kN;
+  g_maps.used = std::min(g_maps.used + 1, MapCache::kN);
+}
+
 // u8 tensor [count][rows][128] -> 3-D map with box {128 B, box_rows, 1}, SWIZZLE_128B,
 // out-of-bounds rows zero-filled (this is how ragged n / m are padded to the tile).
 tid_status make_map(CUtensorMap* map, const void* base, int64_t count, int64_t rows, int box_rows) {
+  const MapKey key{0, base, count, rows, box_rows};
+  if (map_cache_get(key, map)) return TID_OK;
   PFN_encodeTiled_t fn = encode_fn();
   if (!fn) return fail(TID_ECUDA, "cuTensorMapEncodeTiled entry point unavailable");
   if (reinterpret_cast<uintptr_t>(base) % 16) return fail(TID_EINVAL, "descriptor buffer must be 16-byte aligned");
@@ -151,11 +189,14 @@ tid_status make_map(CUtensorMap* map, const void* base, int64_t count, int64_t r
                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return fail(TID_ECUDA, "cuTensorMapEncodeTiled failed (%d)", static_cast<int>(r));
+  map_cache_put(key, *map);
   return TID_OK;
 }
 
 // u8 norm-term digits [count][rows][32] -> 3-D map with box {32 B, 256, 1}, SWIZZLE_32B.
 tid_status make_xmap(CUtensorMap* map, const void* base, int64_t count, int64_t rows) {
+  const MapKey key{1, base, count, rows, kBN};
+  if (map_cache_get(key, map)) return TID_OK;
   PFN_encodeTiled_t fn = encode_fn();
   if (!fn) return fail(TID_ECUDA, "cuTensorMapEncodeTiled entry point unavailable");
   cuuint64_t dims[3] = {static_cast<cuuint64_t>(kXDim), static_cast<cuuint64_t>(rows),
@@ -167,6 +208,7 @@ tid_status make_xmap(CUtensorMap* map, const void* base, int64_t count, int64_t 
                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return fail(TID_ECUDA, "cuTensorMapEncodeTiled (norm digits) failed (%d)", static_cast<int>(r));
+  map_cache_put(key, *map);
   return TID_OK;
 }
 

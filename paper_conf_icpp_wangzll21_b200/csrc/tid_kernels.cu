@@ -866,12 +866,19 @@ extern "C" int tid_debug_read_prof(void* host, size_t bytes) {
 
 cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap,
                          const CUtensorMap* xmap, int grid, cudaStream_t s) {
-  cudaError_t e = cudaFuncSetAttribute(match_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       static_cast<int>(SmemPlan::kAlloc));
-  if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(match_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           static_cast<int>(SmemPlan::kAlloc));
-  if (e != cudaSuccess) return e;
+  // the shared-memory opt-in is per device: set once per device (host overhead matters for C1)
+  static thread_local uint64_t attr_set = 0;  // bit d = device d configured
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev >= 64 || !(attr_set >> dev & 1)) {
+    cudaError_t e = cudaFuncSetAttribute(match_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         static_cast<int>(SmemPlan::kAlloc));
+    if (e != cudaSuccess) return e;
+    e = cudaFuncSetAttribute(match_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             static_cast<int>(SmemPlan::kAlloc));
+    if (e != cudaSuccess) return e;
+    if (dev < 64) attr_set |= uint64_t(1) << dev;
+  }
   if (xmap)
     match_kernel<true><<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, *xmap, p);
   else
