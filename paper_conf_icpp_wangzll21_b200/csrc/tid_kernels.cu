@@ -746,6 +746,12 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             undecided = !pass_sure && !fail_sure;
           }
           uint32_t und = __ballot_sync(0xffffffffu, undecided);
+#ifdef TID_PROF
+          if (lane == 0) {  // g_prof[148 * 32 * 8 - 2 / -1]: undecided rows / warp-units with any
+            atomicAdd(&g_prof[148 * 32 * 8 - 2], static_cast<unsigned long long>(__popc(und)));
+            if (und) atomicAdd(&g_prof[148 * 32 * 8 - 1], 1ull);
+          }
+#endif
           while (und) {  // rare: recompute the row exactly
             const int l = __ffs(und) - 1;
             und &= und - 1;
