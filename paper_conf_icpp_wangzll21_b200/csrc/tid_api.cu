@@ -1242,12 +1242,13 @@ tid_status tid_f16_search_counts(tid_index* idx, const uint16_t* q, int32_t n, i
   TRY(idx->ws_f16nq.ensure(static_cast<size_t>(B) * T * kBM * 4, "f16 query norms"));
   // norm-term operand (R x 256 rows x 32 B) + the scalars max N_R (bits) and C
   const size_t xb = static_cast<size_t>(R) * kBN * 32;
-  TRY(idx->ws_f16nr.ensure(xb + 256, "f16 reference norm terms"));
+  TRY(idx->ws_f16nr.ensure(xb + 256 + static_cast<size_t>(R) * m * 4, "f16 reference norm terms"));
   uint8_t* xop = idx->ws_f16nr.as<uint8_t>();
   uint32_t* nrmax = reinterpret_cast<uint32_t*>(xop + xb);
   float* cterm = reinterpret_cast<float*>(xop + xb + 128);
+  float* nr_rows = reinterpret_cast<float*>(xop + xb + 256);
   CU(launch_f16_norms(dq, B, n, T * kBM, 0.0f, idx->ws_f16nq.as<float>(), s));
-  CU(launch_f16_xop(dr, R, m, nrmax, xop, cterm, s));
+  CU(launch_f16_xop(dr, R, m, nrmax, nr_rows, xop, cterm, s));
   count_kernel(idx, 2);
   const bool dev_counts = is_device_ptr(counts_out);
   TRY(idx->ws_counts.ensure(static_cast<size_t>(B) * R * 4, "count matrix"));

@@ -372,27 +372,42 @@ __global__ void __launch_bounds__(kThreads, 1)
   }
 }
 
-// Largest squared norm of the launch's references (fp32 bits, non-negative: integer max).
-__global__ void nr_max_kernel(const __half* __restrict__ x, int64_t rows, uint32_t* __restrict__ max_bits) {
+// Squared norm N_R (fp32) of every reference row, 8 lanes per row (each 32 contiguous bytes: the
+// row's 256 bytes are read by one coalesced 8-lane group), plus the launch's largest N_R (fp32
+// bits, non-negative: integer max).
+__global__ void nr_rows_kernel(const __half* __restrict__ x, int64_t rows, float* __restrict__ nr,
+                               uint32_t* __restrict__ max_bits) {
   const int64_t g = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+  const int64_t row = g >> 3;
+  const int l8 = static_cast<int>(g & 7);
   float acc = 0.0f;
-  if (g < rows) {
-    const __half2* p = reinterpret_cast<const __half2*>(x + g * kDim);
-#pragma unroll 8
-    for (int i = 0; i < kDim / 2; ++i) {
-      const float2 f = __half22float2(p[i]);
-      acc = fmaf(f.x, f.x, acc);
-      acc = fmaf(f.y, f.y, acc);
+  if (row < rows) {
+    const uint4* p = reinterpret_cast<const uint4*>(x + row * kDim) + 2 * l8;
+#pragma unroll
+    for (int w = 0; w < 2; ++w) {
+      const uint4 u = p[w];
+      const uint32_t words[4] = {u.x, u.y, u.z, u.w};
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const float2 f = __half22float2(*reinterpret_cast<const __half2*>(&words[i]));
+        acc = fmaf(f.x, f.x, acc);
+        acc = fmaf(f.y, f.y, acc);
+      }
     }
   }
-  for (int o = 16; o > 0; o >>= 1) acc = fmaxf(acc, __shfl_xor_sync(0xffffffffu, acc, o));
-  if ((threadIdx.x & 31) == 0) atomicMax(max_bits, __float_as_uint(acc));
+#pragma unroll
+  for (int o = 1; o < 8; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  if (row < rows && l8 == 0) nr[row] = acc;
+  float mx = row < rows ? acc : 0.0f;
+#pragma unroll
+  for (int o = 8; o < 32; o <<= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  if ((threadIdx.x & 31) == 0) atomicMax(max_bits, __float_as_uint(mx));
 }
 
 // Norm-term rows [R][256][16] fp16: (h1, h2, h3, 0 ...) with h1 + h2 + h3 = C - N_R / 2 (three
 // fp16 terms of the fp32 value, 33 significant bits), C = smallest power of two >= max N_R / 2;
-// rows >= m: h1 = -inf.  Also writes C.
-__global__ void xop_kernel(const __half* __restrict__ x, int64_t R, int32_t m, const uint32_t* __restrict__ max_bits,
+// rows >= m: h1 = -inf.  Also writes C.  One thread per row (32 contiguous bytes out).
+__global__ void xop_kernel(const float* __restrict__ nr, int64_t R, int32_t m, const uint32_t* __restrict__ max_bits,
                            __half* __restrict__ xop, float* __restrict__ cterm) {
   const int64_t g = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
   if (g >= R * kBN) return;
@@ -406,15 +421,7 @@ __global__ void xop_kernel(const __half* __restrict__ x, int64_t R, int32_t m, c
 #pragma unroll
   for (int i = 0; i < kXH; ++i) h[i] = __float2half_rn(0.0f);
   if (row < m) {
-    const __half2* p = reinterpret_cast<const __half2*>(x + (ref * m + row) * kDim);
-    float acc = 0.0f;
-#pragma unroll 8
-    for (int i = 0; i < kDim / 2; ++i) {
-      const float2 f = __half22float2(p[i]);
-      acc = fmaf(f.x, f.x, acc);
-      acc = fmaf(f.y, f.y, acc);
-    }
-    const float val = C - 0.5f * acc;
+    const float val = C - 0.5f * nr[ref * m + row];
     h[0] = __float2half_rn(val);
     const float r1 = val - __half2float(h[0]);
     h[1] = __float2half_rn(r1);
@@ -487,15 +494,15 @@ cudaError_t launch_f16_norms(const void* x, int64_t items, int32_t rows, int32_t
   return cudaGetLastError();
 }
 
-cudaError_t launch_f16_xop(const void* r, int64_t R, int32_t m, uint32_t* scratch, void* xop, float* cterm,
-                           cudaStream_t s) {
+cudaError_t launch_f16_xop(const void* r, int64_t R, int32_t m, uint32_t* scratch, float* nr, void* xop,
+                           float* cterm, cudaStream_t s) {
   cudaError_t e = cudaMemsetAsync(scratch, 0, 4, s);
   if (e != cudaSuccess) return e;
   const int64_t rows = R * m;
-  f16::nr_max_kernel<<<static_cast<unsigned>((rows + 255) / 256), 256, 0, s>>>(static_cast<const __half*>(r), rows,
-                                                                              scratch);
-  f16::xop_kernel<<<static_cast<unsigned>((R * kBN + 255) / 256), 256, 0, s>>>(
-      static_cast<const __half*>(r), R, m, scratch, static_cast<__half*>(xop), cterm);
+  f16::nr_rows_kernel<<<static_cast<unsigned>((rows * 8 + 255) / 256), 256, 0, s>>>(static_cast<const __half*>(r),
+                                                                                   rows, nr, scratch);
+  f16::xop_kernel<<<static_cast<unsigned>((R * kBN + 255) / 256), 256, 0, s>>>(nr, R, m, scratch,
+                                                                               static_cast<__half*>(xop), cterm);
   return cudaGetLastError();
 }
 

@@ -124,8 +124,8 @@ cudaError_t launch_f16_prepare(const uint8_t* sift, int64_t rows, int32_t rootsi
 cudaError_t launch_f16_norms(const void* x, int64_t items, int32_t rows, int32_t rows_pad, float pad, float* out,
                              cudaStream_t s);
 // norm-term operand [R][256][16] fp16 of fp16 references [R][m][128] and its constant C (device scalar)
-cudaError_t launch_f16_xop(const void* r, int64_t R, int32_t m, uint32_t* scratch, void* xop, float* cterm,
-                           cudaStream_t s);
+cudaError_t launch_f16_xop(const void* r, int64_t R, int32_t m, uint32_t* scratch, float* nr, void* xop,
+                           float* cterm, cudaStream_t s);
 cudaError_t launch_f16_match(const CUtensorMap& qmap, const CUtensorMap& rmap, const CUtensorMap& xmap,
                              const float* cterm, const float* nq, int32_t B, int32_t n, int32_t T, int64_t R,
                              uint32_t num2, uint32_t den2, uint32_t* counts, int num_sms, cudaStream_t s);
