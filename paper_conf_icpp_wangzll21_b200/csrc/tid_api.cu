@@ -1195,12 +1195,14 @@ tid_status tid_f16_prepare(tid_index* idx, const uint8_t* sift, int64_t rows, in
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   const size_t in_b = static_cast<size_t>(rows) * kDim, out_b = in_b * 2;
   const uint8_t* din = sift;
-  if (!is_device_ptr(sift)) {
+  // the kernel moves 16-byte words: unaligned device buffers are staged through the workspace too
+  const bool aligned = reinterpret_cast<uintptr_t>(sift) % 16 == 0 && reinterpret_cast<uintptr_t>(out) % 16 == 0;
+  if (!is_device_ptr(sift) || !aligned) {
     TRY(idx->ws_f16in.ensure(in_b, "f16 prepare input"));
     TRY(copy_in(idx, idx->ws_f16in.p, sift, in_b, s));
     din = idx->ws_f16in.as<uint8_t>();
   }
-  const bool dev_out = is_device_ptr(out);
+  const bool dev_out = is_device_ptr(out) && aligned;
   void* dout = out;
   if (!dev_out) {
     TRY(idx->ws_f16r.ensure(out_b, "f16 prepare output"));

@@ -457,20 +457,32 @@ __global__ void norms_kernel(const __half* __restrict__ x, int64_t items, int32_
   out[g] = acc;
 }
 
-// SIFT u8 -> [RootSIFT] -> * scale -> fp16 (round to nearest even).  One thread per row.
+// SIFT u8 -> [RootSIFT] -> * scale -> fp16 (round to nearest even).  8 lanes per row, 16 bytes in
+// and 32 bytes out each (coalesced); the row's L1 sum is an exact integer in fp32 (<= 32,640).
 __global__ void prepare_kernel(const uint8_t* __restrict__ sift, int64_t rows, int32_t rootsift, float scale,
                                __half* __restrict__ out) {
-  const int64_t r = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
-  if (r >= rows) return;
-  const uint8_t* s = sift + r * kDim;
+  const int64_t g = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+  const int64_t r = g >> 3;
+  const int l8 = static_cast<int>(g & 7);
+  uint4 in = make_uint4(0, 0, 0, 0);
+  if (r < rows) in = reinterpret_cast<const uint4*>(sift + r * kDim)[l8];
+  const uint8_t* b = reinterpret_cast<const uint8_t*>(&in);
   float sum = 0.0f;
-  if (rootsift)
-    for (int i = 0; i < kDim; ++i) sum += static_cast<float>(s[i]);
-  for (int i = 0; i < kDim; ++i) {
-    float v = static_cast<float>(s[i]);
+#pragma unroll
+  for (int i = 0; i < 16; ++i) sum += static_cast<float>(b[i]);
+#pragma unroll
+  for (int o = 1; o < 8; o <<= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+  if (r >= rows) return;
+  __align__(16) __half h[16];
+#pragma unroll
+  for (int i = 0; i < 16; ++i) {
+    float v = static_cast<float>(b[i]);
     if (rootsift) v = sum > 0.0f ? sqrtf(v / sum) : 0.0f;
-    out[r * kDim + i] = __float2half_rn(v * scale);
+    h[i] = __float2half_rn(v * scale);
   }
+  uint4* dst = reinterpret_cast<uint4*>(out + r * kDim) + 2 * l8;
+  dst[0] = reinterpret_cast<const uint4*>(h)[0];
+  dst[1] = reinterpret_cast<const uint4*>(h)[1];
 }
 
 }  // namespace f16
@@ -480,8 +492,8 @@ size_t f16_smem_bytes() { return f16::Plan::kAlloc; }
 cudaError_t launch_f16_prepare(const uint8_t* sift, int64_t rows, int32_t rootsift, float scale, void* out,
                                cudaStream_t s) {
   if (rows <= 0) return cudaSuccess;
-  f16::prepare_kernel<<<static_cast<unsigned>((rows + 127) / 128), 128, 0, s>>>(sift, rows, rootsift, scale,
-                                                                                 static_cast<__half*>(out));
+  f16::prepare_kernel<<<static_cast<unsigned>((rows * 8 + 255) / 256), 256, 0, s>>>(sift, rows, rootsift, scale,
+                                                                                      static_cast<__half*>(out));
   return cudaGetLastError();
 }
 
