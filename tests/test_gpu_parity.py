@@ -154,6 +154,26 @@ def test_host_tier_equals_hbm(tid):
     np.testing.assert_array_equal(ca.astype(np.int64), oracle.search_counts(qs, refs, kp=kp))
 
 
+def test_host_tier_multichunk_references(tid):
+    """Host tier with the paper's m = 384 (two 256-column chunks per reference, Table 7) and ragged
+    kp: streamed chunks of references == the oracle."""
+    R, m, n, B = 90, 384, 500, 2
+    refs, kp = tidgen.refs(3, R, m, kp_min=150, pad_byte=5)
+    qs, _ = tidgen.queries(3, B, n, R_total=R, m=m, kp_min=150)
+    rb = m * 128
+    with tid.Index(ref_kp=m, hbm_budget_bytes=30 * rb, host_budget_bytes=200 * rb) as b:
+        b.set_tuning(host_chunk_refs=16)
+        b.add_references(refs, kp)
+        info = b.info()
+        cb = b.search_counts(qs)
+        ib, nb = b.search(qs, 6)
+    assert info["hbm_references"] == 30 and info["host_references"] == 60
+    e_ids, e_cnt, e_counts = oracle.search(qs, refs, 6, kp=kp)
+    np.testing.assert_array_equal(cb.astype(np.int64), e_counts)
+    np.testing.assert_array_equal(ib, e_ids)
+    np.testing.assert_array_equal(nb, e_cnt)
+
+
 def test_virtual_shards_merge_equals_single(tid):
     """G shards run one after another on one GPU, merged by the shard-merge kernel == 1 GPU."""
     R, m, n, B, k = 96, 256, 300, 3, 6
