@@ -99,6 +99,19 @@ tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t
                               int64_t count, int64_t* first_local_id);
 
 /*
+ * Zero-copy fill of the pinned host tier (level-2 of the hybrid cache, §6.1; pinned
+ * rather than pageable host memory, Table 5): appends `count` references that live in
+ * the host tier and returns, in *desc_out, a pointer to their pinned storage
+ * u8 [count][ref_kp][128] (initialised to zeros = references that match nothing), which the
+ * caller fills in place — no staging copy.  Every reference has ref_kp keypoints.  Contents are
+ * read when a search streams the tier, so they must be written before the next search; the
+ * pointer stays valid until tid_index_destroy.  first_local_id as in tid_add_references.
+ * Errors: TID_EINVAL (count < 1, null desc_out), TID_ENOMEM (host budget exceeded),
+ * TID_ESTATE (cache_policy FIFO: its host tier holds evicted batches only).
+ */
+tid_status tid_host_tier_map(tid_index* idx, int64_t count, uint8_t** desc_out, int64_t* first_local_id);
+
+/*
  * Index lifecycle (the service's delete / update calls; persistence).
  *   tid_delete_references: the given local ids score 0 and are never ranked again.
  *   tid_update_references: replace the descriptors (u8 [count][ref_kp][128], host or device)

@@ -26,7 +26,7 @@ STATUS = {0: "TID_OK", -1: "TID_EINVAL", -2: "TID_ENOMEM", -3: "TID_ECUDA", -4: 
 EXPORTS = ("tid_index_create", "tid_index_destroy", "tid_add_references", "tid_search", "tid_search_counts",
            "tid_verify", "tid_merge_topk", "tid_nccl_unique_id", "tid_get_info", "tid_profile", "tid_get_stats",
            "tid_set_tuning", "tid_delete_references", "tid_update_references", "tid_index_save", "tid_index_load",
-           "tid_f16_prepare", "tid_f16_search_counts", "tid_last_error")
+           "tid_f16_prepare", "tid_f16_search_counts", "tid_host_tier_map", "tid_last_error")
 
 
 class TidError(RuntimeError):
@@ -91,6 +91,7 @@ def load_library(path: str = LIB_PATH):
     lib.tid_index_load.argtypes = [vp, ctypes.c_char_p, P(i64)]
     lib.tid_f16_prepare.argtypes = [vp, vp, i64, i32, ctypes.c_float, vp, vp]
     lib.tid_f16_search_counts.argtypes = [vp, vp, i32, i64, vp, i32, i64, vp, vp]
+    lib.tid_host_tier_map.argtypes = [vp, i64, P(ctypes.POINTER(ctypes.c_uint8)), P(i64)]
     lib.tid_last_error.restype = ctypes.c_char_p
     for name in EXPORTS[:-1]:
         getattr(lib, name).restype = ctypes.c_int
@@ -182,6 +183,17 @@ class Index:
         first = ctypes.c_int64()
         _check(self._lib.tid_add_references(self._h, dp, kp, count, ctypes.byref(first)))
         return first.value
+
+    def host_tier_map(self, count: int):
+        """Zero-copy fill of the pinned host tier: appends `count` references (ref_kp keypoints
+        each) and returns (first local id, numpy u8 view [count][ref_kp][128] of their pinned
+        storage) to be filled in place before the next search.  The view is valid while the
+        index is open."""
+        ptr = ctypes.POINTER(ctypes.c_uint8)()
+        first = ctypes.c_int64()
+        _check(self._lib.tid_host_tier_map(self._h, count, ctypes.byref(ptr), ctypes.byref(first)))
+        view = np.ctypeslib.as_array(ptr, shape=(count, self.ref_kp, 128))
+        return first.value, view
 
     def delete(self, local_ids):
         ids, k1 = _ptr(np.asarray(local_ids, np.int64), np.int64)

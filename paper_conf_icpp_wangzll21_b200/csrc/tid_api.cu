@@ -815,6 +815,32 @@ tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t
   return TID_OK;
 }
 
+tid_status tid_host_tier_map(tid_index* idx, int64_t count, uint8_t** desc_out, int64_t* first_local_id) {
+  if (!idx) return fail(TID_EINVAL, "null index");
+  if (count < 1 || !desc_out) return fail(TID_EINVAL, "count < 1 or null desc_out");
+  if (idx->cfg.cache_policy == 1) return fail(TID_ESTATE, "FIFO policy: the host tier holds evicted batches only");
+  TRY(set_device(idx));
+  const int64_t rb = idx->ref_bytes;
+  const int64_t host_cap = static_cast<int64_t>(idx->host_budget / rb);
+  if (count > host_cap - idx->n_host)
+    return fail(TID_ENOMEM, "host tier room %lld < %lld", static_cast<long long>(host_cap - idx->n_host),
+                static_cast<long long>(count));
+  const int64_t first = idx->n_hbm + idx->n_host;
+  Segment ns;
+  TRY(alloc_segment(idx, true, count, &ns));
+  memset(ns.desc, 0, static_cast<size_t>(count * rb));
+  ns.first = first;
+  ns.count = count;
+  ns.kp.assign(static_cast<size_t>(count), idx->cfg.ref_kp);
+  *desc_out = ns.desc;
+  idx->segs.push_back(std::move(ns));
+  idx->n_host += count;
+  idx->dead.resize(static_cast<size_t>(first + count), 0);
+  idx->dead_dirty = true;
+  if (first_local_id) *first_local_id = first;
+  return TID_OK;
+}
+
 tid_status tid_delete_references(tid_index* idx, const int64_t* local_ids, int64_t count) {
   if (!idx) return fail(TID_EINVAL, "null index");
   if (count < 0 || (count > 0 && !local_ids)) return fail(TID_EINVAL, "bad ids");

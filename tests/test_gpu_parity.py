@@ -174,6 +174,34 @@ def test_host_tier_multichunk_references(tid):
     np.testing.assert_array_equal(nb, e_cnt)
 
 
+def test_host_tier_map_zero_copy(tid):
+    """tid_host_tier_map: references written in place into the pinned tier search like added ones;
+    unwritten (zero) references match nothing; FIFO indexes refuse it."""
+    R, m, n, B = 40, 256, 300, 2
+    refs, _ = tidgen.refs(8, R, m)
+    qs, _ = tidgen.queries(8, B, n, R_total=R, m=m, n_planted=80)
+    rb = m * 128
+    with tid.Index(ref_kp=m, hbm_budget_bytes=10 * rb, host_budget_bytes=64 * rb) as idx:
+        idx.add_references(refs[:10])                 # HBM
+        first, view = idx.host_tier_map(R - 10 + 4)   # pinned tier, filled in place (+4 left zero)
+        assert first == 10 and view.shape == (R - 6, m, 128) and not view.any()
+        view[:R - 10] = refs[10:]
+        info = idx.info()
+        counts = idx.search_counts(qs)
+        ids, cnt = idx.search(qs, 5)
+    assert info["hbm_references"] == 10 and info["host_references"] == R - 6
+    want = oracle.search_counts(qs, refs)
+    np.testing.assert_array_equal(counts[:, :R].astype(np.int64), want)
+    assert (counts[:, R:] == 0).all()
+    e_ids, e_cnt = oracle.topk(np.concatenate([want, np.zeros((B, 4), np.int64)], axis=1), 5)
+    np.testing.assert_array_equal(ids, e_ids)
+    np.testing.assert_array_equal(cnt, e_cnt)
+    with tid.Index(ref_kp=m, hbm_budget_bytes=10 * rb, host_budget_bytes=64 * rb, cache_policy="fifo") as idx:
+        with pytest.raises(tid.TidError) as e:
+            idx.host_tier_map(4)
+        assert e.value.status == tid.TID_ESTATE
+
+
 def test_virtual_shards_merge_equals_single(tid):
     """G shards run one after another on one GPU, merged by the shard-merge kernel == 1 GPU."""
     R, m, n, B, k = 96, 256, 300, 3, 6
