@@ -347,7 +347,8 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         rate, sample, cores, dt = time_oracle(qs_np, refs, args.oracle_seconds)
-        cpu = {"value": rate, "unit": "comparisons/s", "cores": cores, "kind": "oracle", "sample": sample}
+        cpu = {"value": rate, "unit": "comparisons/s", "cores": cores, "kind": "oracle", "sample": sample,
+               "extrapolated_full_step_s": comps / rate}
 
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "comparisons/s", "n_gpus": world, "steps": args.steps,
