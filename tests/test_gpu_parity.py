@@ -420,3 +420,21 @@ def test_abi_errors_and_empty_queries(tid):
     np.testing.assert_array_equal(ids, e_ids)
     np.testing.assert_array_equal(cnt, e_cnt)
     assert (counts[0] == 0).all()
+
+
+def test_search_massive_ties_stress(tid):
+    """SURVEY §8(d) stress variant: K = 16 clusters (non-target counts ~ 0, massive ties) plus exact
+    duplicate references: the (count desc, id asc) ranking must match the oracle element by element."""
+    R, m, n, B, k = 120, 256, 600, 4, 20
+    refs, _ = tidgen.refs(11, R, m, K=16)
+    refs[60:90] = refs[30:60]  # identical copies -> identical counts -> ascending ids
+    qs, _ = tidgen.queries(11, B, n, R_total=R, m=m, K=16, n_planted=40)
+    with tid.Index(ref_kp=m, query_kp_max=1024) as idx:
+        idx.add_references(refs)
+        counts = idx.search_counts(qs)
+        ids, cnt = idx.search(qs, k)
+    e_ids, e_cnt, e_counts = oracle.search(qs, refs, k)
+    np.testing.assert_array_equal(counts.astype(np.int64), e_counts)
+    np.testing.assert_array_equal(counts[:, 30:60], counts[:, 60:90])
+    np.testing.assert_array_equal(ids, e_ids)
+    np.testing.assert_array_equal(cnt, e_cnt)
