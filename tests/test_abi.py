@@ -68,3 +68,15 @@ def test_config_struct_matches_header():
     names = [x for f in fields for x in f if x]
     assert names == [f for f, _ in tid.Config._fields_]
     assert ctypes.sizeof(tid.Config) == 72
+
+
+def test_plain_c_example_compiles_and_links(tmp_path):
+    """include/tid.h is valid C and libtid.so links from a plain C program (examples/search_example.c;
+    running it needs a GPU)."""
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    lib_dir = os.path.join(root, "paper_conf_icpp_wangzll21_b200")
+    out = tmp_path / "search_example"
+    subprocess.check_call(["gcc", "-O2", "-Wall", "-Werror", "-I", os.path.join(root, "include"),
+                           os.path.join(root, "examples", "search_example.c"), "-L", lib_dir, "-ltid",
+                           f"-Wl,-rpath,{lib_dir}", "-o", str(out)])
+    assert out.exists()
