@@ -438,3 +438,19 @@ def test_search_massive_ties_stress(tid):
     np.testing.assert_array_equal(counts[:, 30:60], counts[:, 60:90])
     np.testing.assert_array_equal(ids, e_ids)
     np.testing.assert_array_equal(cnt, e_cnt)
+
+
+def test_plain_c_example_runs(tid, tmp_path):
+    """The C ABI used from plain C (examples/search_example.c, host buffers): planted references rank
+    first; exit status 0."""
+    import os
+    import subprocess
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    lib_dir = os.path.join(root, "paper_conf_icpp_wangzll21_b200")
+    exe = tmp_path / "search_example"
+    subprocess.check_call(["gcc", "-O2", "-I", os.path.join(root, "include"),
+                           os.path.join(root, "examples", "search_example.c"), "-L", lib_dir, "-ltid",
+                           f"-Wl,-rpath,{lib_dir}", "-o", str(exe)])
+    out = subprocess.run([str(exe)], capture_output=True, text=True, timeout=120)
+    assert out.returncode == 0, out.stdout + out.stderr
+    assert "verify(query 0, reference 3): 200 good matches" in out.stdout
