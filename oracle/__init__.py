@@ -261,7 +261,9 @@ def f16_search_counts(Qs16, Rs16, num: int = 4, den: int = 5, n_q=None, kp=None)
 def compression_error(Qf, Rf, Q16, R16) -> float:
     """Eq. 2: mean over all (i, j) of |rho(R_i, Q_j) - rho_FP16(R_i, Q_j)| / rho(R_i, Q_j),
     rho = Euclidean distance; the fp16 distances are those of the fp16-stored (scaled)
-    descriptors, un-scaled by the caller's scale factor (pass Q16/R16 already divided)."""
+    descriptors, un-scaled by the caller's scale factor (pass Q16/R16 already divided), computed
+    exactly in float64 (reading R13).  Pairs with rho = 0 (0/0 in Eq. 2) are left out of the mean
+    (reading R12).  Pinned in closed form by tests/test_oracle_f16.py."""
     rho = np.sqrt(((np.asarray(Rf, np.float64)[:, None, :] - np.asarray(Qf, np.float64)[None, :, :]) ** 2).sum(-1))
     rho16 = np.sqrt(((np.asarray(R16, np.float64)[:, None, :] - np.asarray(Q16, np.float64)[None, :, :]) ** 2).sum(-1))
     ok = rho > 0

@@ -256,3 +256,29 @@ def test_shard_merge_equals_global(rng):
         mi, mc = oracle.merge_topk(li, lc)
         np.testing.assert_array_equal(mi, gi)
         np.testing.assert_array_equal(mc, gc)
+
+
+def test_verify_multi_pair_strides(rng):
+    """oracle_verify over P = 4 pairs with n != m and per-pair n_q[p], m_r[p] (P:31-35,
+    P:284-288): every pair's count and (d1, i1, d2, i2) rows equal the NumPy brute force of
+    that pair alone, and rows j >= n_q[p] stay untouched (-1).  A pair-stride bug (p*m vs
+    p*n, or a shared n_q) puts another pair's keypoints under pair p and fails here."""
+    P, n, m = 4, 37, 23
+    Q = rand_u8(rng, P, n, 128, hi=48)
+    R = rand_u8(rng, P, m, 128, hi=48)
+    for p in range(P):  # distinct planted matches per pair so the pairs' counts differ
+        R[p, : 3 + 4 * p] = Q[p, : 3 + 4 * p]
+    n_q = np.array([37, 20, 5, 31], np.int32)
+    m_r = np.array([23, 2, 17, 9], np.int32)
+    counts, nn = oracle.verify(Q, R, n_q=n_q, m_r=m_r)
+    assert len(set(counts.tolist())) > 2
+    for p in range(P):
+        e = oracle.np_two_nn(Q[p, : n_q[p]], R[p, : m_r[p]])
+        np.testing.assert_array_equal(nn[p, : n_q[p]], e)
+        assert (nn[p, n_q[p]:] == -1).all()
+        assert counts[p] == oracle.np_match_count(Q[p, : n_q[p]], R[p, : m_r[p]])
+    # without n_q / m_r every stored row takes part
+    c2, nn2 = oracle.verify(Q, R)
+    for p in range(P):
+        np.testing.assert_array_equal(nn2[p], oracle.np_two_nn(Q[p], R[p]))
+        assert c2[p] == oracle.np_match_count(Q[p], R[p])

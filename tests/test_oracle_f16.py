@@ -65,3 +65,39 @@ def test_compression_error_eq2(rng):
     rq, rr = oracle.rootsift(Q[0]), oracle.rootsift(R[0])
     e = oracle.compression_error(rq, rr, oracle.to_fp16(rq), oracle.to_fp16(rr))
     assert 0 < e < 5e-3
+
+
+def test_compression_error_eq2_closed_form():
+    """Eq. 2 (P:510-521) on a 2 x 2 case known in closed form.  Queries q1 = 0, q2 = e1;
+    references r1 = 0.1 e1, r2 = 3 e2.  fp16(0.1) = 1638 / 2^14 = 0.1 - 2^-15 * 0.8 =: 0.1 - u
+    (u = 2.44140625e-5); every other value is exact in fp16.  The four distances:
+    rho(r1,q1) = 0.1 (fp16: 0.1 - u), rho(r1,q2) = 0.9 (fp16: 0.9 + u), rho(r2,q*) exact
+    (3, sqrt 10).  Eq. 2 = (u/0.1 + u/0.9 + 0 + 0) / (m*n = 4) = u * 25/9.
+    Mistakes this catches: rho^2 instead of rho (about 2x), dividing by rho_FP16 (relative
+    2.4e-4), averaging over the two non-zero terms only (1.8x), a dropped |.|."""
+    u = 2.0 ** -15 * 0.8
+    Qf = np.zeros((2, 128))
+    Qf[1, 0] = 1.0
+    Rf = np.zeros((2, 128))
+    Rf[0, 0] = 0.1
+    Rf[1, 1] = 3.0
+    Q16 = oracle.to_fp16(Qf).astype(np.float64)
+    R16 = oracle.to_fp16(Rf).astype(np.float64)
+    assert R16[0, 0] == 1638 / 2 ** 14 == 0.1 - u
+    e = oracle.compression_error(Qf, Rf, Q16, R16)
+    np.testing.assert_allclose(e, u * 25 / 9, rtol=1e-12)
+    # transposing the roles (m x n vs n x m) leaves the mean unchanged
+    np.testing.assert_allclose(oracle.compression_error(Rf, Qf, R16, Q16), u * 25 / 9, rtol=1e-12)
+
+
+def test_compression_error_zero_distance_pairs_excluded():
+    """Reading (DESIGN.md R12): Eq. 2 divides by rho, undefined (0/0) for identical descriptors;
+    those pairs are left out of the mean.  q = r = 0.1 e1 (rho = rho_FP16 = 0) plus
+    q2 = 0 (rho = 0.1, rho_FP16 = 0.1 - u): the mean is over the one defined pair, u / 0.1."""
+    u = 2.0 ** -15 * 0.8
+    Qf = np.zeros((2, 128))
+    Qf[0, 0] = 0.1
+    Rf = np.zeros((1, 128))
+    Rf[0, 0] = 0.1
+    e = oracle.compression_error(Qf, Rf, oracle.to_fp16(Qf).astype(np.float64), oracle.to_fp16(Rf).astype(np.float64))
+    np.testing.assert_allclose(e, u / 0.1, rtol=1e-12)
