@@ -8,8 +8,14 @@ per-GPU shard is fixed as N grows; the per-rank top-k lists are merged with one 
 all-gather.  One step = one tid_search over the whole batch (every §8(a) row: query prep,
 fused TMA->tcgen05->top-2->ratio->count kernel over all references, top-k, shard merge).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config c4|c3|c5|c1]
     torchrun --nproc-per-node N bench.py --gpus N ...
+
+`--gpus N` without a torchrun environment (no WORLD_SIZE) re-launches this script under
+`torch.distributed.run --nproc-per-node N` (127.0.0.1, a free port): one process per GPU, NCCL,
+NCCL_DEBUG=INFO (INIT lines to stderr show the communicator's rank count).  `--dry-run` runs
+the same rank / shard / merge / max-over-ranks plumbing on CPU over gloo (no GPU; the per-rank
+work is the oracle on a tiny shard) and prints the plan as JSON: a host-logic check.
 
 Rank 0 prints ONE JSON line.  `value` = whole-job comparisons/s with queries resident in
 HBM; `e2e` = the same metric through the public API with pinned-host queries in and host
@@ -38,6 +44,9 @@ CONFIGS = {
     "c4": (256, 1000, 125_000, 256, 5),
     "c3": (64, 1000, 100_000, 256, 5),
     "c1": (1, 256, 64, 256, 5),
+    # C5 (hybrid host cache, configs[4]): per GPU, HBM-resident references + a pinned host tier
+    # streamed through HBM on every search; sizes chosen at run time from free HBM / host RAM
+    "c5": (256, 1000, 0, 256, 5),
 }
 RATIO = (4, 5)
 SEED = 2021
@@ -193,11 +202,134 @@ def config_dict(cfg_name, G):
     B, n, Rg, m, k = CONFIGS[cfg_name]
     return {"workload": {"c4": "C4: 256 queries x 1M references sharded 8-way (125,000 refs per GPU; weak scaling)",
                          "c3": "C3: 64 queries vs 100,000 references per GPU",
-                         "c1": "C1: 1 query vs 64 references"}[cfg_name],
+                         "c1": "C1: 1 query vs 64 references",
+                         "c5": "C5: hybrid host cache - up to 10M references over the GPUs; per GPU the "
+                               "HBM-resident part plus a pinned host tier streamed through HBM every search "
+                               f"(B = {B}; 'c5' key: the split actually held)"}[cfg_name],
             "queries": B, "query_kp": n, "refs_per_gpu": Rg, "refs_total": Rg * G, "ref_kp": m, "dim": 128,
             "top_k": k, "ratio": f"{RATIO[0]}/{RATIO[1]}", "parallelism": f"ref-shard x{G}" + (
                 " + NCCL all-gather top-k" if G > 1 else ""),
             "l2": "inputs larger than L2 (reference shard %.1f GB/GPU >> 126 MB)" % (Rg * m * 128 / 1e9)}
+
+
+# ----------------------------------------------------------------------------- multi-rank plumbing
+def relaunch(n: int) -> int:
+    """`bench.py --gpus N` outside torchrun: start N ranks (one per GPU) under
+    torch.distributed.run on this node and return its exit code.  Only rank 0 prints."""
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    env.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")  # keep stdout = the one JSON line
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    log("launching: " + " ".join(cmd))
+    return subprocess.call(cmd, env=env)
+
+
+def dry_run(args):
+    """The multi-rank host logic of the bench on CPU (gloo): shard plan, per-rank local top-k,
+    all-gather + merge in the shared total order, max over ranks.  The per-rank matching is the
+    oracle on a tiny shard (this is a plumbing check, not a measurement)."""
+    import torch
+    import torch.distributed as dist
+
+    import oracle
+    import tidgen
+    from paper_conf_icpp_wangzll21_b200.dist import shard_plan
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if world > 1:
+        dist.init_process_group("gloo")
+    Rg, m, n, B, k = 6, 64, 80, 3, 4
+    start, end = shard_plan(Rg * world, world, rank)
+    refs, _ = tidgen.refs(start, end - start, m, seed=SEED)
+    qs, targets = tidgen.queries(0, B, n, R_total=Rg * world, m=m, n_planted=30, seed=SEED)
+    t0 = time.perf_counter()
+    ids, cnt = oracle.topk(oracle.search_counts(qs, refs), k, id_base=start)
+    dt = time.perf_counter() - t0
+    spans = [(start, end)]
+    if world > 1:
+        gi = [torch.zeros((B, k), dtype=torch.int64) for _ in range(world)]
+        gc = [torch.zeros((B, k), dtype=torch.int32) for _ in range(world)]
+        dist.all_gather(gi, torch.from_numpy(ids))
+        dist.all_gather(gc, torch.from_numpy(cnt))
+        ids, cnt = oracle.merge_topk(np.stack([t.numpy() for t in gi]), np.stack([t.numpy() for t in gc]))
+        sp = [None] * world
+        dist.all_gather_object(sp, (start, end))
+        spans = sp
+        t = torch.tensor([dt], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dt = float(t.item())
+    if rank == 0:
+        print(json.dumps({"dry_run": True, "n_gpus": world, "shards": spans, "refs_total": Rg * world,
+                          "planted_top1": float(np.mean(ids[:, 0] == targets)), "max_rank_s": dt,
+                          "top_ids": ids.tolist()}), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+# ----------------------------------------------------------------------------- C5: hybrid host cache
+def mem_available() -> int:
+    try:
+        for line in open("/proc/meminfo"):
+            if line.startswith("MemAvailable:"):
+                return int(line.split()[1]) * 1024
+    except OSError:
+        pass
+    return 0
+
+
+def build_c5(args, tid, tidgen, torch, dist, world, rank, local, nccl_id, m):
+    """configs[4] (§6.1, Table 6): this rank's share of the
+    --c5-refs reference set, HBM-resident up to the library's automatic HBM budget (level 1) and
+    the rest in the pinned host tier (level 2), filled IN PLACE by the generator through
+    tid_host_tier_map (no staging copy), streamed through HBM on every search.  When the host
+    cannot pin the rest, the shard is what fits (stated in the JSON line)."""
+    want = -(-args.c5_refs // world)
+    rb = m * 128
+    host_bytes = int(args.c5_host_frac * mem_available() / max(1, torch.cuda.device_count() if world > 1 else 1))
+    probe = tid.Index(ref_kp=m, device=local)
+    hbm_cap = probe.info()["hbm_capacity_references"]
+    probe.close()
+    n_hbm = min(want, hbm_cap)
+    n_host = min(want - n_hbm, host_bytes // rb)
+    Rg = n_hbm + n_host
+    if world > 1:  # equal shards: the smallest any rank can hold
+        t = torch.tensor([Rg, n_hbm], dtype=torch.int64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MIN)
+        Rg, n_hbm = int(t[0]), min(n_hbm, int(t[1]))
+        n_host = Rg - n_hbm
+    start = rank * Rg
+    idx = tid.Index(ref_kp=m, query_kp_max=1024, ratio=RATIO, device=local, id_base=start, rank=rank,
+                    world_size=world, nccl_id=nccl_id, host_budget_bytes=n_host * rb)
+    t0 = time.perf_counter()
+    step = 65536
+    for off in range(0, n_hbm, step):
+        c = min(step, n_hbm - off)
+        r, _ = tidgen.refs(start + off, c, m, seed=SEED)
+        idx.add_references(r)
+    t_hbm = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    if n_host:
+        first, view = idx.host_tier_map(n_host)
+        assert first == n_hbm
+        for off in range(0, n_host, step):
+            c = min(step, n_host - off)
+            tidgen.refs(start + n_hbm + off, c, m, seed=SEED, out=view[off:off + c])
+    t_host = time.perf_counter() - t0
+    info = idx.info()
+    log(f"[rank {rank}] c5: {n_hbm} HBM refs ({t_hbm:.0f}s) + {n_host} host-tier refs filled in place "
+        f"({t_host:.0f}s); info {info}")
+    sample = min(n_hbm, 65536)
+    refs, _ = tidgen.refs(start, sample, m, seed=SEED)  # oracle sample (cpu_baseline)
+    c5 = {"refs_requested_total": args.c5_refs, "refs_per_gpu": Rg, "hbm_refs_per_gpu": n_hbm,
+          "host_tier_refs_per_gpu": n_host, "host_tier_bytes_per_gpu": n_host * rb,
+          "hbm_capacity_refs": hbm_cap, "hbm_bytes_per_ref": info["hbm_bytes_per_reference"]}
+    return idx, refs, start, Rg, c5
 
 
 # ----------------------------------------------------------------------------- our arm
@@ -211,6 +343,11 @@ def main():
     ap.add_argument("--refs-per-gpu", type=int, default=0, help="override the per-GPU reference count")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--oracle-seconds", type=float, default=12.0)
+    ap.add_argument("--dry-run", action="store_true", help="CPU/gloo check of the multi-rank plumbing (no GPU)")
+    ap.add_argument("--batch", type=int, default=0, help="override the query batch B")
+    ap.add_argument("--c5-refs", type=int, default=10_000_000, help="c5: total references (all ranks)")
+    ap.add_argument("--c5-host-frac", type=float, default=0.6,
+                    help="c5: share of this rank's MemAvailable the pinned host tier may take")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
@@ -218,6 +355,11 @@ def main():
         B, n, _, m, k = CONFIGS[args.config]
         CONFIGS[args.config] = (B, n, args.refs_per_gpu, m, k)
 
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(relaunch(args.gpus))
+    if args.dry_run:
+        dry_run(args)
+        return
     if args.impl == "reference":
         run_reference(args, args.config)
         return
@@ -228,6 +370,7 @@ def main():
     import tidgen
     import paper_conf_icpp_wangzll21_b200 as tid
 
+    from paper_conf_icpp_wangzll21_b200.dist import shard_plan
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
@@ -237,23 +380,32 @@ def main():
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     B, n, Rg, m, k = CONFIGS[args.config]
-    start = rank * Rg
-    t0 = time.perf_counter()
-    refs, _ = tidgen.refs(start, Rg, m, seed=SEED)
-    # queries: pinned host copy (for e2e) + device copy (for the device-resident value)
-    qs_np, targets = tidgen.queries(0, B, n, R_total=Rg * world, m=m, seed=SEED)
-    log(f"[rank {rank}] generated {Rg} refs + {B} queries in {time.perf_counter() - t0:.1f}s")
-
+    if args.batch:
+        B = args.batch
+        CONFIGS[args.config] = (B, n, Rg, m, k)
     nccl_id = None
     if world > 1:
         obj = [tid.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         nccl_id = obj[0]
-    idx = tid.Index(ref_kp=m, query_kp_max=1024, ratio=RATIO, device=local, id_base=start, rank=rank,
-                    world_size=world, nccl_id=nccl_id)
-    t0 = time.perf_counter()
-    idx.add_references(refs)
-    log(f"[rank {rank}] ingest {time.perf_counter() - t0:.1f}s; info {idx.info()}")
+    c5 = None
+    if args.config == "c5":
+        idx, refs, start, Rg, c5 = build_c5(args, tid, tidgen, torch, dist, world, rank, local, nccl_id, m)
+        CONFIGS["c5"] = (B, n, Rg, m, k)
+        qs_np, targets = tidgen.queries(0, B, n, R_total=Rg * world, m=m, seed=SEED)
+    else:
+        start, end = shard_plan(Rg * world, world, rank)  # contiguous id shards
+        assert end - start == Rg
+        t0 = time.perf_counter()
+        refs, _ = tidgen.refs(start, Rg, m, seed=SEED)
+        # queries: pinned host copy (for e2e) + device copy (for the device-resident value)
+        qs_np, targets = tidgen.queries(0, B, n, R_total=Rg * world, m=m, seed=SEED)
+        log(f"[rank {rank}] generated {Rg} refs + {B} queries in {time.perf_counter() - t0:.1f}s")
+        idx = tid.Index(ref_kp=m, query_kp_max=1024, ratio=RATIO, device=local, id_base=start, rank=rank,
+                        world_size=world, nccl_id=nccl_id)
+        t0 = time.perf_counter()
+        idx.add_references(refs)
+        log(f"[rank {rank}] ingest {time.perf_counter() - t0:.1f}s; info {idx.info()}")
 
     dq = torch.from_numpy(qs_np).cuda()
     hq = torch.from_numpy(qs_np).pin_memory()
@@ -344,20 +496,26 @@ def main():
                             "below the tensor peak; see DESIGN.md section 7",
             "pipes_ncu": pipes_from_profile(traffic)}
 
+    # CPU oracle on rank 0's host cores, after every timed region (the other ranks wait)
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and not args.no_cpu_baseline:
         rate, sample, cores, dt = time_oracle(qs_np, refs, args.oracle_seconds)
         cpu = {"value": rate, "unit": "comparisons/s", "cores": cores, "kind": "oracle", "sample": sample,
                "extrapolated_full_step_s": comps / rate}
+    if world > 1:
+        dist.barrier()
 
     if rank == 0:
+        info = idx.info()
         line = {"metric": METRIC, "value": value, "unit": "comparisons/s", "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
                 "vs_baseline": None, "dtype": "u8", "data": "synthetic (tidgen: clustered u8 SIFT-like descriptors, "
                 "200 planted matches per query)", "config": config_dict(args.config, world),
                 "p50_search_latency_ms": p50, "clocks": clk.summary(), "e2e": e2e,
                 "gpu_launches": int(st["kernel_launches"]), "roofline": roof, "cpu_baseline": cpu,
-                "planted_top1": planted_ok}
+                "planted_top1": planted_ok, "c5": c5,
+                "nccl": {"comm_nranks": info["world_size"], "merge": "ncclAllGather of B*k u64 keys + GPU merge"}
+                if world > 1 else None}
         print(json.dumps(line), flush=True)
     idx.close()
     if world > 1:

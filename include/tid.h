@@ -25,7 +25,9 @@
  *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
  *     Device outputs are valid once `stream` completes; host outputs are valid
  *     when the call returns (the call synchronises the stream).
- *   - One index per host thread; an index is not thread-safe.
+ *   - One index per host thread; an index is not thread-safe.  Successive calls on one index
+ *     may pass different streams: each call's work is ordered after the previous call's
+ *     (the index records an event at the end of every call and the next call waits on it).
  *   - The library requires an sm_100a device (B200): TID_EUNSUPPORTED otherwise.
  *     There is no CPU fallback.
  */
@@ -60,8 +62,8 @@ typedef struct {
   uint32_t ratio_den;
   uint64_t hbm_budget_bytes;   /* reference descriptor bytes kept resident in HBM (level-1 cache,
                                   §6.1); 0 = auto (free HBM minus 8 GiB workspace).
-                                  Each resident reference additionally holds ref_kp*32 bytes of
-                                  norm-term digits and ceil(ref_kp/256) KiB of column terms.      */
+                                  Each resident reference additionally holds ceil(ref_kp/256) KiB
+                                  of column terms (W = 256 sum r - N_R per keypoint).             */
   uint64_t host_budget_bytes;  /* pinned host tier capacity in bytes (level-2 cache); 0 = none    */
   int64_t  id_base;            /* global id of this rank's first reference (shard offset)         */
   int32_t  rank;               /* this process's rank; 0 when world_size == 1                     */
@@ -92,7 +94,10 @@ tid_status tid_index_destroy(tid_index* idx);
  *   first_local_id (out, nullable): local index of the first appended reference;
  *                its global id is cfg.id_base + local index.
  * References go to HBM until hbm_budget_bytes, then to the pinned host tier until
- * host_budget_bytes (FIFO order preserved).  All-or-nothing: TID_ENOMEM adds nothing.
+ * host_budget_bytes (FIFO order preserved).  All-or-nothing: on any error (TID_ENOMEM,
+ * TID_ECUDA, ...) no reference is added and ids are unchanged (under cache_policy FIFO, batches
+ * already swapped out to the host tier to make room stay there: tier placement only, never
+ * results).
  * The squared norms N_R are computed here and kept in HBM.
  */
 tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t* kp_counts,
@@ -131,8 +136,12 @@ tid_status tid_index_load(tid_index* idx, const char* path, int64_t* first_local
  * One-to-many search, batched over B queries.
  *   queries          : u8 [B][n][128], host or device; n <= query_kp_max.
  *   n_q              : int32 [B] valid keypoints per query (<= n), host or device; NULL = all n.
- *   k                : 1..64 and k <= total references over all ranks (deleted references are
- *                      never ranked: if fewer than k live references exist, the tail is id -1).
+ *   k                : 1..64 and k <= total references over all ranks, else TID_EINVAL on every
+ *                      rank (with world_size > 1 the total is all-reduced first, so all ranks
+ *                      decide alike).  Deleted references are never ranked: if fewer than k
+ *                      live references exist, the tail is id -1, count 0.
+ *                      A rank whose shard is empty still takes part (it contributes no
+ *                      candidates); TID_ESTATE only when no rank holds a reference.
  *   ref_ids_out      : int64 [B][k]  global reference ids, rank order (count desc, id asc).
  *   match_counts_out : int32 [B][k]  their good-match counts.
  * With world_size > 1 the call is collective: every rank passes the same queries
@@ -211,7 +220,11 @@ typedef struct {
   int64_t hbm_bytes;           /* device bytes allocated by the index                */
   int64_t host_bytes;          /* pinned host bytes allocated by the index           */
   int32_t num_sms;
-  int32_t world_size;
+  int32_t world_size;          /* shards; with an NCCL communicator, ncclCommCount's rank count */
+  int64_t hbm_capacity_references;  /* references the HBM budget holds (resident tier capacity) */
+  int64_t host_capacity_references; /* references the pinned host budget holds                  */
+  int64_t hbm_bytes_per_reference;  /* HBM bytes one resident reference occupies (descriptors +
+                                       per-keypoint norm terms + column terms)                   */
 } tid_info;
 
 tid_status tid_get_info(const tid_index* idx, tid_info* out);
@@ -233,15 +246,15 @@ tid_status tid_get_stats(tid_index* idx, tid_stats* out); /* synchronises record
 
 /* Tuning knobs (0 = automatic).  refs_per_job: references resident per CTA job (1..4);
  * grid: persistent CTAs for the match kernel; host_chunk_refs: references per
- * host-tier staging buffer; exact_only: accepted for ABI stability and ignored (every
- * scan is exact; the search path recomputes the rare +-1-undecided rows exactly).
- * Results never depend on these knobs. */
+ * host-tier staging buffer; window_refs: references per count window of tid_search
+ * (automatic: the whole local set while its B x R u32 count matrix fits 512 MiB, else
+ * 512 MiB / (4 B) references; each window's counts are reduced into a running top-k, so the
+ * search workspace does not grow with R).  Results never depend on these knobs. */
 typedef struct {
   int32_t refs_per_job;
   int32_t grid;
   int64_t host_chunk_refs;
-  int32_t exact_only;
-  int32_t reserved;
+  int64_t window_refs;
 } tid_tuning;
 
 tid_status tid_set_tuning(tid_index* idx, const tid_tuning* t);

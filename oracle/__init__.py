@@ -60,6 +60,7 @@ def _L():
         lib.oracle_search_counts.argtypes = [vp, vp, i32, i64, vp, vp, i32, i64, u32, u32, vp]
         lib.oracle_topk.argtypes = [vp, i64, i64, i64, i32, vp, vp]
         lib.oracle_merge_topk.argtypes = [vp, vp, i32, i64, i32, vp, vp]
+        lib.oracle_f64_search_counts.argtypes = [vp, vp, i32, i64, vp, vp, i32, i64, u32, u32, vp]
         _lib = lib
     return _lib
 
@@ -256,6 +257,21 @@ def f16_search_counts(Qs16, Rs16, num: int = 4, den: int = 5, n_q=None, kp=None)
             out[b, r] = f16_match_count(Qs16[b], Rs16[r], num, den, None if n_q is None else n_q[b],
                                         None if kp is None else kp[r])
     return out
+
+
+def f16_search_counts_c(Qs16, Rs16, num: int = 4, den: int = 5, n_q=None, kp=None) -> np.ndarray:
+    """The same counts as ``f16_search_counts`` from the C oracle (float64 direct sums, OpenMP over
+    pairs; oracle_f64_search_counts) — for sizes the NumPy formulation cannot reach.  Pinned
+    against the NumPy formulation and the exact integer oracle in tests/test_oracle_f16.py."""
+    Q = np.ascontiguousarray(np.asarray(Qs16, np.float16).astype(np.float64))
+    R = np.ascontiguousarray(np.asarray(Rs16, np.float16).astype(np.float64))
+    B, n = Q.shape[0], Q.shape[1]
+    Rn, m = R.shape[0], R.shape[1]
+    nq = None if n_q is None else _c(n_q, np.int32)
+    kpa = None if kp is None else _c(kp, np.int32)
+    counts = np.empty((B, Rn), np.int32)
+    _L().oracle_f64_search_counts(_p(Q), _p(nq), n, B, _p(R), _p(kpa), m, Rn, num, den, _p(counts))
+    return counts
 
 
 def compression_error(Qf, Rf, Q16, R16) -> float:

@@ -171,3 +171,41 @@ void oracle_merge_topk(const int64_t* ids, const int32_t* cnts, int32_t G, int64
   }
   free(c);
 }
+
+/*
+ * f1 float path (§4.2, §5.1, Alg. 2):
+ * good-match counts of B queries against R references whose descriptors are fp16 values,
+ * passed here already widened to double (exact).  The same definition as above, in float64:
+ * d = sum_t (q_t - r_t)^2 summed in index order, 2-NN per query row by a value scan (for the
+ * count only the two smallest distances matter), ratio test on squared distances in
+ * the rational form of reading R1, den^2 * d1 < num^2 * d2 (strict), reading R3 for m_r < 2.
+ */
+void oracle_f64_search_counts(const double* Qs, const int32_t* n_q, int32_t n, int64_t B,
+                              const double* Rs, const int32_t* kp, int32_t m, int64_t R,
+                              uint32_t num, uint32_t den, int32_t* counts) {
+  const double n2 = (double)num * (double)num, d2c = (double)den * (double)den;
+#pragma omp parallel for collapse(2) schedule(dynamic, 16)
+  for (int64_t b = 0; b < B; ++b)
+    for (int64_t r = 0; r < R; ++r) {
+      const int32_t nq = n_q ? n_q[b] : n, mr = kp ? kp[r] : m;
+      int32_t c = 0;
+      if (mr >= 2) {
+        for (int32_t j = 0; j < nq; ++j) {
+          const double* q = Qs + ((size_t)b * n + j) * DIM;
+          double d1 = 1.0 / 0.0, d2 = 1.0 / 0.0;
+          for (int32_t i = 0; i < mr; ++i) {
+            const double* x = Rs + ((size_t)r * m + i) * DIM;
+            double d = 0.0;
+            for (int t = 0; t < DIM; ++t) {
+              const double df = q[t] - x[t];
+              d += df * df;
+            }
+            if (d < d1) { d2 = d1; d1 = d; }
+            else if (d < d2) { d2 = d; }
+          }
+          c += d2c * d1 < n2 * d2;
+        }
+      }
+      counts[b * R + r] = c;
+    }
+}

@@ -46,7 +46,9 @@ class Config(ctypes.Structure):
 class Info(ctypes.Structure):
     _fields_ = [("num_references", ctypes.c_int64), ("hbm_references", ctypes.c_int64),
                 ("host_references", ctypes.c_int64), ("hbm_bytes", ctypes.c_int64), ("host_bytes", ctypes.c_int64),
-                ("num_sms", ctypes.c_int32), ("world_size", ctypes.c_int32)]
+                ("num_sms", ctypes.c_int32), ("world_size", ctypes.c_int32),
+                ("hbm_capacity_references", ctypes.c_int64), ("host_capacity_references", ctypes.c_int64),
+                ("hbm_bytes_per_reference", ctypes.c_int64)]
 
 
 class Stats(ctypes.Structure):
@@ -56,7 +58,7 @@ class Stats(ctypes.Structure):
 
 class Tuning(ctypes.Structure):
     _fields_ = [("refs_per_job", ctypes.c_int32), ("grid", ctypes.c_int32), ("host_chunk_refs", ctypes.c_int64),
-                ("exact_only", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("window_refs", ctypes.c_int64)]
 
 
 _lib = None
@@ -109,15 +111,46 @@ def _is_torch(x):
     return type(x).__module__.startswith("torch")
 
 
+_TORCH_DT = {np.uint8: "torch.uint8", np.int32: "torch.int32", np.int64: "torch.int64", np.uint32: "torch.uint32",
+             np.float16: "torch.float16"}
+
+
 def _ptr(x, dtype=None):
-    """(pointer, keepalive) of a C-contiguous numpy array / torch tensor; None passes NULL."""
+    """(pointer, keepalive) of an INPUT: a numpy array (converted to a C-contiguous copy of
+    `dtype` if needed) or a torch tensor (must already be contiguous and of `dtype`); None
+    passes NULL."""
     if x is None:
         return None, None
     if _is_torch(x):
-        assert x.is_contiguous(), "tensor must be contiguous"
+        if not x.is_contiguous():
+            raise ValueError("tensor must be contiguous")
+        if dtype is not None and str(x.dtype) != _TORCH_DT[dtype]:
+            raise TypeError(f"tensor dtype {x.dtype}, expected {_TORCH_DT[dtype]}")
         return x.data_ptr(), x
     a = np.ascontiguousarray(x, dtype=dtype)
     return a.ctypes.data, a
+
+
+def _out_ptr(x, shape, dtype, device: int, what: str):
+    """Pointer of a caller-supplied OUTPUT buffer, checked instead of converted (a converted copy
+    would silently drop the results; a smaller or narrower buffer would be overrun): exact
+    shape and dtype, C-contiguous and writable, and — for a CUDA tensor — on the index's device."""
+    shape = tuple(int(v) for v in shape)
+    if _is_torch(x):
+        if tuple(x.shape) != shape or str(x.dtype) != _TORCH_DT[dtype]:
+            raise TypeError(f"{what}: got {tuple(x.shape)} {x.dtype}, expected {shape} {_TORCH_DT[dtype]}")
+        if not x.is_contiguous():
+            raise ValueError(f"{what}: tensor must be contiguous")
+        if x.is_cuda and x.device.index != device:
+            raise ValueError(f"{what}: tensor on {x.device}, the index is on cuda:{device}")
+        return x.data_ptr()
+    if not isinstance(x, np.ndarray):
+        raise TypeError(f"{what}: expected a numpy array or torch tensor, got {type(x).__name__}")
+    if x.shape != shape or x.dtype != np.dtype(dtype):
+        raise TypeError(f"{what}: got {x.shape} {x.dtype}, expected {shape} {np.dtype(dtype)}")
+    if not x.flags["C_CONTIGUOUS"] or not x.flags["WRITEABLE"]:
+        raise ValueError(f"{what}: array must be C-contiguous and writable")
+    return x.ctypes.data
 
 
 def _stream(*tensors):
@@ -224,8 +257,8 @@ class Index:
             ids, cnt = np.empty((B, k), np.int64), np.empty((B, k), np.int32)
         else:
             ids, cnt = out
-        ip, k3 = _ptr(ids)
-        cp, k4 = _ptr(cnt)
+        ip = _out_ptr(ids, (B, k), np.int64, self.device, "ids")
+        cp = _out_ptr(cnt, (B, k), np.int32, self.device, "counts")
         _check(self._lib.tid_search(self._h, qp, nqp, n, B, k, ip, cp, _stream(queries, ids)))
         return ids, cnt
 
@@ -237,7 +270,7 @@ class Index:
         nqp, k2 = _ptr(n_q, np.int32)
         if out is None:
             out = np.empty((B, R), np.uint32)
-        op, k3 = _ptr(out)
+        op = _out_ptr(out, (B, R), np.uint32, self.device, "counts")
         _check(self._lib.tid_search_counts(self._h, qp, nqp, n, B, op, _stream(queries, out)))
         return out
 
@@ -251,7 +284,7 @@ class Index:
         sp, k1 = _ptr(sift, np.uint8)
         if out is None:
             out = np.empty(shp, np.float16)
-        op, k2 = _ptr(out)
+        op = _out_ptr(out, shp, np.float16, self.device, "out")
         _check(self._lib.tid_f16_prepare(self._h, sp, rows, 1 if rootsift else 0, float(scale), op,
                                          _stream(sift, out)))
         return out
@@ -265,7 +298,7 @@ class Index:
         rp, k2 = _ptr(r16, np.float16)
         if out is None:
             out = np.empty((B, R), np.uint32)
-        op, k3 = _ptr(out)
+        op = _out_ptr(out, (B, R), np.uint32, self.device, "counts")
         _check(self._lib.tid_f16_search_counts(self._h, qp, n, B, rp, m, R, op, _stream(q16, out)))
         return out
 
@@ -283,8 +316,8 @@ class Index:
             nn = np.empty((P, n, 4), np.int32) if want_nn else None
         else:
             counts, nn = out
-        cp, k5 = _ptr(counts)
-        np_, k6 = _ptr(nn)
+        cp = _out_ptr(counts, (P,), np.uint32, self.device, "counts")
+        np_ = None if nn is None else _out_ptr(nn, (P, n, 4), np.int32, self.device, "nn")
         _check(self._lib.tid_verify(self._h, qp, n, rp, m, P, nqp, mrp, cp, np_, _stream(q, r, counts)))
         return counts, nn
 
@@ -310,8 +343,8 @@ class Index:
         _check(self._lib.tid_get_stats(self._h, ctypes.byref(s)))
         return {f: getattr(s, f) for f, _ in Stats._fields_}
 
-    def set_tuning(self, refs_per_job: int = 0, grid: int = 0, host_chunk_refs: int = 0, exact_only: bool = False):
-        t = Tuning(refs_per_job, grid, host_chunk_refs, 1 if exact_only else 0, 0)
+    def set_tuning(self, refs_per_job: int = 0, grid: int = 0, host_chunk_refs: int = 0, window_refs: int = 0):
+        t = Tuning(refs_per_job, grid, host_chunk_refs, window_refs)
         _check(self._lib.tid_set_tuning(self._h, ctypes.byref(t)))
 
 

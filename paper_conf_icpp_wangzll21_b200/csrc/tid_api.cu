@@ -50,7 +50,9 @@ struct NcclApi {
   ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
   ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
   ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t, cudaStream_t) = nullptr;
   const char* (*GetErrorString)(ncclResult_t) = nullptr;
+  ncclResult_t (*CommCount)(const ncclComm_t, int*) = nullptr;
 };
 
 const NcclApi& nccl() {
@@ -73,7 +75,10 @@ const NcclApi& nccl() {
   api.CommDestroy = reinterpret_cast<decltype(api.CommDestroy)>(dlsym(h, "ncclCommDestroy"));
   api.AllGather = reinterpret_cast<decltype(api.AllGather)>(dlsym(h, "ncclAllGather"));
   api.GetErrorString = reinterpret_cast<decltype(api.GetErrorString)>(dlsym(h, "ncclGetErrorString"));
-  api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.AllGather && api.GetErrorString;
+  api.AllReduce = reinterpret_cast<decltype(api.AllReduce)>(dlsym(h, "ncclAllReduce"));
+  api.CommCount = reinterpret_cast<decltype(api.CommCount)>(dlsym(h, "ncclCommCount"));
+  api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.AllGather && api.AllReduce &&
+           api.GetErrorString;
   if (!api.ok) api.err = "libnccl.so.2 lacks a required symbol";
   return api;
 }
@@ -249,7 +254,6 @@ struct Segment {
   bool on_host = false;
   uint8_t* desc = nullptr;    // [cap][m][128]: device (HBM) or pinned host
   int32_t* colkey = nullptr;  // device, HBM segments only: [cap][cpr][256] column terms W (search)
-  uint8_t* extra = nullptr;   // device, HBM segments only: [cap][m][32] norm-term digits (search MMA)
   int64_t cap = 0, count = 0, first = 0;
   std::vector<int32_t> kp;    // keypoint count per reference (0 = deleted / empty)
 };
@@ -272,11 +276,16 @@ struct tid_index {
   int64_t hbm_alloc = 0, host_alloc = 0;
   cudaStream_t copy_stream = nullptr;
   cudaEvent_t ev_h2d[2] = {nullptr, nullptr}, ev_free[2] = {nullptr, nullptr};
+  // every call that touches the workspaces waits for the previous call's work (whatever stream it
+  // ran on) and records this event at its end: one index may be driven from several streams
+  cudaEvent_t ev_last = nullptr;
   // workspaces
   DevBuf ws_q, ws_nq, ws_nvalid, ws_counts, ws_cand, ws_keys, ws_gather, ws_ids, ws_cnts, ws_r, ws_colkey, ws_nn,
       ws_kp, ws_mr;
-  DevBuf stage_desc[2], stage_colkey[2], stage_kp[2], stage_extra[2];
+  DevBuf stage_desc[2], stage_colkey[2], stage_kp[2];
   DevBuf ws_qs;                   // shifted queries q' = q ^ 0x80 (search)
+  DevBuf ws_rtot;                 // collective reference count (all-reduce)
+  int64_t* h_rtot = nullptr;      // pinned host copy of it
   DevBuf ws_f16q, ws_f16r, ws_f16nq, ws_f16nr, ws_f16in;  // f1 float path
   int64_t host_chunk = 0;
   tid_tuning tune{};
@@ -298,6 +307,16 @@ tid_status set_device(tid_index* idx) {
 void count_kernel(tid_index* idx, int n = 1) {
   if (idx->prof) idx->stats.kernel_launches += n;
 }
+
+// Cross-call ordering of the per-index workspaces (see tid_index::ev_last): the constructor makes
+// `s` wait for everything the previous call enqueued; the destructor records the end of this call
+// (also on early error returns, so partially enqueued work is still ordered before the next call).
+struct CallGuard {
+  tid_index* idx;
+  cudaStream_t s;
+  CallGuard(tid_index* i, cudaStream_t st) : idx(i), s(st) { cudaStreamWaitEvent(s, idx->ev_last, 0); }
+  ~CallGuard() { cudaEventRecord(idx->ev_last, s); }
+};
 
 tid_status copy_in(tid_index* idx, void* dst, const void* src, size_t bytes, cudaStream_t s) {
   if (bytes == 0) return TID_OK;
@@ -335,15 +354,13 @@ void plan_search(const tid_index* idx, int64_t n_refs, int64_t B, int T, int* G_
   *qpj_out = qpj;
 }
 
-tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const uint8_t* rbase, const uint8_t* xbase,
-                               int64_t map_count, int64_t ref_map_base, const int32_t* colkey, int64_t n_refs, int64_t B,
+tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const uint8_t* rbase, int64_t map_count, int64_t ref_map_base, const int32_t* colkey, int64_t n_refs, int64_t B,
                                int32_t n,
                                int T, const int32_t* nvalid, uint32_t* counts, int64_t ldc, int64_t col0,
                                cudaStream_t s) {
   if (n_refs <= 0) return TID_OK;
-  CUtensorMap rmap, xmap;
+  CUtensorMap rmap;
   TRY(make_map(&rmap, rbase, map_count, idx->cfg.ref_kp, kBN));
-  TRY(make_xmap(&xmap, xbase, map_count, idx->cfg.ref_kp));
   MatchParams p{};
   p.mode = kModeSearch;
   p.qs = idx->ws_qs.as<uint8_t>();
@@ -368,7 +385,6 @@ tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const ui
   p.ldc = ldc;
   p.col0 = col0;
   p.nn_out = nullptr;
-  (void)idx->tune.exact_only;  // the scan is always exact (two-partition top-2)
   p.num2 = idx->cfg.ratio_num * idx->cfg.ratio_num;
   p.den2 = idx->cfg.ratio_den * idx->cfg.ratio_den;
   int grid = idx->tune.grid > 0 ? idx->tune.grid : idx->num_sms;
@@ -386,7 +402,7 @@ tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const ui
     ++idx->prof_used;
     CU(cudaEventRecord(e0, s));
   }
-  cudaError_t e = launch_match(p, qmap, rmap, &xmap, grid, s);
+  cudaError_t e = launch_match(p, qmap, rmap, true, grid, s);
   if (e != cudaSuccess) return fail(TID_ECUDA, "match kernel launch: %s", cudaGetErrorString(e));
   if (idx->prof) {
     CU(cudaEventRecord(e1, s));
@@ -396,82 +412,151 @@ tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const ui
   return TID_OK;
 }
 
-// Full local count matrix counts[B][R_local] for queries already resident in ws_q.
-tid_status run_counts(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, int32_t n, int64_t B,
-                      uint32_t* counts, cudaStream_t s) {
+// A run of consecutive local ids [first, first + cnt) inside one segment (offset `off`), inside one
+// count window.  Host-tier pieces are at most host_chunk references (one staging buffer).
+struct Piece {
+  const Segment* sg;
+  int64_t off, cnt, first;
+  int64_t win;  // window index
+};
+
+// The work list of one search pass: local ids [0, R) in id order, cut at window boundaries
+// (windows of W ids) and, in the host tier, into staging chunks.
+std::vector<Piece> plan_pieces(const tid_index* idx, int64_t W) {
+  std::vector<Piece> out;
+  const int64_t R = idx->n_hbm + idx->n_host;
+  for (int64_t w0 = 0, wi = 0; w0 < R; w0 += W, ++wi) {
+    const int64_t w1 = std::min(R, w0 + W);
+    for (const Segment& sg : idx->segs) {
+      const int64_t a = std::max(w0, sg.first), b = std::min(w1, sg.first + sg.count);
+      if (a >= b) continue;
+      const int64_t step = sg.on_host ? idx->host_chunk : (b - a);
+      for (int64_t x = a; x < b; x += step) out.push_back({&sg, x - sg.first, std::min(step, b - x), x, wi});
+    }
+  }
+  return out;
+}
+
+// One pass over every local reference for the B queries already on the device (dq): query prep
+// (a2), then per window of W reference ids the fused match kernel into counts[B][W] (ldc = W,
+// column = local id - window start), HBM segments in place (level 1) and host-tier chunks
+// streamed through two staging buffers on the copy stream (level 2, double buffered: chunk i+1
+// is copied while chunk i computes, across window boundaries too).  After each window's last
+// piece `on_window(w0, wlen)` runs on stream s (top-k of the window); the next window's
+// kernels are ordered after it on the same stream, so one counts buffer serves every window.
+template <class OnWindow>
+tid_status run_pass(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, int32_t n, int64_t B, int64_t W,
+                    uint32_t* counts, cudaStream_t s, OnWindow on_window) {
   const int T = static_cast<int>(ceil_div(n, kBM));
   const int64_t R = idx->n_hbm + idx->n_host;
   TRY(idx->ws_nq.ensure(static_cast<size_t>(B) * T * kBM * 4, "query norms"));
   TRY(idx->ws_qs.ensure(static_cast<size_t>(B) * n * kDim, "shifted queries"));
   launch_query_prep(dq, B, n, T, idx->ws_nq.as<int32_t>(), idx->ws_qs.as<uint8_t>(), s);
   count_kernel(idx);
-  CU(cudaMemsetAsync(counts, 0, static_cast<size_t>(B) * R * 4, s));
   CUtensorMap qmap;
   TRY(make_map(&qmap, idx->ws_qs.p, B, n, kBM));
-  // level 1: HBM-resident segments
-  for (const Segment& sg : idx->segs)
-    if (!sg.on_host && sg.count > 0)
-      TRY(launch_search_range(idx, qmap, sg.desc, sg.extra, sg.cap, 0, sg.colkey, sg.count, B, n, T, nvalid, counts, R, sg.first,
-                              s));
-  // level 2: pinned host tier, streamed through two HBM staging buffers on the copy stream
-  if (idx->n_host > 0) {
-    const int64_t chunk = idx->host_chunk;
-    const int64_t rb = idx->ref_bytes;
+  const std::vector<Piece> pieces = plan_pieces(idx, W);
+  std::vector<int64_t> next_host(pieces.size() + 1, -1);  // index of the next host piece after i
+  for (int64_t i = static_cast<int64_t>(pieces.size()) - 1, nh = -1; i >= 0; --i) {
+    next_host[i] = nh;
+    if (pieces[i].sg->on_host) nh = i;
+  }
+  int64_t first_host = -1;
+  for (size_t i = 0; i < pieces.size() && first_host < 0; ++i)
+    if (pieces[i].sg->on_host) first_host = static_cast<int64_t>(i);
+  const int64_t chunk = idx->host_chunk, rb = idx->ref_bytes;
+  std::vector<int> host_buf(pieces.size(), 0);
+  if (first_host >= 0) {
     for (int b = 0; b < 2; ++b) {
       TRY(idx->stage_desc[b].ensure(static_cast<size_t>(chunk * rb), "host-tier staging"));
       TRY(idx->stage_colkey[b].ensure(static_cast<size_t>(chunk) * idx->cpr * kColBytes, "staging keys"));
       TRY(idx->stage_kp[b].ensure(static_cast<size_t>(chunk) * 4, "staging kp"));
-      TRY(idx->stage_extra[b].ensure(static_cast<size_t>(chunk) * idx->cfg.ref_kp * kXDim, "staging norm digits"));
     }
     // the copy stream must not overwrite staging buffers still read by a previous call
     CU(cudaEventRecord(idx->ev_free[0], s));
     CU(cudaEventRecord(idx->ev_free[1], s));
-    struct Piece { const Segment* sg; int64_t off, cnt; };
-    std::vector<Piece> pieces;
-    for (const Segment& sg : idx->segs)
-      if (sg.on_host)
-        for (int64_t off = 0; off < sg.count; off += chunk) pieces.push_back({&sg, off, std::min(chunk, sg.count - off)});
-    auto issue_copy = [&](size_t i) -> tid_status {
-      const int b = static_cast<int>(i & 1);
-      const Piece& pc = pieces[i];
-      CU(cudaStreamWaitEvent(idx->copy_stream, idx->ev_free[b], 0));
-      CU(cudaMemcpyAsync(idx->stage_desc[b].p, pc.sg->desc + pc.off * rb, static_cast<size_t>(pc.cnt * rb),
-                         cudaMemcpyHostToDevice, idx->copy_stream));
-      CU(cudaMemcpyAsync(idx->stage_kp[b].p, pc.sg->kp.data() + pc.off, static_cast<size_t>(pc.cnt) * 4,
-                         cudaMemcpyHostToDevice, idx->copy_stream));
-      CU(cudaEventRecord(idx->ev_h2d[b], idx->copy_stream));
-      if (idx->prof) idx->stats.h2d_bytes += pc.cnt * rb + pc.cnt * 4;
-      return TID_OK;
-    };
-    if (!pieces.empty()) TRY(issue_copy(0));
-    for (size_t i = 0; i < pieces.size(); ++i) {
-      const int b = static_cast<int>(i & 1);
-      if (i + 1 < pieces.size()) TRY(issue_copy(i + 1));  // prefetch the next chunk while this one computes
+    for (size_t i = 0, h = 0; i < pieces.size(); ++i)
+      if (pieces[i].sg->on_host) host_buf[i] = static_cast<int>(h++ & 1);
+  }
+  auto issue_copy = [&](int64_t i) -> tid_status {
+    const int b = host_buf[i];
+    const Piece& pc = pieces[i];
+    CU(cudaStreamWaitEvent(idx->copy_stream, idx->ev_free[b], 0));
+    CU(cudaMemcpyAsync(idx->stage_desc[b].p, pc.sg->desc + pc.off * rb, static_cast<size_t>(pc.cnt * rb),
+                       cudaMemcpyHostToDevice, idx->copy_stream));
+    CU(cudaMemcpyAsync(idx->stage_kp[b].p, pc.sg->kp.data() + pc.off, static_cast<size_t>(pc.cnt) * 4,
+                       cudaMemcpyHostToDevice, idx->copy_stream));
+    CU(cudaEventRecord(idx->ev_h2d[b], idx->copy_stream));
+    if (idx->prof) idx->stats.h2d_bytes += pc.cnt * rb + pc.cnt * 4;
+    return TID_OK;
+  };
+  if (first_host >= 0) TRY(issue_copy(first_host));
+  int64_t cur_win = -1;
+  for (size_t i = 0; i < pieces.size(); ++i) {
+    const Piece& pc = pieces[i];
+    const int64_t w0 = pc.win * W;
+    if (pc.win != cur_win) {  // first piece of a window: clear its counts (kernels accumulate)
+      cur_win = pc.win;
+      CU(cudaMemsetAsync(counts, 0, static_cast<size_t>(B) * W * 4, s));
+    }
+    if (pc.sg->on_host) {
+      const int b = host_buf[i];
+      if (next_host[i] >= 0) TRY(issue_copy(next_host[i]));  // prefetch the next chunk while this one computes
       CU(cudaStreamWaitEvent(s, idx->ev_h2d[b], 0));
-      const Piece& pc = pieces[i];
       RefPrepParams rp{};
       rp.desc = idx->stage_desc[b].as<uint8_t>();
       rp.src = nullptr;
       rp.kp = idx->stage_kp[b].as<int32_t>();
       rp.colkey = idx->stage_colkey[b].as<int32_t>();
-      rp.extra = idx->stage_extra[b].as<uint8_t>();
+      rp.search = 1;
       rp.count = pc.cnt;
       rp.m = idx->cfg.ref_kp;
       rp.cpr = idx->cpr;
       launch_ref_prep(rp, s);
       count_kernel(idx);
-      TRY(launch_search_range(idx, qmap, idx->stage_desc[b].as<uint8_t>(), rp.extra, chunk, 0, rp.colkey, pc.cnt, B,
-                              n, T,
-                              nvalid, counts, R, pc.sg->first + pc.off, s));
+      TRY(launch_search_range(idx, qmap, idx->stage_desc[b].as<uint8_t>(), chunk, 0, rp.colkey, pc.cnt, B,
+                              n, T, nvalid, counts, W, pc.first - w0, s));
       CU(cudaEventRecord(idx->ev_free[b], s));
+    } else {
+      TRY(launch_search_range(idx, qmap, pc.sg->desc, pc.sg->cap, pc.off,
+                              pc.sg->colkey + pc.off * idx->cpr * kColInts, pc.cnt, B, n, T, nvalid, counts, W,
+                              pc.first - w0, s));
     }
+    if (i + 1 == pieces.size() || pieces[i + 1].win != pc.win) TRY(on_window(w0, std::min(W, R - w0)));
   }
   return TID_OK;
+}
+
+// References per count window of a search: the whole local set when its [B][R] u32 count matrix
+// fits the window budget (512 MiB, or the tuning's window_refs), else windows of that size
+// (workspace independent of R: a 10 M-reference host tier needs no 10 GB count matrix).
+int64_t window_refs(const tid_index* idx, int64_t B, int64_t R) {
+  int64_t W = idx->tune.window_refs > 0 ? idx->tune.window_refs
+                                        : std::max<int64_t>(4096, (int64_t(512) << 20) / (4 * std::max<int64_t>(B, 1)));
+  return std::max<int64_t>(1, std::min(W, R));
+}
+
+// Test hook: with TID_FAULT_ALLOC=N in the environment the N-th segment allocation from then on
+// fails with TID_ENOMEM (checks that tid_add_references is all-or-nothing).  Unset: no effect.
+bool injected_alloc_failure() {
+  static thread_local std::string armed;
+  static thread_local long left = 0;
+  const char* v = getenv("TID_FAULT_ALLOC");
+  if (!v || !*v) {
+    armed.clear();
+    return false;
+  }
+  if (armed != v) {
+    armed = v;
+    left = strtol(v, nullptr, 10);
+  }
+  return left > 0 && --left == 0;
 }
 
 // Allocate a segment of `cap` references in one tier (all-or-nothing).
 tid_status alloc_segment(tid_index* idx, bool on_host, int64_t cap, Segment* out) {
   const int64_t rb = idx->ref_bytes;
+  if (injected_alloc_failure()) return fail(TID_ENOMEM, "injected allocation failure (TID_FAULT_ALLOC)");
   Segment sg;
   sg.on_host = on_host;
   sg.cap = cap;
@@ -485,9 +570,7 @@ tid_status alloc_segment(tid_index* idx, bool on_host, int64_t cap, Segment* out
   } else {
     cudaError_t e1 = cudaMalloc(&sg.desc, static_cast<size_t>(cap * rb));
     cudaError_t e2 = e1 == cudaSuccess ? cudaMalloc(&sg.colkey, static_cast<size_t>(cap) * idx->cpr * kColBytes) : e1;
-    cudaError_t e3 =
-        e2 == cudaSuccess ? cudaMalloc(&sg.extra, static_cast<size_t>(cap) * idx->cfg.ref_kp * kXDim) : e2;
-    if (e1 != cudaSuccess || e2 != cudaSuccess || e3 != cudaSuccess) {
+    if (e1 != cudaSuccess || e2 != cudaSuccess) {
       cudaGetLastError();
       if (sg.desc) cudaFree(sg.desc);
       if (sg.colkey) cudaFree(sg.colkey);
@@ -506,12 +589,10 @@ void free_segment(tid_index* idx, Segment& sg) {
   } else {
     if (sg.desc) cudaFree(sg.desc);
     if (sg.colkey) cudaFree(sg.colkey);
-    if (sg.extra) cudaFree(sg.extra);
     idx->hbm_alloc -= sg.cap * idx->hbm_ref_bytes;
   }
   sg.desc = nullptr;
   sg.colkey = nullptr;
-  sg.extra = nullptr;
 }
 
 // Ingest `take` references (host or device `src`, kp_host per reference) into HBM segment sg at
@@ -526,7 +607,7 @@ tid_status ingest_hbm(tid_index* idx, Segment& sg, int64_t pos, const uint8_t* s
   rp.cpr = idx->cpr;
   rp.count = take;
   rp.colkey = sg.colkey + pos * idx->cpr * kColInts;
-  rp.extra = sg.extra + pos * idx->cfg.ref_kp * kXDim;
+  rp.search = 1;
   if (src_dev) {
     rp.src = src;
   } else {
@@ -610,7 +691,6 @@ tid_status check_search_args(tid_index* idx, const uint8_t* queries, int32_t n, 
   if (n < 1 || n > idx->cfg.query_kp_max) return fail(TID_EINVAL, "n=%d outside 1..query_kp_max=%d", n, idx->cfg.query_kp_max);
   if (B < 1) return fail(TID_EINVAL, "B=%lld must be >= 1", static_cast<long long>(B));
   if (B > (1LL << 31) / 2) return fail(TID_EINVAL, "B too large");
-  if (idx->n_hbm + idx->n_host == 0) return fail(TID_ESTATE, "index holds no references");
   return TID_OK;
 }
 
@@ -662,7 +742,7 @@ tid_status tid_index_create(const tid_config* cfg, tid_index** out) {
   idx->num_sms = prop.multiProcessorCount;
   idx->cpr = static_cast<int>(ceil_div(cfg->ref_kp, kBN));
   idx->ref_bytes = static_cast<int64_t>(cfg->ref_kp) * kDim;
-  idx->hbm_ref_bytes = idx->ref_bytes + static_cast<int64_t>(cfg->ref_kp) * kXDim + static_cast<int64_t>(idx->cpr) * kColBytes;
+  idx->hbm_ref_bytes = idx->ref_bytes + static_cast<int64_t>(idx->cpr) * kColBytes;
   size_t free_b = 0, total_b = 0;
   cudaMemGetInfo(&free_b, &total_b);
   const uint64_t reserve = 8ull << 30;
@@ -674,6 +754,7 @@ tid_status tid_index_create(const tid_config* cfg, tid_index** out) {
   idx->host_budget = cfg->host_budget_bytes;
   idx->host_chunk = 16384;
   cudaError_t e = cudaStreamCreateWithFlags(&idx->copy_stream, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&idx->ev_last, cudaEventDisableTiming);
   for (int b = 0; b < 2 && e == cudaSuccess; ++b) {
     e = cudaEventCreateWithFlags(&idx->ev_h2d[b], cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&idx->ev_free[b], cudaEventDisableTiming);
@@ -709,8 +790,7 @@ tid_status tid_index_destroy(tid_index* idx) {
   DevBuf* bufs[] = {&idx->ws_q, &idx->ws_nq, &idx->ws_nvalid, &idx->ws_counts, &idx->ws_cand, &idx->ws_keys,
                     &idx->ws_gather, &idx->ws_ids, &idx->ws_cnts, &idx->ws_r, &idx->ws_colkey, &idx->ws_nn,
                     &idx->ws_kp, &idx->ws_mr, &idx->stage_desc[0], &idx->stage_desc[1], &idx->stage_colkey[0],
-                    &idx->stage_colkey[1], &idx->stage_kp[0], &idx->stage_kp[1], &idx->stage_extra[0],
-                    &idx->stage_extra[1], &idx->ws_qs, &idx->ws_f16q, &idx->ws_f16r, &idx->ws_f16nq,
+                    &idx->stage_colkey[1], &idx->stage_kp[0], &idx->stage_kp[1], &idx->ws_qs, &idx->ws_f16q, &idx->ws_f16r, &idx->ws_f16nq,
                     &idx->ws_f16nr, &idx->ws_f16in};
   for (DevBuf* b : bufs) b->release();
   for (auto& pr : idx->prof_ev) { cudaEventDestroy(pr.first); cudaEventDestroy(pr.second); }
@@ -719,6 +799,9 @@ tid_status tid_index_destroy(tid_index* idx) {
     if (idx->ev_free[b]) cudaEventDestroy(idx->ev_free[b]);
   }
   if (idx->copy_stream) cudaStreamDestroy(idx->copy_stream);
+  if (idx->ev_last) cudaEventDestroy(idx->ev_last);
+  if (idx->h_rtot) cudaFreeHost(idx->h_rtot);
+  idx->ws_rtot.release();
   if (idx->comm) nccl().CommDestroy(idx->comm);
   delete idx;
   return TID_OK;
@@ -730,6 +813,7 @@ tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t
   if (count < 0) return fail(TID_EINVAL, "count < 0");
   if (count > 0 && !desc) return fail(TID_EINVAL, "null descriptors");
   TRY(set_device(idx));
+  CallGuard guard(idx, nullptr);
   const int64_t first = idx->n_hbm + idx->n_host;
   if (first_local_id) *first_local_id = first;
   if (count == 0) return TID_OK;
@@ -765,6 +849,36 @@ tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t
                   static_cast<long long>(count), static_cast<long long>(hbm_room),
                   static_cast<long long>(host_cap - idx->n_host));
   }
+  // ---- transaction: from here on a failure rolls the index back to its state before the call
+  // (segments created by this call freed, the tail segment's count restored, counters restored),
+  // so TID_ENOMEM / TID_ECUDA add nothing.  (FIFO swap-outs above are not undone: they move
+  // whole batches between tiers and change neither ids nor search results.)
+  const size_t segs0 = idx->segs.size();
+  const int64_t tail_count0 = segs0 ? idx->segs.back().count : 0;
+  const int64_t n_hbm0 = idx->n_hbm, n_host0 = idx->n_host;
+  auto rollback = [&](tid_status st) -> tid_status {
+    const std::string msg = g_err;
+    cudaStreamSynchronize(nullptr);
+    cudaGetLastError();
+    while (idx->segs.size() > segs0) {
+      free_segment(idx, idx->segs.back());
+      idx->segs.pop_back();
+    }
+    if (segs0) {
+      Segment& t = idx->segs.back();
+      t.count = tail_count0;
+      t.kp.resize(static_cast<size_t>(tail_count0));
+    }
+    idx->n_hbm = n_hbm0;
+    idx->n_host = n_host0;
+    g_err = msg;
+    return st;
+  };
+#define TRY_TX(x)                            \
+  do {                                       \
+    tid_status s__ = (x);                    \
+    if (s__ != TID_OK) return rollback(s__); \
+  } while (0)
   // ---- HBM part (append to the last HBM segment if it is the id-tail and has room, else a new one)
   int64_t done = 0;
   while (done < to_hbm) {
@@ -776,13 +890,13 @@ tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t
                                                : std::max<int64_t>(to_hbm - done, std::min<int64_t>(idx->n_hbm, room));
       cap = std::min(cap, room);
       Segment ns;
-      TRY(alloc_segment(idx, false, cap, &ns));
+      TRY_TX(alloc_segment(idx, false, cap, &ns));
       ns.first = first + done;
       idx->segs.push_back(std::move(ns));
       sg = &idx->segs.back();
     }
     const int64_t take = std::min(to_hbm - done, sg->cap - sg->count);
-    TRY(ingest_hbm(idx, *sg, sg->count, desc + done * rb, dev_in, kp.data() + done, take));
+    TRY_TX(ingest_hbm(idx, *sg, sg->count, desc + done * rb, dev_in, kp.data() + done, take));
     sg->kp.insert(sg->kp.end(), kp.begin() + done, kp.begin() + done + take);
     sg->count += take;
     idx->n_hbm += take;
@@ -797,19 +911,21 @@ tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t
       int64_t cap = std::max<int64_t>(to_host - hdone, std::min<int64_t>(idx->n_host, room));
       cap = std::min(cap, room);
       Segment ns;
-      TRY(alloc_segment(idx, true, cap, &ns));
+      TRY_TX(alloc_segment(idx, true, cap, &ns));
       ns.first = first + to_hbm + hdone;
       idx->segs.push_back(std::move(ns));
       sg = &idx->segs.back();
     }
     const int64_t take = std::min(to_host - hdone, sg->cap - sg->count);
-    CU(cudaMemcpy(sg->desc + sg->count * rb, desc + (to_hbm + hdone) * rb, static_cast<size_t>(take * rb),
-                  cudaMemcpyDefault));
+    if (cudaMemcpy(sg->desc + sg->count * rb, desc + (to_hbm + hdone) * rb, static_cast<size_t>(take * rb),
+                   cudaMemcpyDefault) != cudaSuccess)
+      return rollback(fail(TID_ECUDA, "host-tier copy: %s", cudaGetErrorString(cudaGetLastError())));
     sg->kp.insert(sg->kp.end(), kp.begin() + to_hbm + hdone, kp.begin() + to_hbm + hdone + take);
     sg->count += take;
     idx->n_host += take;
     hdone += take;
   }
+#undef TRY_TX
   idx->dead.resize(static_cast<size_t>(first + count), 0);
   idx->dead_dirty = true;
   return TID_OK;
@@ -820,6 +936,8 @@ tid_status tid_host_tier_map(tid_index* idx, int64_t count, uint8_t** desc_out, 
   if (count < 1 || !desc_out) return fail(TID_EINVAL, "count < 1 or null desc_out");
   if (idx->cfg.cache_policy == 1) return fail(TID_ESTATE, "FIFO policy: the host tier holds evicted batches only");
   TRY(set_device(idx));
+  CallGuard guard(idx, nullptr);
+  CU(cudaStreamSynchronize(nullptr));  // a search may still be streaming the tier
   const int64_t rb = idx->ref_bytes;
   const int64_t host_cap = static_cast<int64_t>(idx->host_budget / rb);
   if (count > host_cap - idx->n_host)
@@ -845,6 +963,7 @@ tid_status tid_delete_references(tid_index* idx, const int64_t* local_ids, int64
   if (!idx) return fail(TID_EINVAL, "null index");
   if (count < 0 || (count > 0 && !local_ids)) return fail(TID_EINVAL, "bad ids");
   TRY(set_device(idx));
+  CallGuard guard(idx, nullptr);
   std::vector<int64_t> ids(static_cast<size_t>(count));
   if (count) CU(cudaMemcpy(ids.data(), local_ids, static_cast<size_t>(count) * 8, cudaMemcpyDefault));
   const int64_t R = idx->n_hbm + idx->n_host;
@@ -863,7 +982,7 @@ tid_status tid_delete_references(tid_index* idx, const int64_t* local_ids, int64
       CU(cudaMemcpy(idx->ws_kp.p, &zero, 4, cudaMemcpyHostToDevice));
       rp.kp = idx->ws_kp.as<int32_t>();
       rp.colkey = sg->colkey + off * idx->cpr * kColInts;
-      rp.extra = sg->extra + off * idx->cfg.ref_kp * kXDim;
+      rp.search = 1;
       rp.count = 1;
       rp.m = idx->cfg.ref_kp;
       rp.cpr = idx->cpr;
@@ -882,6 +1001,7 @@ tid_status tid_update_references(tid_index* idx, const int64_t* local_ids, const
   if (!idx) return fail(TID_EINVAL, "null index");
   if (count < 0 || (count > 0 && (!local_ids || !desc))) return fail(TID_EINVAL, "bad arguments");
   TRY(set_device(idx));
+  CallGuard guard(idx, nullptr);
   std::vector<int64_t> ids(static_cast<size_t>(count));
   if (count) CU(cudaMemcpy(ids.data(), local_ids, static_cast<size_t>(count) * 8, cudaMemcpyDefault));
   std::vector<int32_t> kp(static_cast<size_t>(count), idx->cfg.ref_kp);
@@ -914,6 +1034,7 @@ tid_status tid_index_save(const tid_index* cidx, const char* path) {
   tid_index* idx = const_cast<tid_index*>(cidx);
   if (!idx || !path) return fail(TID_EINVAL, "null argument");
   TRY(set_device(idx));
+  CU(cudaEventSynchronize(idx->ev_last));
   FILE* f = fopen(path, "wb");
   if (!f) return fail(TID_EINVAL, "cannot open %s for writing", path);
   const int64_t R = idx->n_hbm + idx->n_host, rb = idx->ref_bytes;
@@ -990,19 +1111,22 @@ tid_status tid_search_counts(tid_index* idx, const uint8_t* queries, const int32
                              uint32_t* counts_out, void* stream) {
   TRY(check_search_args(idx, queries, n, B));
   if (!counts_out) return fail(TID_EINVAL, "null counts_out");
+  const int64_t R = idx->n_hbm + idx->n_host;
+  if (R == 0) return fail(TID_ESTATE, "index holds no references");
   TRY(set_device(idx));
   cudaStream_t s = static_cast<cudaStream_t>(stream);
+  CallGuard guard(idx, s);
   const uint8_t* dq;
   const int32_t* dnv;
   TRY(stage_queries(idx, queries, n_q, n, B, &dq, &dnv, s));
-  const int64_t R = idx->n_hbm + idx->n_host;
   const bool dev_out = is_device_ptr(counts_out);
   uint32_t* counts = counts_out;
   if (!dev_out) {
     TRY(idx->ws_counts.ensure(static_cast<size_t>(B) * R * 4, "count matrix"));
     counts = idx->ws_counts.as<uint32_t>();
   }
-  TRY(run_counts(idx, dq, dnv, n, B, counts, s));
+  // one window = every local reference: the output IS the full count matrix
+  TRY(run_pass(idx, dq, dnv, n, B, R, counts, s, [](int64_t, int64_t) { return TID_OK; }));
   bool host_out = false;
   if (!dev_out) TRY(copy_out(idx, counts_out, counts, static_cast<size_t>(B) * R * 4, s, &host_out));
   if (host_out) CU(cudaStreamSynchronize(s));
@@ -1010,53 +1134,117 @@ tid_status tid_search_counts(tid_index* idx, const uint8_t* queries, const int32
   return TID_OK;
 }
 
+namespace {
+// Collective: the total reference count over all ranks (one NCCL all-reduce of an int64).
+tid_status total_references(tid_index* idx, cudaStream_t s, int64_t* out) {
+  const int64_t R = idx->n_hbm + idx->n_host;
+  if (idx->comm == nullptr) {
+    *out = R;
+    return TID_OK;
+  }
+  if (!idx->h_rtot) {
+    if (cudaHostAlloc(reinterpret_cast<void**>(&idx->h_rtot), 8, cudaHostAllocPortable) != cudaSuccess) {
+      cudaGetLastError();
+      idx->h_rtot = nullptr;
+      return fail(TID_ENOMEM, "pinned scalar allocation failed");
+    }
+  }
+  TRY(idx->ws_rtot.ensure(8, "reference total"));
+  *idx->h_rtot = R;
+  CU(cudaMemcpyAsync(idx->ws_rtot.p, idx->h_rtot, 8, cudaMemcpyHostToDevice, s));
+  NC(nccl().AllReduce(idx->ws_rtot.p, idx->ws_rtot.p, 1, ncclInt64, ncclSum, idx->comm, s));
+  CU(cudaMemcpyAsync(idx->h_rtot, idx->ws_rtot.p, 8, cudaMemcpyDeviceToHost, s));
+  CU(cudaStreamSynchronize(s));
+  *out = *idx->h_rtot;
+  return TID_OK;
+}
+}  // namespace
+
 tid_status tid_search(tid_index* idx, const uint8_t* queries, const int32_t* n_q, int32_t n, int64_t B, int32_t k,
                       int64_t* ref_ids_out, int32_t* match_counts_out, void* stream) {
   TRY(check_search_args(idx, queries, n, B));
   if (!ref_ids_out || !match_counts_out) return fail(TID_EINVAL, "null outputs");
   if (k < 1 || k > 64) return fail(TID_EINVAL, "k=%d outside 1..64", k);
-  const int64_t R = idx->n_hbm + idx->n_host;
-  if (idx->comm == nullptr && k > R)
-    return fail(TID_EINVAL, "k=%d exceeds the number of references (%lld)", k, static_cast<long long>(R));
   TRY(set_device(idx));
   cudaStream_t s = static_cast<cudaStream_t>(stream);
-  const uint8_t* dq;
-  const int32_t* dnv;
+  CallGuard guard(idx, s);
+  const int64_t R = idx->n_hbm + idx->n_host;
+  // k <= total references, decided identically on every rank (collective count with NCCL), so a
+  // rank never leaves the others waiting in the all-gather below
+  int64_t R_total = 0;
+  TRY(total_references(idx, s, &R_total));
+  if (R_total == 0) return fail(TID_ESTATE, "index holds no references");
+  if (k > R_total)
+    return fail(TID_EINVAL, "k=%d exceeds the number of references (%lld)", k, static_cast<long long>(R_total));
+  const uint8_t* dq = nullptr;
+  const int32_t* dnv = nullptr;
   TRY(stage_queries(idx, queries, n_q, n, B, &dq, &dnv, s));
-  TRY(idx->ws_counts.ensure(static_cast<size_t>(B) * R * 4, "count matrix"));
-  uint32_t* counts = idx->ws_counts.as<uint32_t>();
-  TRY(run_counts(idx, dq, dnv, n, B, counts, s));
-  // a6: per-(query, segment) top-k, then merge the segments
-  int64_t segs = std::max<int64_t>(1, std::min<int64_t>(ceil_div(2LL * idx->num_sms, B), ceil_div(R, 4096)));
-  segs = std::min<int64_t>(segs, 1024);
-  TRY(idx->ws_cand.ensure(static_cast<size_t>(B) * segs * k * 8, "top-k candidates"));
   TRY(sync_dead(idx, s));
   TRY(idx->ws_ids.ensure(static_cast<size_t>(B) * k * 8, "ids"));
   TRY(idx->ws_cnts.ensure(static_cast<size_t>(B) * k * 4, "counts"));
   const bool dev_ids = is_device_ptr(ref_ids_out), dev_cnt = is_device_ptr(match_counts_out);
   int64_t* ids = dev_ids ? ref_ids_out : idx->ws_ids.as<int64_t>();
   int32_t* cnts = dev_cnt ? match_counts_out : idx->ws_cnts.as<int32_t>();
-  // one segment on one GPU: the top-k kernel writes the final ranking (no merge launch)
-  const bool direct = idx->comm == nullptr && segs == 1;
-  launch_topk(counts, B, R, R, idx->cfg.id_base, k, static_cast<int32_t>(segs),
-              idx->any_dead ? idx->dead_dev.as<uint8_t>() : nullptr, idx->ws_cand.as<uint64_t>(), s,
-              direct ? ids : nullptr, direct ? cnts : nullptr);
-  count_kernel(idx);
-  if (idx->comm == nullptr) {
-    if (!direct) {
-      launch_merge(idx->ws_cand.as<uint64_t>(), static_cast<int32_t>(segs), B, k, segs * k, k, nullptr, ids, cnts, s);
-      count_kernel(idx);
-    }
+  const bool collective = idx->comm != nullptr;
+  if (collective) TRY(idx->ws_keys.ensure(static_cast<size_t>(B) * k * 8, "local keys"));
+  uint64_t* local_keys = collective ? idx->ws_keys.as<uint64_t>() : nullptr;
+  if (R > 0) {
+    // a6: per window, per-(query, segment) top-k of the window's counts, then merge.  One window:
+    // merge the segments straight into the result (one segment, no comm: the top-k kernel
+    // writes it).  Several windows: the running top-k is list 0 of every query's candidate
+    // lists, merged in place with the window's segments after each window.
+    const int64_t W = window_refs(idx, B, R);
+    const int64_t nwin = ceil_div(R, W);
+    auto segs_for = [&](int64_t len) {
+      int64_t sg = std::max<int64_t>(1, std::min<int64_t>(ceil_div(2LL * idx->num_sms, B), ceil_div(len, 4096)));
+      return static_cast<int32_t>(std::min<int64_t>(sg, 1024));
+    };
+    const int32_t lists = (nwin > 1 ? 1 : 0) + segs_for(W);
+    TRY(idx->ws_cand.ensure(static_cast<size_t>(B) * lists * k * 8, "top-k candidates"));
+    TRY(idx->ws_counts.ensure(static_cast<size_t>(B) * W * 4, "count window"));
+    uint64_t* cand = idx->ws_cand.as<uint64_t>();
+    if (nwin > 1) CU(cudaMemsetAsync(cand, 0, static_cast<size_t>(B) * lists * k * 8, s));  // empty running lists
+    const uint8_t* dead = idx->any_dead ? idx->dead_dev.as<uint8_t>() : nullptr;
+    uint32_t* counts = idx->ws_counts.as<uint32_t>();
+    auto on_window = [&](int64_t w0, int64_t wlen) -> tid_status {
+      const int32_t segs = segs_for(wlen);
+      const bool last = w0 + wlen >= R;
+      if (nwin == 1) {
+        const bool direct = !collective && segs == 1;
+        launch_topk(counts, B, wlen, W, idx->cfg.id_base + w0, k, segs, dead, cand, lists, 0, s,
+                    direct ? ids : nullptr, direct ? cnts : nullptr);
+        count_kernel(idx);
+        if (!direct) {
+          launch_merge(cand, segs, B, k, static_cast<int64_t>(lists) * k, k, local_keys, collective ? nullptr : ids,
+                       collective ? nullptr : cnts, s);
+          count_kernel(idx);
+        }
+      } else {
+        launch_topk(counts, B, wlen, W, idx->cfg.id_base + w0, k, segs, dead ? dead + w0 : nullptr, cand, lists, 1, s);
+        // running top-k (list 0) + this window's segments -> list 0, or the result after the last window
+        if (!last) {
+          launch_merge(cand, 1 + segs, B, k, static_cast<int64_t>(lists) * k, k, cand, nullptr, nullptr, s,
+                       static_cast<int64_t>(lists) * k);
+        } else {
+          launch_merge(cand, 1 + segs, B, k, static_cast<int64_t>(lists) * k, k, local_keys, collective ? nullptr : ids,
+                       collective ? nullptr : cnts, s);
+        }
+        count_kernel(idx, 2);
+      }
+      return TID_OK;
+    };
+    TRY(run_pass(idx, dq, dnv, n, B, W, counts, s, on_window));
   } else {
+    // empty shard (collective only): contribute empty candidate lists to the all-gather
+    CU(cudaMemsetAsync(local_keys, 0, static_cast<size_t>(B) * k * 8, s));
+  }
+  if (collective) {
     // a9: local top-k -> NCCL all-gather over NVLink -> identical merge on every rank
     const int G = idx->cfg.world_size;
-    TRY(idx->ws_keys.ensure(static_cast<size_t>(B) * k * 8, "local keys"));
     TRY(idx->ws_gather.ensure(static_cast<size_t>(G) * B * k * 8, "gathered keys"));
-    launch_merge(idx->ws_cand.as<uint64_t>(), static_cast<int32_t>(segs), B, k, segs * k, k,
-                 idx->ws_keys.as<uint64_t>(), nullptr, nullptr, s);
-    NC(nccl().AllGather(idx->ws_keys.p, idx->ws_gather.p, static_cast<size_t>(B) * k, ncclUint64, idx->comm, s));
+    NC(nccl().AllGather(local_keys, idx->ws_gather.p, static_cast<size_t>(B) * k, ncclUint64, idx->comm, s));
     launch_merge(idx->ws_gather.as<uint64_t>(), G, B, k, k, B * k, nullptr, ids, cnts, s);
-    count_kernel(idx, 2);
+    count_kernel(idx);
   }
   CU(cudaGetLastError());
   bool host_out = false;
@@ -1075,6 +1263,7 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
   if (P < 1 || P > (1LL << 31) - 1) return fail(TID_EINVAL, "P=%lld invalid", static_cast<long long>(P));
   TRY(set_device(idx));
   cudaStream_t s = static_cast<cudaStream_t>(stream);
+  CallGuard guard(idx, s);
   const int cpr = static_cast<int>(ceil_div(m, kBN));
   const int T = static_cast<int>(ceil_div(n, kBM));
   const uint8_t* dq;
@@ -1135,6 +1324,7 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
   TRY(make_map(&rmap, dr, P, m, kBN));
   MatchParams p{};
   p.mode = kModeVerify;
+  p.m = m;  // stored rows per reference: the last chunk's all-padding pieces are skipped
   p.n_jobs = static_cast<int32_t>(P);
   p.refs_per_job = 1;
   p.cpr = cpr;
@@ -1169,7 +1359,7 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
     ++idx->prof_used;
     CU(cudaEventRecord(e0, s));
   }
-  cudaError_t e = launch_match(p, qmap, rmap, nullptr, grid, s);
+  cudaError_t e = launch_match(p, qmap, rmap, false, grid, s);
   if (e != cudaSuccess) return fail(TID_ECUDA, "match kernel launch: %s", cudaGetErrorString(e));
   if (idx->prof) {
     CU(cudaEventRecord(e1, s));
@@ -1190,6 +1380,7 @@ tid_status tid_merge_topk(tid_index* idx, const int64_t* ids_in, const int32_t* 
   if (G < 1 || B < 1 || k < 1 || k > 64) return fail(TID_EINVAL, "bad G/B/k");
   TRY(set_device(idx));
   cudaStream_t s = static_cast<cudaStream_t>(stream);
+  CallGuard guard(idx, s);
   const int64_t tot = static_cast<int64_t>(G) * B * k;
   TRY(idx->ws_ids.ensure(static_cast<size_t>(tot) * 8, "merge ids"));
   TRY(idx->ws_cnts.ensure(static_cast<size_t>(tot) * 4, "merge counts"));
@@ -1219,6 +1410,7 @@ tid_status tid_f16_prepare(tid_index* idx, const uint8_t* sift, int64_t rows, in
   if (rows == 0) return TID_OK;
   TRY(set_device(idx));
   cudaStream_t s = static_cast<cudaStream_t>(stream);
+  CallGuard guard(idx, s);
   const size_t in_b = static_cast<size_t>(rows) * kDim, out_b = in_b * 2;
   const uint8_t* din = sift;
   // the kernel moves 16-byte words: unaligned device buffers are staged through the workspace too
@@ -1253,6 +1445,7 @@ tid_status tid_f16_search_counts(tid_index* idx, const uint16_t* q, int32_t n, i
   if (B > (1LL << 30) || R > (1LL << 31) - 1) return fail(TID_EINVAL, "B or R too large");
   TRY(set_device(idx));
   cudaStream_t s = static_cast<cudaStream_t>(stream);
+  CallGuard guard(idx, s);
   const int T = static_cast<int>(ceil_div(n, kBM));
   const size_t qb = static_cast<size_t>(B) * n * kDim * 2, rb = static_cast<size_t>(R) * m * kDim * 2;
   const uint16_t* dq = q;
@@ -1306,7 +1499,12 @@ tid_status tid_get_info(const tid_index* idx, tid_info* out) {
   out->hbm_bytes = idx->hbm_alloc;
   out->host_bytes = idx->host_alloc;
   out->num_sms = idx->num_sms;
+  out->hbm_capacity_references = static_cast<int64_t>(idx->hbm_budget / idx->ref_bytes);
+  out->host_capacity_references = static_cast<int64_t>(idx->host_budget / idx->ref_bytes);
+  out->hbm_bytes_per_reference = idx->hbm_ref_bytes;
   out->world_size = idx->cfg.world_size;
+  int nranks = 0;  // with a communicator: the rank count NCCL itself reports
+  if (idx->comm && nccl().CommCount && nccl().CommCount(idx->comm, &nranks) == ncclSuccess) out->world_size = nranks;
   return TID_OK;
 }
 
@@ -1338,6 +1536,7 @@ tid_status tid_set_tuning(tid_index* idx, const tid_tuning* t) {
   if (t->refs_per_job < 0 || t->refs_per_job > kMaxSlots) return fail(TID_EINVAL, "refs_per_job outside 0..4");
   if (t->grid < 0) return fail(TID_EINVAL, "grid < 0");
   if (t->host_chunk_refs < 0) return fail(TID_EINVAL, "host_chunk_refs < 0");
+  if (t->window_refs < 0) return fail(TID_EINVAL, "window_refs < 0");
   idx->tune = *t;
   if (t->host_chunk_refs > 0) idx->host_chunk = t->host_chunk_refs;
   return TID_OK;

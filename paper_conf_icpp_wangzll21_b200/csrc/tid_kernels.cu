@@ -289,7 +289,8 @@ struct SmemPlan {
   static constexpr uint32_t kTEmpty = kTFull + 8 * kTmemBufs;
   static constexpr uint32_t kTQFull = kTEmpty + 8 * kTmemBufs;           // query tiles staged in TMEM (search)
   static constexpr uint32_t kTQEmpty = kTQFull + 8 * kTQ;
-  static constexpr uint32_t kAxFull = kTQEmpty + 8 * kTQ;
+  static constexpr uint32_t kXReady = kTQEmpty + 8 * kTQ;                // norm digits expanded on chip (search)
+  static constexpr uint32_t kAxFull = kXReady + 8 * kMaxSlots;
   static constexpr uint32_t kTmemPtr = kAxFull + 8;
   static constexpr uint32_t kEnd = kTmemPtr + 16;
   static constexpr uint32_t kAlloc = kEnd + 1024;                          // + alignment slack
@@ -448,6 +449,19 @@ __device__ __forceinline__ void exact_row_global(const MatchParams& p, int qi, i
   d2 = a2;
 }
 
+// Pieces of kPiece columns in a reference's last 256-column chunk that can hold real keypoints:
+// columns >= m are padding for every reference (m = 384: the second chunk is half padding), so
+// those pieces are neither computed nor scanned (a chunk with fewer than 4 pieces leaves the
+// static buffer / phase schedule with odd use counts: use_parity() tracks the flips).
+__device__ __forceinline__ int piece_count_last(int m, int cpr) {
+  return (m - (cpr - 1) * kBN + kPiece - 1) / kPiece;
+}
+// Phase flips of the two TMEM buffers after a chunk of np pieces (buffer pp & 1): buffer 0 is used
+// ceil(np / 2) times, buffer 1 floor(np / 2) times; bit b set when that count is odd.
+__device__ __forceinline__ uint32_t use_parity(int np) {
+  return (((np + 1) >> 1) & 1u) | (((np >> 1) & 1u) << 1);
+}
+
 // ------------------------------------------------------------------ fused match kernel
 // One persistent CTA per SM.  A job = (up to kNG = 3 references resident in SMEM, fewer chunks'
 // worth for m > 256) x (range of query tiles streamed through a kQStages ring; search: copied
@@ -462,7 +476,7 @@ __device__ __forceinline__ void exact_row_global(const MatchParams& p, int qi, i
 template <bool kFold>
 __global__ void __launch_bounds__(kNumThreads, 1)
     match_kernel(const __grid_constant__ CUtensorMap qmap, const __grid_constant__ CUtensorMap rmap,
-                 const __grid_constant__ CUtensorMap xmap, const MatchParams p) {
+                 const MatchParams p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const uint32_t sbase = smem_u32(smem);
@@ -477,6 +491,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
   auto tempty = [&](int i) { return sbase + SmemPlan::kTEmpty + 8 * i; };
   auto tqfull = [&](int i) { return sbase + SmemPlan::kTQFull + 8 * i; };
   auto tqempty = [&](int i) { return sbase + SmemPlan::kTQEmpty + 8 * i; };
+  auto xready = [&](int i) { return sbase + SmemPlan::kXReady + 8 * i; };
   const uint32_t axfull = sbase + SmemPlan::kAxFull;
   uint32_t* tmem_ptr_smem = reinterpret_cast<uint32_t*>(smem + SmemPlan::kTmemPtr);
 
@@ -488,14 +503,17 @@ __global__ void __launch_bounds__(kNumThreads, 1)
   if (threadIdx.x == 0) {
     prefetch_tmap(&qmap);
     prefetch_tmap(&rmap);
-    if (kFold) prefetch_tmap(&xmap);
     // query stages: search copies each tile to TMEM (freed by that copy); verify feeds the MMAs from
     // shared memory (freed by the kNG MMA warps' commits)
     for (int i = 0; i < kQStages; ++i) { mbar_init(qfull(i), 1); mbar_init(qempty(i), kFold ? 1 : kNG); }
     for (int i = 0; i < kTQ; ++i) { mbar_init(tqfull(i), 1); mbar_init(tqempty(i), kNG); }
     mbar_init(axfull, 1);
     // reference slots: MMA operands + column keys read by every epilogue warp
-    for (int i = 0; i < kMaxSlots; ++i) { mbar_init(rfull(i), 1); mbar_init(rempty(i), kNG + kEpiWarps); }
+    for (int i = 0; i < kMaxSlots; ++i) {
+      mbar_init(rfull(i), 1);
+      mbar_init(rempty(i), kNG + kEpiWarps);
+      mbar_init(xready(i), kEpiWarps);  // search: every epilogue warp wrote its share of the slot's digits
+    }
     for (int i = 0; i < kTmemBufs; ++i) { mbar_init(tfull(i), 1); mbar_init(tempty(i), 4); }
     fence_barrier_init();
   }
@@ -526,14 +544,11 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         const int nslots = J.nr * cpr;
         for (int sl = 0; sl < nslots; ++sl) {
           PROF_B(); mbar_wait_sleep(rempty(sl), (slot_par >> sl & 1u) ^ 1); PROF_E(0);
-          mbar_expect_tx(rfull(sl), kRTileBytes + kColBytes + (kFold ? kXTileBytes : 0));
+          mbar_expect_tx(rfull(sl), kRTileBytes + kColBytes);
           const int s = sl / cpr, c = sl % cpr;
           const int64_t ref = J.ref_first + s;
           tma_load_3d(sbase + SmemPlan::kR + sl * kRTileBytes, &rmap, rfull(sl), 0, c * kBN,
                       static_cast<int>(p.ref_map_base + ref));
-          if (kFold)
-            tma_load_3d(sbase + SmemPlan::kX + sl * kXTileBytes, &xmap, rfull(sl), 0, c * kBN,
-                        static_cast<int>(p.ref_map_base + ref));
           bulk_load(sbase + SmemPlan::kCol + sl * kColBytes, p.colkey + (ref * cpr + c) * kColInts, kColBytes,
                     rfull(sl));
           slot_par ^= 1u << sl;
@@ -579,6 +594,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     // 64-column buffers (whole warp, one elected lane).  Every warp commits the release of every
     // query tile (waiting for tiles it never used, so the stage phases stay in order).
     const int mw = warp - kFirstMmaWarp;
+    const int np_last = piece_count_last(p.m, cpr);
+    uint32_t ph_t = 0;  // bit b: phase flip of this group's TMEM buffer b (chunks with an odd use count)
     uint32_t qctr = 0;
     if (kFold) mbar_wait(axfull, 0);  // constant norm-term operand in TMEM
     uint32_t slot_par = 0;  // bit sl = phase parity of reference slot sl
@@ -604,14 +621,18 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           for (int c = 0; c < cpr; ++c) {
             const int sl = s * cpr + c;
             if (!(ready_mask >> sl & 1u)) {
-              PROF_B(); mbar_wait(rfull(sl), (slot_par >> sl & 1u)); PROF_E(2);
+              PROF_B(); mbar_wait(rfull(sl), (slot_par >> sl & 1u));
+              if (kFold) mbar_wait(xready(sl), (slot_par >> sl & 1u));  // norm digits expanded
+              PROF_E(2);
               ready_mask |= 1u << sl;
             }
             const uint64_t bd0 = smem_desc_sw128(sbase + SmemPlan::kR + sl * kRTileBytes);
+            const int np = c == cpr - 1 ? np_last : kPiecesPerChunk;
 #pragma unroll
             for (int pp = 0; pp < kPiecesPerChunk; ++pp) {  // static buffer / phase (see the epilogue)
+              if (pp >= np) break;  // all-padding pieces of the last chunk are never computed
               const uint32_t buf = mw * kNB + (pp & 1);
-              PROF_B(); mbar_wait(tempty(buf), ((pp >> 1) & 1) ^ 1); PROF_E(0);
+              PROF_B(); mbar_wait(tempty(buf), (((pp >> 1) ^ (ph_t >> (pp & 1))) & 1) ^ 1); PROF_E(0);
               tc_fence_after();
               // rows kPiece*pp.. of the chunk: SWIZZLE_128B core groups of 8 rows x 128 B
               const uint64_t bd = bd0 + pp * (kPiece * kDim >> 4);
@@ -625,6 +646,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               else
                 mma_piece<kIdescI8>(tmem_base + buf * kPiece, ad, bd, tfull(buf));
             }
+            ph_t ^= use_parity(np);
           }
         }
         if (s == J.nr - 1) {  // this warp's release of query tile t (covers all its prior MMAs)
@@ -640,7 +662,10 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         if (++s == J.nr) { s = 0; ++t; }
       }
       for (int sl = 0; sl < nslots; ++sl) {
-        if (!(ready_mask >> sl & 1u)) mbar_wait(rfull(sl), (slot_par >> sl & 1u));  // keep rempty phases ordered
+        if (!(ready_mask >> sl & 1u)) {  // keep rempty / xready phases ordered
+          mbar_wait(rfull(sl), (slot_par >> sl & 1u));
+          if (kFold) mbar_wait(xready(sl), (slot_par >> sl & 1u));
+        }
         mma_commit(rempty(sl));
         slot_par ^= 1u << sl;
       }
@@ -659,6 +684,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     const int nq_ld = T * kBM;
     const bool ratio32 = p.num2 <= 511u && p.den2 <= 511u;  // den^2 * d fits 32 bits (d <= 8,323,200)
     uint32_t slot_par = 0;                // bit sl = phase parity of reference slot sl
+    const int np_last = piece_count_last(p.m, cpr);
+    uint32_t ph_t = 0;                    // bit b: phase flip of TMEM buffer b (see the MMA warps)
     uint32_t v[64];
 
     for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
@@ -668,6 +695,51 @@ __global__ void __launch_bounds__(kNumThreads, 1)
       // column keys of every slot of the job (also orders this warp's rempty arrivals)
       PROF_B();
       for (int sl = 0; sl < nslots; ++sl) mbar_wait(rfull(sl), slot_par >> sl & 1u);
+      if constexpr (kFold) {
+        // the fifth MMA K-step's B operand, expanded here from the column terms W (HBM keeps only W:
+        // 4 B per keypoint instead of 32 B of digits).  Column i of a slot: 32 u8 digits of
+        // E = floor(W / 2) against the constant operand a = (255 x 15, 1, 255 x 15, 1):
+        // E = 255 * (sum of the 30 "255"-weighted digits) + d15 + d31, filled greedily (255, 255, ...,
+        // rest, 0, ...) in positions 0..14, 16..30 and d15 = E mod 255, d31 = 0 (capacity 7,650 * 255 +
+        // 254 > max E = 1,048,576).  Padding columns (W < 0) get zero digits.  Both 16-byte halves of
+        // the constant operand are equal, so the SWIZZLE_32B placement of a row's two halves does not
+        // change the product: rows are written plainly, 32 B each.
+        for (int x = ew * 32 + lane; x < nslots * kBN; x += kEpiWarps * 32) {
+          const int sl = x / kBN, col = x % kBN;
+          int W;
+          asm volatile("ld.shared.s32 %0, [%1];" : "=r"(W) : "r"(sbase + SmemPlan::kCol + sl * kColBytes + col * 4));
+          const uint32_t E = W > 0 ? static_cast<uint32_t>(W) >> 1 : 0u;
+          const uint32_t hi = E / 255u, lo = E - 255u * (E / 255u);
+          uint32_t w8[8];
+#pragma unroll
+          for (int wi = 0; wi < 8; ++wi) {
+            uint32_t word = 0;
+#pragma unroll
+            for (int bi = 0; bi < 4; ++bi) {
+              const int t = wi * 4 + bi;                          // digit position 0..31
+              const int rank = t < 15 ? t : (t < 31 && t > 15 ? t - 1 : -1);  // order among the 30 "255" digits
+              uint32_t dg;
+              if (t == 15) dg = lo;
+              else if (t == 31) dg = 0u;
+              else {
+                const int32_t rest = static_cast<int32_t>(hi) - 255 * rank;
+                dg = rest <= 0 ? 0u : (rest >= 255 ? 255u : static_cast<uint32_t>(rest));
+              }
+              word |= dg << (8 * bi);
+            }
+            w8[wi] = word;
+          }
+          const uint32_t dst = sbase + SmemPlan::kX + sl * kXTileBytes + col * kXDim;
+          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst), "r"(w8[0]), "r"(w8[1]), "r"(w8[2]),
+                       "r"(w8[3]) : "memory");
+          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst + 16), "r"(w8[4]), "r"(w8[5]), "r"(w8[6]),
+                       "r"(w8[7]) : "memory");
+        }
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> tensor-core reads
+        __syncwarp();
+        if (lane == 0)
+          for (int sl = 0; sl < nslots; ++sl) mbar_arrive(xready(sl));
+      }
       PROF_E(4);
       // own units u = g, g + kNG, ...; unit u = (tile t = u / nr, reference s = u % nr), and
       // t = (query qi - q_first) * T + tq.  Tracked incrementally (no divisions per unit).
@@ -696,10 +768,12 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             // 4 pieces per chunk through the group's 2 buffers: each buffer is used twice per chunk,
             // so buffer and phase are compile-time functions of pp (fully unrolled)
             static_assert(kNB == 2 && kPiecesPerChunk == 4, "static buffer / phase schedule");
+            const int np = c == cpr - 1 ? np_last : kPiecesPerChunk;
 #pragma unroll
             for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
+              if (pp >= np) break;  // all-padding pieces (m not a multiple of 64 x 4) are not computed
               const uint32_t buf = g * kNB + (pp & 1);
-              PROF_B(); mbar_wait(tfull(buf), (pp >> 1) & 1); PROF_E(0);
+              PROF_B(); mbar_wait(tfull(buf), ((pp >> 1) ^ (ph_t >> (pp & 1))) & 1); PROF_E(0);
               tc_fence_after();
 #ifndef TID_NOLOAD  // timing experiment only: scan stale registers (wrong results)
               tmem_ld64(taddr_q + buf * kPiece, v);
@@ -721,6 +795,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               }
               PROF_E(1);
             }
+            ph_t ^= use_parity(np);
             PROF_B();
             int x1, x2;
             finish_fold(R, T1, T2, x1, x2);
@@ -770,10 +845,12 @@ __global__ void __launch_bounds__(kNumThreads, 1)
 #pragma unroll
           for (int b = 0; b < 16; ++b) R[b] = INT_MAX;
           int T1 = INT_MAX, T2 = INT_MAX;
+          const int np = c == cpr - 1 ? np_last : kPiecesPerChunk;
 #pragma unroll
           for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
+            if (pp >= np) break;
             const uint32_t buf = g * kNB + (pp & 1);
-            PROF_B(); mbar_wait(tfull(buf), (pp >> 1) & 1); PROF_E(0);
+            PROF_B(); mbar_wait(tfull(buf), ((pp >> 1) ^ (ph_t >> (pp & 1))) & 1); PROF_E(0);
             tc_fence_after();
             // x64 loads; the buffer is released as soon as its last load has landed
 #pragma unroll
@@ -792,6 +869,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               PROF_E(1);
             }
           }
+          ph_t ^= use_parity(np);
           PROF_B();
           int k1, k2;
           finish_partition(R, T1, T2, k1, k2);
@@ -870,8 +948,8 @@ extern "C" int tid_debug_read_prof(void* host, size_t bytes) {
 #endif
 
 
-cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap,
-                         const CUtensorMap* xmap, int grid, cudaStream_t s) {
+cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap, bool fold, int grid,
+                         cudaStream_t s) {
   // the shared-memory opt-in is per device: set once per device (host overhead matters for C1)
   static thread_local uint64_t attr_set = 0;  // bit d = device d configured
   int dev = 0;
@@ -885,10 +963,10 @@ cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CU
     if (e != cudaSuccess) return e;
     if (dev < 64) attr_set |= uint64_t(1) << dev;
   }
-  if (xmap)
-    match_kernel<true><<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, *xmap, p);
+  if (fold)
+    match_kernel<true><<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, p);
   else
-    match_kernel<false><<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, rmap, p);
+    match_kernel<false><<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, p);
   return cudaGetLastError();
 }
 
@@ -929,30 +1007,9 @@ __global__ void ref_prep_kernel(RefPrepParams p) {
 #pragma unroll
       for (int w = 0; w < kDim / 16; ++w) dst[w] = make_uint4(0, 0, 0, 0);
     }
-    if (p.extra) {
-      // u8 digits b of E = floor(W / 2) against the constant operand a = (255 x 15, 1, 255 x 15, 1):
-      // E = 255 * (sum of the 30 "255" digits) + b15 + b31  (capacity 1,951,260 >= max E = 1,048,576)
-      uint32_t d[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-      if (real) {
-        const uint32_t E = static_cast<uint32_t>(256 * sum - norm) >> 1;
-        uint32_t hi = E / 255;
-        const uint32_t lo = E - hi * 255;
-        uint8_t* db = reinterpret_cast<uint8_t*>(d);
-        for (int t = 0; t < kXDim && hi; ++t) {
-          if (t == 15 || t == 31) continue;
-          const uint32_t v = hi < 255 ? hi : 255;
-          db[t] = static_cast<uint8_t>(v);
-          hi -= v;
-        }
-        db[15] = static_cast<uint8_t>(lo);
-      }
-      uint4* xd = reinterpret_cast<uint4*>(p.extra + (r * p.m + i) * kXDim);
-      xd[0] = make_uint4(d[0], d[1], d[2], d[3]);
-      xd[1] = make_uint4(d[4], d[5], d[6], d[7]);
-    }
   }
   int32_t* ck = p.colkey + (r * p.cpr + c) * kColInts;
-  if (p.extra) {
+  if (p.search) {
     const int kpc = max(0, min(kp - c * kBN, kBN));  // real columns in this chunk
     ck[ii] = real ? 256 * sum - norm : -1 - kpc;
   } else {
@@ -1037,11 +1094,14 @@ __device__ void block_select(const uint64_t* lists, int k, uint64_t* out, uint64
   }
 }
 
-// grid (B, segs), 256 threads, dyn smem = 256*k*8 + 33*8.  With one segment and ids_out set, the
-// block's winners are the final ranking: written as (ids, counts) directly (no merge launch).
+// grid (B, segs), 256 threads, dyn smem = 256*k*8 + 33*8.  Block (b, seg) writes its k winners to
+// list (list0 + seg) of query b, lists_per_b lists per query (a search over several reference
+// windows keeps its running top-k in list 0 and the window's segments after it).  With one
+// segment and ids_out set, the block's winners are the final ranking: written as (ids, counts)
+// directly (no merge launch).
 __global__ void topk_kernel(const uint32_t* __restrict__ counts, int64_t R, int64_t ldc, int64_t id_base, int32_t k,
-                            const uint8_t* __restrict__ dead, uint64_t* __restrict__ cand_out,
-                            int64_t* __restrict__ ids_out, int32_t* __restrict__ counts_out) {
+                            const uint8_t* __restrict__ dead, uint64_t* __restrict__ cand_out, int32_t lists_per_b,
+                            int32_t list0, int64_t* __restrict__ ids_out, int32_t* __restrict__ counts_out) {
   extern __shared__ uint64_t tk_smem[];
   uint64_t* lists = tk_smem;
   uint64_t* red = tk_smem + blockDim.x * k;
@@ -1063,7 +1123,7 @@ __global__ void topk_kernel(const uint32_t* __restrict__ counts, int64_t R, int6
     }
   }
   __syncthreads();
-  uint64_t* out = cand_out + (static_cast<int64_t>(b) * segs + seg) * k;
+  uint64_t* out = cand_out + (static_cast<int64_t>(b) * lists_per_b + list0 + seg) * k;
   block_select(lists, k, out, red);
   if (ids_out) {  // segs == 1: final (count desc, id asc) ranking
     __syncthreads();
@@ -1075,23 +1135,34 @@ __global__ void topk_kernel(const uint32_t* __restrict__ counts, int64_t R, int6
   }
 }
 
+// Opt a kernel into > 48 KiB of dynamic shared memory once per (device, size): the attribute is
+// per device, so one bit per device and size class (thread-local: no shared mutable state).
+template <class F>
+void ensure_smem_attr(F* fn, size_t smem, int which) {
+  if (smem <= 48 * 1024) return;
+  static thread_local size_t done[2][64] = {};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 64 && done[which][dev] >= smem) return;
+  cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
+  if (dev < 64) done[which][dev] = smem;
+}
+
 void launch_topk(const uint32_t* counts, int64_t B, int64_t R, int64_t ldc, int64_t id_base, int32_t k, int32_t segs,
-                 const uint8_t* dead, uint64_t* cand_out, cudaStream_t s, int64_t* ids_out, int32_t* counts_out) {
+                 const uint8_t* dead, uint64_t* cand_out, int32_t lists_per_b, int32_t list0, cudaStream_t s,
+                 int64_t* ids_out, int32_t* counts_out) {
   const size_t smem = (256 * static_cast<size_t>(k) + 33) * 8;
-  static size_t attr = 0;
-  if (smem > 48 * 1024 && smem > attr) {
-    cudaFuncSetAttribute(topk_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
-    attr = smem;
-  }
+  ensure_smem_attr(topk_kernel, smem, 0);
   topk_kernel<<<dim3(static_cast<unsigned>(B), static_cast<unsigned>(segs)), 256, smem, s>>>(
-      counts, R, ldc, id_base, k, dead, cand_out, segs == 1 ? ids_out : nullptr, segs == 1 ? counts_out : nullptr);
+      counts, R, ldc, id_base, k, dead, cand_out, lists_per_b, list0, segs == 1 ? ids_out : nullptr,
+      segs == 1 ? counts_out : nullptr);
 }
 
 // ------------------------------------------------------------------ a6/a9: merge ranked lists
 // L candidate lists of k keys per query (list l of query b at cand[b*sb + l*sl]).  One block
 // of 128 threads per query: each thread gathers its share, sorts it, then block_select.
-__global__ void merge_kernel(const uint64_t* __restrict__ cand, int32_t L, int32_t k, int64_t sb, int64_t sl,
-                             uint64_t* __restrict__ keys_out, int64_t* __restrict__ ids_out,
+__global__ void merge_kernel(const uint64_t* cand, int32_t L, int32_t k, int64_t sb, int64_t sl,
+                             uint64_t* keys_out, int64_t keys_stride, int64_t* __restrict__ ids_out,
                              int32_t* __restrict__ counts_out) {
   extern __shared__ uint64_t mg_smem[];
   uint64_t* lists = mg_smem;  // blockDim.x * k
@@ -1116,22 +1187,19 @@ __global__ void merge_kernel(const uint64_t* __restrict__ cand, int32_t L, int32
   block_select(lists, k, win, red);
   for (int i = threadIdx.x; i < k; i += blockDim.x) {
     const uint64_t key = win[i];
-    if (keys_out) keys_out[static_cast<int64_t>(b) * k + i] = key;
+    if (keys_out) keys_out[static_cast<int64_t>(b) * keys_stride + i] = key;
     if (ids_out) ids_out[static_cast<int64_t>(b) * k + i] = key ? static_cast<int64_t>(kIdMask - (key & kIdMask)) : -1;
     if (counts_out) counts_out[static_cast<int64_t>(b) * k + i] = static_cast<int32_t>(key >> 40);
   }
 }
 
 void launch_merge(const uint64_t* cand, int32_t L, int64_t B, int32_t k, int64_t sb, int64_t sl, uint64_t* keys_out,
-                  int64_t* ids_out, int32_t* counts_out, cudaStream_t s) {
+                  int64_t* ids_out, int32_t* counts_out, cudaStream_t s, int64_t keys_stride) {
   const int threads = 128;
   const size_t smem = (threads * static_cast<size_t>(k) + 33 + k) * 8;
-  static size_t attr = 0;
-  if (smem > 48 * 1024 && smem > attr) {
-    cudaFuncSetAttribute(merge_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
-    attr = smem;
-  }
-  merge_kernel<<<static_cast<unsigned>(B), threads, smem, s>>>(cand, L, k, sb, sl, keys_out, ids_out, counts_out);
+  ensure_smem_attr(merge_kernel, smem, 1);
+  merge_kernel<<<static_cast<unsigned>(B), threads, smem, s>>>(cand, L, k, sb, sl, keys_out,
+                                                               keys_stride > 0 ? keys_stride : k, ids_out, counts_out);
 }
 
 __global__ void pack_kernel(const int64_t* ids, const int32_t* counts, int64_t n, uint64_t* keys) {

@@ -96,7 +96,8 @@ struct RefPrepParams {
   const uint8_t* src;        // optional source to copy from (null = in place)
   const int32_t* kp;         // [count] or null (= m)
   int32_t* colkey;           // [count][cpr][256]: packed keys (verify) or column terms (search)
-  uint8_t* extra;            // search only: [count][m][32] u8 digits of floor(W / 2) (null = verify keys)
+  int32_t search;            // 1: search column terms W (the norm-term digits are expanded on chip
+                             //    by the match kernel); 0: verify packed keys
   int64_t count;
   int32_t m;
   int32_t cpr;
@@ -105,15 +106,20 @@ struct RefPrepParams {
 void launch_ref_prep(const RefPrepParams& p, cudaStream_t s);
 void launch_query_prep(const uint8_t* q, int64_t B, int32_t n, int32_t tiles_per_q, int32_t* nq,
                        uint8_t* qs, cudaStream_t s);
-cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap,
-                         const CUtensorMap* xmap, int grid, cudaStream_t s);
+// fold = search path (s8 x u8 + on-chip norm-term K-step, counts); otherwise verify (exact 2-NN)
+cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap, bool fold, int grid,
+                         cudaStream_t s);
 // ids_out / counts_out (optional): with segs == 1 the final ranking is written directly
+// Candidate lists: cand_out holds lists_per_b lists of k keys per query; the launch's segments
+// fill lists list0 .. list0 + segs - 1.
 void launch_topk(const uint32_t* counts, int64_t B, int64_t R, int64_t ldc, int64_t id_base, int32_t k,
-                 int32_t segs, const uint8_t* dead, uint64_t* cand_out, cudaStream_t s, int64_t* ids_out = nullptr,
-                 int32_t* counts_out = nullptr);
+                 int32_t segs, const uint8_t* dead, uint64_t* cand_out, int32_t lists_per_b, int32_t list0,
+                 cudaStream_t s, int64_t* ids_out = nullptr, int32_t* counts_out = nullptr);
+// keys_out (optional) row stride keys_stride (0 = k); may alias list 0 of cand (in-place running merge:
+// every block reads all its lists before writing).
 void launch_merge(const uint64_t* cand, int32_t L, int64_t B, int32_t k, int64_t list_stride_b,
                   int64_t list_stride_l, uint64_t* keys_out, int64_t* ids_out, int32_t* counts_out,
-                  cudaStream_t s);
+                  cudaStream_t s, int64_t keys_stride = 0);
 void launch_pack_lists(const int64_t* ids, const int32_t* counts, int64_t n, uint64_t* keys, cudaStream_t s);
 size_t match_smem_bytes();
 

@@ -80,3 +80,36 @@ def test_plain_c_example_compiles_and_links(tmp_path):
                            os.path.join(root, "examples", "search_example.c"), "-L", lib_dir, "-ltid",
                            f"-Wl,-rpath,{lib_dir}", "-o", str(out)])
     assert out.exists()
+
+
+def test_binding_checks_output_buffers():
+    """Caller-supplied outputs are checked, never converted: a wrong dtype / shape, a
+    non-contiguous or read-only array, or a CUDA tensor on another device raises before any
+    library call (an int32 ids buffer would otherwise be overrun by the int64 writes)."""
+    import numpy as np
+    import pytest
+    import torch
+    from paper_conf_icpp_wangzll21_b200 import _out_ptr, _ptr
+    ok = np.empty((3, 5), np.int64)
+    assert _out_ptr(ok, (3, 5), np.int64, 0, "ids") == ok.ctypes.data
+    with pytest.raises(TypeError):
+        _out_ptr(np.empty((3, 5), np.int32), (3, 5), np.int64, 0, "ids")
+    with pytest.raises(TypeError):
+        _out_ptr(np.empty((3, 4), np.int64), (3, 5), np.int64, 0, "ids")
+    with pytest.raises(ValueError):
+        _out_ptr(np.empty((5, 3), np.int64).T, (3, 5), np.int64, 0, "ids")
+    ro = np.empty((3, 5), np.int64)
+    ro.flags.writeable = False
+    with pytest.raises(ValueError):
+        _out_ptr(ro, (3, 5), np.int64, 0, "ids")
+    with pytest.raises(TypeError):
+        _out_ptr(torch.empty((3, 5), dtype=torch.int32), (3, 5), np.int64, 0, "ids")
+    t = torch.empty((3, 5), dtype=torch.int64)
+    assert _out_ptr(t, (3, 5), np.int64, 0, "ids") == t.data_ptr()
+    with pytest.raises(TypeError):
+        _out_ptr([0] * 15, (15,), np.int64, 0, "ids")
+    # inputs: torch tensors must already have the right dtype (no silent reinterpretation)
+    with pytest.raises(TypeError):
+        _ptr(torch.zeros((2, 3, 128), dtype=torch.int32), np.uint8)
+    p, keep = _ptr(np.zeros((2, 3, 128), np.int64), np.uint8)  # numpy inputs are converted
+    assert keep.dtype == np.uint8

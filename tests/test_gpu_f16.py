@@ -85,3 +85,20 @@ def test_f16_ratio_boundary(tid):
         got = idx.f16_search_counts(q, R)
     assert got.tolist() == [[0, 5]]
     np.testing.assert_array_equal(got.astype(np.int64), oracle.f16_search_counts(q, R))
+
+
+def test_f16_rootsift_parity_at_scale(tid):
+    """f1 acceptance at the verdict's scale: 64 RootSIFT queries (1000 keypoints) x 2,000 references
+    (256 keypoints) in fp16 — 128,000 pairs — vs the C float64 oracle on the same fp16 values:
+    |count difference| <= 1 for >= 99.9 % of pairs, and the planted target ranks first."""
+    B, n, R, m = 64, 1000, 2000, 256
+    Rr, _ = tidgen.refs(0, R, m, seed=2021)
+    Q, tg = tidgen.queries(0, B, n, R_total=R, m=m, seed=2021)
+    with tid.Index(query_kp_max=1024) as idx:
+        q16, r16 = idx.f16_prepare(Q, True, 1.0), idx.f16_prepare(Rr, True, 1.0)
+        got = idx.f16_search_counts(q16, r16).astype(np.int64)
+    want = oracle.f16_search_counts_c(q16, r16).astype(np.int64)
+    diff = np.abs(got - want)
+    assert diff.max() <= 2, diff.max()
+    assert np.mean(diff <= 1) >= 0.999, np.mean(diff <= 1)
+    np.testing.assert_array_equal(np.argmax(got, 1), tg)

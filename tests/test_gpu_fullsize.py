@@ -3,7 +3,8 @@
 C4 (bench default: 256 queries x 1000 keypoints vs a 125,000-reference x 256-keypoint shard)
 and C3 (64 x 100,000) are too large for the oracle in full, so they are checked
   * on sampled outputs the oracle computes one by one: the count of every (query, reference)
-    pair in a seeded random sample, plus every planted target, exactly;
+    pair in a seeded random sample, plus every planted target, exactly; and whole count rows
+    (4 C4 queries x all 125,000 references, 2 C3 queries x all 100,000) element by element;
   * by properties that hold at any size: every planted target ranks first; the top-k returned by
     tid_search equals the (count desc, id asc) ranking of the full GPU count matrix re-sorted
     on the host; counts never exceed n.
@@ -33,7 +34,7 @@ def tid():
     return t
 
 
-def _sampled_search_check(tid, B, n, R, m, k, n_sample_q, n_sample_r):
+def _sampled_search_check(tid, B, n, R, m, k, n_sample_q, n_sample_r, n_full_q):
     import torch
     refs, _ = tidgen.refs(0, R, m, seed=SEED)
     qs, targets = tidgen.queries(0, B, n, R_total=R, m=m, seed=SEED)
@@ -61,16 +62,21 @@ def _sampled_search_check(tid, B, n, R, m, k, n_sample_q, n_sample_r):
         rsel = np.unique(np.concatenate([rng.choice(R, size=n_sample_r, replace=False), [targets[q]], ids[q]]))
         want = oracle.search_counts(qs[q:q + 1], refs[rsel])[0]
         np.testing.assert_array_equal(counts[q, rsel], want, err_msg=f"query {q}")
+    # whole count rows: n_full_q seeded queries against EVERY reference, element by element
+    # (SURVEY §8(d) oracle plan; the oracle's OpenMP over references on all host cores)
+    fsel = np.sort(np.random.default_rng(SEED + 7 * B).choice(B, size=n_full_q, replace=False))
+    want = oracle.search_counts(qs[fsel], refs)
+    np.testing.assert_array_equal(counts[fsel], want)
 
 
 def test_c4_fullsize_sampled(tid):
-    """C4 per-GPU shard (bench.py's workload): 256 queries x 125,000 references."""
-    _sampled_search_check(tid, B=256, n=1000, R=125_000, m=256, k=5, n_sample_q=16, n_sample_r=120)
+    """C4 per-GPU shard (bench.py's workload): 256 queries x 125,000 references; 4 whole rows."""
+    _sampled_search_check(tid, B=256, n=1000, R=125_000, m=256, k=5, n_sample_q=16, n_sample_r=120, n_full_q=4)
 
 
 def test_c3_fullsize_sampled(tid):
-    """C3: 64 queries x 100,000 references."""
-    _sampled_search_check(tid, B=64, n=1000, R=100_000, m=256, k=5, n_sample_q=8, n_sample_r=120)
+    """C3: 64 queries x 100,000 references; 2 whole rows."""
+    _sampled_search_check(tid, B=64, n=1000, R=100_000, m=256, k=5, n_sample_q=8, n_sample_r=120, n_full_q=2)
 
 
 def test_c2_full_verify_bitexact(tid):

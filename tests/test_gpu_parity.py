@@ -203,10 +203,12 @@ def test_host_tier_map_zero_copy(tid):
 
 
 def test_virtual_shards_merge_equals_single(tid):
-    """G shards run one after another on one GPU, merged by the shard-merge kernel == 1 GPU."""
+    """G shards run one after another on one GPU, merged by the shard-merge kernel == the
+    oracle's global top-k (and the 1-GPU search)."""
     R, m, n, B, k = 96, 256, 300, 3, 6
     refs, _ = tidgen.refs(0, R, m, K=16)        # K=16 clusters: many equal counts -> id tie-breaks
     qs, _ = tidgen.queries(0, B, n, R_total=R, m=m, K=16, n_planted=30)
+    e_ids, e_cnt, _ = oracle.search(qs, refs, k)
     with tid.Index(ref_kp=m) as one:
         one.add_references(refs)
         gi, gc = one.search(qs, k)
@@ -223,8 +225,10 @@ def test_virtual_shards_merge_equals_single(tid):
                 li.append(i); lc.append(c)
         with tid.Index(ref_kp=m) as mg:
             mi, mc = mg.merge_topk(np.stack(li), np.stack(lc))
-        np.testing.assert_array_equal(mi, gi)
-        np.testing.assert_array_equal(mc, gc)
+        np.testing.assert_array_equal(mi, e_ids)
+        np.testing.assert_array_equal(mc, e_cnt)
+    np.testing.assert_array_equal(gi, e_ids)
+    np.testing.assert_array_equal(gc, e_cnt)
 
 
 def test_device_tensors_and_stream(tid):
@@ -251,8 +255,8 @@ def test_device_tensors_and_stream(tid):
 def test_search_fast_path_fallback(tid, rng, hi):
     """Search path (folded norms: d known to +-1 from the MMA, exact global-memory recompute of
     the rows whose ratio decision that leaves open): low-range data makes many rows undecided,
-    full-range data almost none; both must equal the oracle bit for bit.  `exact_only` is an
-    accepted no-op tuning flag (kept for ABI stability) and must not change anything."""
+    full-range data almost none; both must equal the oracle bit for bit (count matrix and
+    top-k)."""
     R, m, n, B = 24, 256, 300, 2
     refs = rng.integers(0, hi, (R, m, 128), dtype=np.uint8)
     qs = rng.integers(0, hi, (B, n, 128), dtype=np.uint8)
@@ -261,10 +265,11 @@ def test_search_fast_path_fallback(tid, rng, hi):
     with tid.Index(ref_kp=m) as idx:
         idx.add_references(refs)
         fast = idx.search_counts(qs)
-        idx.set_tuning(exact_only=True)
-        exact = idx.search_counts(qs)
-    np.testing.assert_array_equal(fast, exact)
-    np.testing.assert_array_equal(fast.astype(np.int64), oracle.search_counts(qs, refs))
+        ids, cnt = idx.search(qs, 5)
+    e_ids, e_cnt, e_counts = oracle.search(qs, refs, 5)
+    np.testing.assert_array_equal(fast.astype(np.int64), e_counts)
+    np.testing.assert_array_equal(ids, e_ids)
+    np.testing.assert_array_equal(cnt, e_cnt)
 
 
 def test_search_boundary_ratios(tid):
@@ -290,15 +295,14 @@ def test_search_boundary_ratios(tid):
 
 
 def test_nccl_collective_path_single_rank(tid):
-    """The multi-GPU path (local top-k -> ncclAllGather -> merge kernel) on a one-rank NCCL
-    communicator must return exactly the single-GPU result."""
+    """The multi-GPU path (collective reference count, local top-k -> ncclAllGather -> merge
+    kernel) on a one-rank NCCL communicator must return exactly the oracle's top-k, with one
+    count window and with several (running top-k), host and device buffers."""
     import torch  # loads PyTorch's NCCL first; libtid resolves the already-loaded library
     R, m, n, B, k = 80, 256, 300, 4, 7
     refs, _ = tidgen.refs(0, R, m, K=16)
     qs, _ = tidgen.queries(0, B, n, R_total=R, m=m, K=16, n_planted=40)
-    with tid.Index(ref_kp=m) as one:
-        one.add_references(refs)
-        gi, gc = one.search(qs, k)
+    gi, gc, _ = oracle.search(qs, refs, k)
     with tid.Index(ref_kp=m, rank=0, world_size=1, nccl_id=tid.nccl_unique_id()) as col:
         col.add_references(refs)
         ci, cc = col.search(qs, k)
@@ -306,10 +310,128 @@ def test_nccl_collective_path_single_rank(tid):
         di, dc = col.search(dq, k, out=(torch.empty((B, k), dtype=torch.int64, device="cuda"),
                                        torch.empty((B, k), dtype=torch.int32, device="cuda")))
         torch.cuda.synchronize()
+        col.set_tuning(window_refs=13)
+        wi, wc = col.search(qs, k)
+        with pytest.raises(tid.TidError) as e:
+            col.search(qs, R + 1)  # k > total references: refused on every rank alike
+        assert e.value.status == tid.TID_EINVAL
     np.testing.assert_array_equal(ci, gi)
     np.testing.assert_array_equal(cc, gc)
     np.testing.assert_array_equal(di.cpu().numpy(), gi)
     np.testing.assert_array_equal(dc.cpu().numpy(), gc)
+    np.testing.assert_array_equal(wi, gi)
+    np.testing.assert_array_equal(wc, gc)
+
+
+def test_nccl_empty_shard(tid):
+    """A rank whose shard is empty still joins the collective (it used to return
+    TID_ESTATE before the all-gather and hang the other ranks).  On a one-rank communicator the
+    total is then 0: TID_ESTATE, raised after the collective count, consistently; once a
+    reference exists the same index searches normally."""
+    R, m, n, B = 5, 256, 200, 2
+    refs, _ = tidgen.refs(0, R, m)
+    qs, _ = tidgen.queries(0, B, n, R_total=R, m=m, n_planted=40)
+    with tid.Index(ref_kp=m, rank=0, world_size=1, nccl_id=tid.nccl_unique_id()) as col:
+        with pytest.raises(tid.TidError) as e:
+            col.search(qs, 1)
+        assert e.value.status == tid.TID_ESTATE
+        col.add_references(refs)
+        ids, cnt = col.search(qs, R)
+    e_ids, e_cnt, _ = oracle.search(qs, refs, R)
+    np.testing.assert_array_equal(ids, e_ids)
+    np.testing.assert_array_equal(cnt, e_cnt)
+
+
+@pytest.mark.parametrize("W", [1, 7, 64, 4096])
+def test_search_count_windows(tid, W):
+    """tid_search over several count windows (window_refs = W): each window's counts are reduced
+    into a running top-k (so the workspace does not grow with R); the ranking must equal the
+    oracle's over the whole set, incl. heavy id tie-breaks (K = 16), deleted references, ragged
+    kp and a host tier whose staging chunks straddle window boundaries."""
+    R, m, n, B, k = 150, 256, 260, 3, 9
+    refs, kp = tidgen.refs(0, R, m, K=16, kp_min=100, pad_byte=9)
+    qs, _ = tidgen.queries(0, B, n, R_total=R, m=m, K=16, n_planted=40)
+    dead = [3, 64, 65, 149]
+    keep = np.setdiff1d(np.arange(R), dead)
+    c = oracle.search_counts(qs, refs, kp=kp)
+    e_ids, e_cnt = oracle.np_rank(c[:, keep], k)
+    e_ids = keep[e_ids]
+    rb = m * 128
+    for host in (False, True):
+        kw = dict(hbm_budget_bytes=40 * rb, host_budget_bytes=200 * rb) if host else {}
+        with tid.Index(ref_kp=m, **kw) as idx:
+            idx.add_references(refs, kp)
+            idx.set_tuning(window_refs=W, host_chunk_refs=11)
+            idx.delete(dead)
+            ids, cnt = idx.search(qs, k)
+            if host:
+                assert idx.info()["host_references"] == R - 40
+        np.testing.assert_array_equal(ids, e_ids, err_msg=f"host={host}")
+        np.testing.assert_array_equal(cnt, e_cnt, err_msg=f"host={host}")
+
+
+def test_add_all_or_nothing(tid, monkeypatch):
+    """tid_add_references is all-or-nothing: an allocation failure in
+    the middle of an add (injected with TID_FAULT_ALLOC: here the host-tier segment, after a new
+    HBM segment was already allocated and filled) leaves the index exactly as before — same
+    counts per tier, same ids, same search results — and the next add succeeds."""
+    m, n, B, k = 256, 300, 2, 5
+    rb = m * 128
+    refs, _ = tidgen.refs(0, 30, m)
+    qs, _ = tidgen.queries(0, B, n, R_total=30, m=m, n_planted=40)
+    with tid.Index(ref_kp=m, hbm_budget_bytes=10 * rb, host_budget_bytes=100 * rb) as idx:
+        assert idx.add_references(refs[:5]) == 0
+        before = idx.info()
+        monkeypatch.setenv("TID_FAULT_ALLOC", "2")  # 1st alloc: new HBM segment; 2nd: host tier
+        with pytest.raises(tid.TidError) as e:
+            idx.add_references(refs[5:25])
+        assert e.value.status == tid.TID_ENOMEM
+        monkeypatch.delenv("TID_FAULT_ALLOC")
+        assert idx.info() == before
+        ids, cnt = idx.search(qs, k)
+        e_ids, e_cnt, _ = oracle.search(qs, refs[:5], k)
+        np.testing.assert_array_equal(ids, e_ids)
+        np.testing.assert_array_equal(cnt, e_cnt)
+        idx.delete([1])  # dead flags sized to the committed references only
+        assert idx.add_references(refs[5:30]) == 5
+        info = idx.info()
+        assert (info["hbm_references"], info["host_references"]) == (10, 20)
+        ids, cnt = idx.search(qs, k)
+    c = oracle.search_counts(qs, refs)
+    c[:, 1] = -1
+    e_ids, e_cnt = oracle.np_rank(c, k)
+    np.testing.assert_array_equal(ids, e_ids)
+    np.testing.assert_array_equal(cnt, e_cnt)
+
+
+def test_calls_on_different_streams(tid):
+    """One index driven from two non-blocking torch streams back to back, device outputs, no host
+    synchronisation in between: each call's work is ordered after the previous call's (the
+    index's end-of-call event), so reused workspaces are never overwritten in flight."""
+    import torch
+    R, m, n, B, k = 200, 256, 1000, 8, 5
+    refs, _ = tidgen.refs(0, R, m)
+    qa, _ = tidgen.queries(0, B, n, R_total=R, m=m)
+    qb, _ = tidgen.queries(50, B, 700, R_total=R, m=m)
+    with tid.Index(ref_kp=m) as idx:
+        idx.add_references(refs)
+        s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+        da, db = torch.from_numpy(qa).cuda(), torch.from_numpy(qb).cuda()
+        torch.cuda.synchronize()
+        outs = []
+        for i in range(4):
+            st = s1 if i % 2 == 0 else s2
+            with torch.cuda.stream(st):
+                o = (torch.empty((B, k), dtype=torch.int64, device="cuda"),
+                     torch.empty((B, k), dtype=torch.int32, device="cuda"))
+                idx.search(da if i % 2 == 0 else db, k, out=o)
+                outs.append(o)
+        torch.cuda.synchronize()
+    ea, eac, _ = oracle.search(qa, refs, k)
+    eb, ebc, _ = oracle.search(qb, refs, k)
+    for i, (ids, cnt) in enumerate(outs):
+        np.testing.assert_array_equal(ids.cpu().numpy(), ea if i % 2 == 0 else eb)
+        np.testing.assert_array_equal(cnt.cpu().numpy(), eac if i % 2 == 0 else ebc)
 
 
 @pytest.mark.parametrize("m,n,kp_min", [(384, 768, 384), (384, 768, 100), (1024, 300, 500)])
@@ -454,3 +576,21 @@ def test_plain_c_example_runs(tid, tmp_path):
     out = subprocess.run([str(exe)], capture_output=True, text=True, timeout=120)
     assert out.returncode == 0, out.stdout + out.stderr
     assert "verify(query 0, reference 3): 200 good matches" in out.stdout
+
+
+def test_hbm_capacity_per_reference(tid):
+    """HBM capacity (the paper's second headline metric): a resident
+    m = 256 reference costs its 32,768 descriptor bytes plus 1 KiB of column terms W (the
+    fifth MMA K-step's norm digits are expanded on chip from W, not stored), so the automatic
+    budget of a 180 GB B200 holds >= 5 M references; m = 384 costs 49,152 + 2 KiB."""
+    import torch
+    free, total = torch.cuda.mem_get_info()
+    with tid.Index(ref_kp=256) as idx:
+        info = idx.info()
+    assert info["hbm_bytes_per_reference"] == 256 * 128 + 1024
+    cap = info["hbm_capacity_references"]
+    assert cap * 256 * 128 <= free
+    if total > 170e9:
+        assert cap >= 4_900_000, cap
+    with tid.Index(ref_kp=384) as idx:
+        assert idx.info()["hbm_bytes_per_reference"] == 384 * 128 + 2048

@@ -101,3 +101,26 @@ def test_compression_error_zero_distance_pairs_excluded():
     Rf[0, 0] = 0.1
     e = oracle.compression_error(Qf, Rf, oracle.to_fp16(Qf).astype(np.float64), oracle.to_fp16(Rf).astype(np.float64))
     np.testing.assert_allclose(e, u / 0.1, rtol=1e-12)
+
+
+def test_f16_c_oracle_equals_numpy_and_exact(rng):
+    """The C float64 oracle (oracle_f64_search_counts) against two independent references:
+    (i) the NumPy float formulation on RootSIFT fp16 data with ragged n_q / kp (distances from a
+    broadcast matrix + partition, a different summation order); (ii) the exact integer oracle
+    on u8 SIFT x 2^-7 (exact in fp16)."""
+    R, _ = tidgen.refs(11, 7, 96)
+    Q, _ = tidgen.queries(11, 3, 120, R_total=7, m=96, n_planted=40)
+    q16 = oracle.to_fp16(oracle.rootsift(Q))
+    r16 = oracle.to_fp16(oracle.rootsift(R))
+    n_q = np.array([120, 77, 5], np.int32)
+    kp = np.array([96, 1, 2, 50, 96, 0, 33], np.int32)
+    got = oracle.f16_search_counts_c(q16, r16, n_q=n_q, kp=kp)
+    want = np.zeros_like(got)
+    for b in range(3):
+        for r in range(7):
+            want[b, r] = oracle.f16_match_count(q16[b], r16[r], n_q=int(n_q[b]), m_r=int(kp[r]))
+    np.testing.assert_array_equal(got, want)
+    assert got[:, 1].sum() == 0 and got[:, 5].sum() == 0 and got.max() > 0
+    s = 2.0 ** -7
+    np.testing.assert_array_equal(oracle.f16_search_counts_c(oracle.to_fp16(Q, s), oracle.to_fp16(R, s)),
+                                  oracle.search_counts(Q, R))
