@@ -34,7 +34,7 @@ DIM = 128
 def build(force: bool = False) -> str:
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         tmp = _LIB + ".tmp%d" % os.getpid()
-        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-shared", "-fPIC", "-o", tmp, _SRC])
+        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-ffp-contract=off", "-shared", "-fPIC", "-o", tmp, _SRC])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -61,6 +61,9 @@ def _L():
         lib.oracle_topk.argtypes = [vp, i64, i64, i64, i32, vp, vp]
         lib.oracle_merge_topk.argtypes = [vp, vp, i32, i64, i32, vp, vp]
         lib.oracle_f64_search_counts.argtypes = [vp, vp, i32, i64, vp, vp, i32, i64, u32, u32, vp]
+        f32 = ctypes.c_float
+        lib.oracle_geometric.argtypes = [vp, i32, i32, i64, vp, vp, vp, vp, f32, f32, f32, f32, f32, f32, i32,
+                                         ctypes.c_uint64, u32, u32, vp, vp, vp]
         _lib = lib
     return _lib
 
@@ -272,6 +275,27 @@ def f16_search_counts_c(Qs16, Rs16, num: int = 4, den: int = 5, n_q=None, kp=Non
     counts = np.empty((B, Rn), np.int32)
     _L().oracle_f64_search_counts(_p(Q), _p(nq), n, B, _p(R), _p(kpa), m, Rn, num, den, _p(counts))
     return counts
+
+
+def geometric(nn, q_xy, r_xy, *, border=0.0, q_size=(1e9, 1e9), r_size=(1e9, 1e9), inlier_px=3.0,
+              iterations=256, seed=2021, num=4, den=5, n_q=None, m_r=None):
+    """f4 post-match verification (readings R14-R16 in the C
+    header): from verify's nn [P][n][4], query / reference keypoint coordinates [P][n][2] /
+    [P][m][2] -> (good [P] = ratio-test matches surviving edge removal, inliers [P] of the best
+    2-point similarity hypothesis, model [P][4] = (a, b, tx, ty))."""
+    nn = _c(nn, np.int64)
+    P, n = nn.shape[0], nn.shape[1]
+    q_xy, r_xy = _c(q_xy, np.float32), _c(r_xy, np.float32)
+    m = r_xy.shape[1]
+    assert q_xy.shape == (P, n, 2) and r_xy.shape[0] == P and r_xy.shape[2] == 2
+    nq = None if n_q is None else _c(n_q, np.int32)
+    mr = None if m_r is None else _c(m_r, np.int32)
+    good, inl = np.empty(P, np.int32), np.empty(P, np.int32)
+    model = np.empty((P, 4), np.float64)
+    _L().oracle_geometric(_p(nn), n, m, P, _p(nq), _p(mr), _p(q_xy), _p(r_xy), border, q_size[0], q_size[1],
+                          r_size[0], r_size[1], inlier_px, iterations, seed, num, den, _p(good), _p(inl),
+                          _p(model))
+    return good, inl, model
 
 
 def compression_error(Qf, Rf, Q16, R16) -> float:

@@ -209,3 +209,115 @@ void oracle_f64_search_counts(const double* Qs, const int32_t* n_q, int32_t n, i
       counts[b * R + r] = c;
     }
 }
+
+/*
+ * f4 post-match verification (§3.1 P:284-285 "the geometric
+ * verification is performed to remove the outliers that may be mismatched", "ratio
+ * test and edge feature removing").  The paper names the steps but defines neither; the
+ * readings (R14-R16) are:
+ *   R14 edge-feature removal: a good match (ratio test passed) is dropped when its query
+ *       keypoint or its nearest reference keypoint lies within `border` pixels of its image's
+ *       edge: x < border or y < border or x >= W - border or y >= H - border.
+ *   R15 geometric model: a 2-D similarity transform from query to reference coordinates,
+ *       X = a x - b y + tx, Y = b x + a y + ty, fitted exactly to 2 matches (p1, p2 -> q1, q2):
+ *       dp = p2 - p1, dq = q2 - q1, den = |dp|^2 (den == 0: no hypothesis),
+ *       a = (dpx dqx + dpy dqy) / den, b = (dpx dqy - dpy dqx) / den,
+ *       tx = q1x - (a p1x - b p1y), ty = q1y - (b p1x + a p1y);
+ *       a match is an inlier when (a x - b y + tx - X)^2 + (b x + a y + ty - Y)^2 < thr^2.
+ *   R16 hypotheses: RANSAC with `iters` hypotheses; hypothesis t draws the match pair from
+ *       h = splitmix64(seed * 2^32 + pair) mixed with t (below): u = h mod M, v = (h >> 32) mod
+ *       (M - 1), v += (v >= u); iters == 0 means every pair u < v (exhaustive, the limit).
+ *       The best hypothesis has the most inliers, ties to the earliest; M < 2 gives 0 inliers
+ *       and no model.  Matches are numbered in ascending query-keypoint order.
+ * All geometry in IEEE double with every operation rounded separately (the file is compiled
+ * with -ffp-contract=off), in the order written above.
+ */
+static uint64_t geo_mix(uint64_t z) {
+  z += 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+static int geo_fit(const double* p1, const double* p2, const double* q1, const double* q2, double m[4]) {
+  const double dpx = p2[0] - p1[0], dpy = p2[1] - p1[1];
+  const double dqx = q2[0] - q1[0], dqy = q2[1] - q1[1];
+  const double den = dpx * dpx + dpy * dpy;
+  if (den == 0.0) return 0;
+  const double a = (dpx * dqx + dpy * dqy) / den;
+  const double b = (dpx * dqy - dpy * dqx) / den;
+  m[0] = a;
+  m[1] = b;
+  m[2] = q1[0] - (a * p1[0] - b * p1[1]);
+  m[3] = q1[1] - (b * p1[0] + a * p1[1]);
+  return 1;
+}
+
+static int32_t geo_inliers(const double* P, const double* Q, int32_t M, const double m[4], double thr2) {
+  int32_t c = 0;
+  for (int32_t k = 0; k < M; ++k) {
+    const double x = P[2 * k], y = P[2 * k + 1];
+    const double ex = m[0] * x - m[1] * y + m[2] - Q[2 * k];
+    const double ey = m[1] * x + m[0] * y + m[3] - Q[2 * k + 1];
+    c += ex * ex + ey * ey < thr2;
+  }
+  return c;
+}
+
+/*
+ * nn [P][n][4] (d1, i1, d2, i2) from oracle_verify; q_xy [P][n][2], r_xy [P][m][2] (float).
+ * Outputs per pair: good[p] = matches after the ratio test and edge removal, inl[p] = inliers of
+ * the best hypothesis, model[p][4] = (a, b, tx, ty) (zeros when there is none).
+ */
+void oracle_geometric(const int64_t* nn, int32_t n, int32_t m, int64_t P, const int32_t* n_q,
+                      const int32_t* m_r, const float* q_xy, const float* r_xy, float border,
+                      float qw, float qh, float rw, float rh, float thr, int32_t iters, uint64_t seed,
+                      uint32_t num, uint32_t den, int32_t* good, int32_t* inl, double* model) {
+#pragma omp parallel for schedule(dynamic, 1)
+  for (int64_t p = 0; p < P; ++p) {
+    const int32_t nq = n_q ? n_q[p] : n, mr = m_r ? m_r[p] : m;
+    double* Pp = (double*)malloc(sizeof(double) * 2 * (size_t)(nq > 0 ? nq : 1));
+    double* Qp = (double*)malloc(sizeof(double) * 2 * (size_t)(nq > 0 ? nq : 1));
+    int32_t M = 0;
+    for (int32_t j = 0; j < nq; ++j) {
+      const int64_t* o = nn + ((size_t)p * n + j) * 4;
+      if (!oracle_ratio_pass(o[0], o[2], mr, num, den)) continue;
+      const float* a = q_xy + ((size_t)p * n + j) * 2;
+      const float* b = r_xy + ((size_t)p * m + o[1]) * 2;
+      if (a[0] < border || a[1] < border || a[0] >= qw - border || a[1] >= qh - border) continue;
+      if (b[0] < border || b[1] < border || b[0] >= rw - border || b[1] >= rh - border) continue;
+      Pp[2 * M] = a[0]; Pp[2 * M + 1] = a[1];
+      Qp[2 * M] = b[0]; Qp[2 * M + 1] = b[1];
+      ++M;
+    }
+    const double thr2 = (double)thr * (double)thr;
+    int32_t best = 0;
+    double bm[4] = {0, 0, 0, 0};
+    if (M >= 2) {
+      best = -1;
+      const uint64_t h0 = geo_mix((seed << 32) + (uint64_t)p);
+      const int64_t H = iters > 0 ? iters : (int64_t)M * (M - 1) / 2;
+      int32_t u = 0, v = 1;
+      for (int64_t t = 0; t < H; ++t) {
+        if (iters > 0) {
+          const uint64_t h = geo_mix(h0 ^ (uint64_t)t);
+          u = (int32_t)(h % (uint64_t)M);
+          v = (int32_t)((h >> 32) % (uint64_t)(M - 1));
+          v += v >= u;
+        } else if (t > 0) {  /* exhaustive: (0,1), (0,2), ..., (0,M-1), (1,2), ... */
+          if (++v == M) { ++u; v = u + 1; }
+        }
+        double mm[4];
+        if (!geo_fit(Pp + 2 * u, Pp + 2 * v, Qp + 2 * u, Qp + 2 * v, mm)) continue;
+        const int32_t c = geo_inliers(Pp, Qp, M, mm, thr2);
+        if (c > best) { best = c; memcpy(bm, mm, sizeof(bm)); }
+      }
+      if (best < 0) best = 0;
+    }
+    good[p] = M;
+    inl[p] = best;
+    if (model) memcpy(model + 4 * p, bm, sizeof(bm));
+    free(Pp);
+    free(Qp);
+  }
+}

@@ -136,8 +136,9 @@ def _out_ptr(x, shape, dtype, device: int, what: str):
     would silently drop the results; a smaller or narrower buffer would be overrun): exact
     shape and dtype, C-contiguous and writable, and — for a CUDA tensor — on the index's device."""
     shape = tuple(int(v) for v in shape)
+    ok_dt = {_TORCH_DT[dtype]} | ({"torch.int32"} if dtype is np.uint32 else set())  # counts: 4-byte ints
     if _is_torch(x):
-        if tuple(x.shape) != shape or str(x.dtype) != _TORCH_DT[dtype]:
+        if tuple(x.shape) != shape or str(x.dtype) not in ok_dt:
             raise TypeError(f"{what}: got {tuple(x.shape)} {x.dtype}, expected {shape} {_TORCH_DT[dtype]}")
         if not x.is_contiguous():
             raise ValueError(f"{what}: tensor must be contiguous")
@@ -146,7 +147,7 @@ def _out_ptr(x, shape, dtype, device: int, what: str):
         return x.data_ptr()
     if not isinstance(x, np.ndarray):
         raise TypeError(f"{what}: expected a numpy array or torch tensor, got {type(x).__name__}")
-    if x.shape != shape or x.dtype != np.dtype(dtype):
+    if x.shape != shape or (x.dtype != np.dtype(dtype) and not (dtype is np.uint32 and x.dtype == np.int32)):
         raise TypeError(f"{what}: got {x.shape} {x.dtype}, expected {shape} {np.dtype(dtype)}")
     if not x.flags["C_CONTIGUOUS"] or not x.flags["WRITEABLE"]:
         raise ValueError(f"{what}: array must be C-contiguous and writable")

@@ -185,6 +185,24 @@ __device__ __forceinline__ void mma_piece_fold_ts(uint32_t tmem_d, uint32_t a_tm
       : "memory");
 }
 
+// Verify piece with A in TMEM: the four u8 x u8 K-steps (A = 8 TMEM columns per K-step), B from SMEM.
+__device__ __forceinline__ void mma_piece_ts(uint32_t tmem_d, uint32_t a_tmem, uint64_t bdesc, uint32_t bar) {
+  asm volatile(
+      "{\n\t.reg .pred e, f, t;\n\t.reg .b32 a1, a2, a3;\n\t.reg .b64 b1, b2, b3;\n\t"
+      "setp.ne.b32 f, 0, 0;\n\t"
+      "setp.eq.b32 t, 0, 0;\n\t"
+      "add.u32 a1, %1, 8;\n\tadd.u32 a2, %1, 16;\n\tadd.u32 a3, %1, 24;\n\t"
+      "add.s64 b1, %2, 2;\n\tadd.s64 b2, %2, 4;\n\tadd.s64 b3, %2, 6;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, f;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [a1], b1, %3, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [a2], b2, %3, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [a3], b3, %3, t;\n\t"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%4];\n\t}" ::"r"(tmem_d),
+      "r"(a_tmem), "l"(bdesc), "r"(kIdescI8), "r"(bar)
+      : "memory");
+}
+
 __device__ __forceinline__ void mma_commit(uint32_t bar) {
   asm volatile(
       "{\n\t.reg .pred e;\n\t"
@@ -453,7 +471,7 @@ __device__ __forceinline__ void exact_row_global(const MatchParams& p, int qi, i
 // columns >= m are padding for every reference (m = 384: the second chunk is half padding), so
 // those pieces are neither computed nor scanned (a chunk with fewer than 4 pieces leaves the
 // static buffer / phase schedule with odd use counts: use_parity() tracks the flips).
-__device__ __forceinline__ int piece_count_last(int m, int cpr) {
+__host__ __device__ __forceinline__ int piece_count_last(int m, int cpr) {
   return (m - (cpr - 1) * kBN + kPiece - 1) / kPiece;
 }
 // Phase flips of the two TMEM buffers after a chunk of np pieces (buffer pp & 1): buffer 0 is used
@@ -473,7 +491,10 @@ __device__ __forceinline__ uint32_t use_parity(int np) {
 // groups (3 epilogue warps per SMSP) hide each other's TMEM-load and barrier latency.
 // kFold: the search path (folded norms, no column keys in the scan, counts only);
 // otherwise the verify path (packed column keys, exact (d1, i1, d2, i2)).
-template <bool kFold>
+// kSkip: the last chunk of every reference has fewer than 4 pieces that can hold keypoints
+// (m mod 256 in 1..192): those pieces are skipped, with the buffer phases tracked at run time;
+// otherwise every chunk is 4 pieces and the schedule is fully static.
+template <bool kFold, bool kSkip>
 __global__ void __launch_bounds__(kNumThreads, 1)
     match_kernel(const __grid_constant__ CUtensorMap qmap, const __grid_constant__ CUtensorMap rmap,
                  const MatchParams p) {
@@ -503,16 +524,15 @@ __global__ void __launch_bounds__(kNumThreads, 1)
   if (threadIdx.x == 0) {
     prefetch_tmap(&qmap);
     prefetch_tmap(&rmap);
-    // query stages: search copies each tile to TMEM (freed by that copy); verify feeds the MMAs from
-    // shared memory (freed by the kNG MMA warps' commits)
-    for (int i = 0; i < kQStages; ++i) { mbar_init(qfull(i), 1); mbar_init(qempty(i), kFold ? 1 : kNG); }
+    // query stages: each tile is copied SMEM -> TMEM once (freed by that copy); the MMAs read A from TMEM
+    for (int i = 0; i < kQStages; ++i) { mbar_init(qfull(i), 1); mbar_init(qempty(i), 1); }
     for (int i = 0; i < kTQ; ++i) { mbar_init(tqfull(i), 1); mbar_init(tqempty(i), kNG); }
     mbar_init(axfull, 1);
     // reference slots: MMA operands + column keys read by every epilogue warp
     for (int i = 0; i < kMaxSlots; ++i) {
       mbar_init(rfull(i), 1);
       mbar_init(rempty(i), kNG + kEpiWarps);
-      mbar_init(xready(i), kEpiWarps);  // search: every epilogue warp wrote its share of the slot's digits
+      mbar_init(xready(i), 1);  // search: the producer warp expanded the slot's norm digits
     }
     for (int i = 0; i < kTmemBufs; ++i) { mbar_init(tfull(i), 1); mbar_init(tempty(i), 4); }
     fence_barrier_init();
@@ -530,173 +550,33 @@ __global__ void __launch_bounds__(kNumThreads, 1)
 
   PROF_DECL
   if (warp == kProducerWarp) {
-    // ===================== TMA producer =====================
-    if (lane == 0) {
-      if (kFold) {  // constant norm-term operand -> TMEM, once
-        tc_fence_after();
-        tmem_cp_128x256b(tmem_base + kAxCol, smem_desc_sw32(sbase + SmemPlan::kAx));
-        commit_one(axfull);
-      }
+    // ===================== TMA producer (lane 0) + norm-digit expansion (whole warp) =====================
+    if (kFold && lane == 0) {  // constant norm-term operand -> TMEM, once
+      tc_fence_after();
+      tmem_cp_128x256b(tmem_base + kAxCol, smem_desc_sw32(sbase + SmemPlan::kAx));
+      commit_one(axfull);
+    }
+    {
       uint32_t qctr = 0;
       uint32_t slot_par = 0;  // bit sl = phase parity of reference slot sl
       for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
         const Job J = decode_job(p, j);
         const int nslots = J.nr * cpr;
-        for (int sl = 0; sl < nslots; ++sl) {
-          PROF_B(); mbar_wait_sleep(rempty(sl), (slot_par >> sl & 1u) ^ 1); PROF_E(0);
-          mbar_expect_tx(rfull(sl), kRTileBytes + kColBytes);
-          const int s = sl / cpr, c = sl % cpr;
-          const int64_t ref = J.ref_first + s;
-          tma_load_3d(sbase + SmemPlan::kR + sl * kRTileBytes, &rmap, rfull(sl), 0, c * kBN,
-                      static_cast<int>(p.ref_map_base + ref));
-          bulk_load(sbase + SmemPlan::kCol + sl * kColBytes, p.colkey + (ref * cpr + c) * kColInts, kColBytes,
-                    rfull(sl));
-          slot_par ^= 1u << sl;
-        }
-        const int ntiles = J.nq * T;
-        if (kFold) {
-          // TMA tile t+1 into shared memory while tile t is copied to its TMEM slot (the MMAs read A
-          // from TMEM, so each query tile crosses the shared-memory port once, not once per piece)
-          auto issue = [&](int t) {
-            const uint32_t gq = qctr + t, st = gq % kQStages;
-            PROF_B(); mbar_wait_sleep(qempty(st), ((gq / kQStages) & 1) ^ 1); PROF_E(1);
-            mbar_expect_tx(qfull(st), kQTileBytes);
-            tma_load_3d(sbase + SmemPlan::kQ + st * kQTileBytes, &qmap, qfull(st), 0, (t % T) * kBM, J.q_first + t / T);
-          };
-          if (ntiles > 0) issue(0);
-          for (int t = 0; t < ntiles; ++t) {
-            if (t + 1 < ntiles) issue(t + 1);
-            const uint32_t gq = qctr + t, st = gq % kQStages, sl = gq % kTQ;
-            mbar_wait(qfull(st), (gq / kQStages) & 1);
-            mbar_wait_sleep(tqempty(sl), ((gq / kTQ) & 1) ^ 1);
-            tc_fence_after();
-            const uint64_t sd = smem_desc_sw128(sbase + SmemPlan::kQ + st * kQTileBytes);
-#pragma unroll
-            for (int k = 0; k < kDim / kXDim; ++k) tmem_cp_128x256b(tmem_base + kTQBase + sl * kQCols + 8 * k, sd + 2 * k);
-            commit_one(tqfull(sl));
-            commit_one(qempty(st));
-          }
-          qctr += ntiles;
-        } else {
-        for (int t = 0; t < ntiles; ++t, ++qctr) {
-          const int st = qctr % kQStages;
-          PROF_B(); mbar_wait_sleep(qempty(st), ((qctr / kQStages) & 1) ^ 1); PROF_E(1);
-          mbar_expect_tx(qfull(st), kQTileBytes);
-          tma_load_3d(sbase + SmemPlan::kQ + st * kQTileBytes, &qmap, qfull(st), 0, (t % T) * kBM, J.q_first + t / T);
-        }
-        }
-      }
-    }
-  } else if (warp < kFirstEpiWarp) {
-    // ===================== MMA issuers: warp mw serves epilogue group mw =====================
-    // Issuing tcgen05.mma costs the issuing SMSP throughput, so the kNG issuers sit on SMSPs 1-3.
-    // Warp mw issues the pieces of the units u with u % kNG == mw, in order, into its group's two
-    // 64-column buffers (whole warp, one elected lane).  Every warp commits the release of every
-    // query tile (waiting for tiles it never used, so the stage phases stay in order).
-    const int mw = warp - kFirstMmaWarp;
-    const int np_last = piece_count_last(p.m, cpr);
-    uint32_t ph_t = 0;  // bit b: phase flip of this group's TMEM buffer b (chunks with an odd use count)
-    uint32_t qctr = 0;
-    if (kFold) mbar_wait(axfull, 0);  // constant norm-term operand in TMEM
-    uint32_t slot_par = 0;  // bit sl = phase parity of reference slot sl
-    for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
-      const Job J = decode_job(p, j);
-      const int nslots = J.nr * cpr;
-      const int U = J.nq * T * J.nr;
-      uint32_t ready_mask = 0;
-      int waited = 0, t = 0, s = 0, g = 0;
-      for (int u = 0; u < U; ++u) {
-        if (g == mw) {
-          while (waited <= t) {
-            const uint32_t gq = qctr + waited;
-            PROF_B();
-            if (kFold) mbar_wait(tqfull(gq % kTQ), (gq / kTQ) & 1);
-            else mbar_wait(qfull(gq % kQStages), (gq / kQStages) & 1);
-            PROF_E(1);
-            ++waited;
-          }
-          const uint32_t st = (qctr + t) % kQStages;
-          const uint64_t ad = smem_desc_sw128(sbase + SmemPlan::kQ + st * kQTileBytes);
-          const uint32_t at = tmem_base + kTQBase + ((qctr + t) % kTQ) * kQCols;  // search: A in TMEM
-          for (int c = 0; c < cpr; ++c) {
-            const int sl = s * cpr + c;
-            if (!(ready_mask >> sl & 1u)) {
-              PROF_B(); mbar_wait(rfull(sl), (slot_par >> sl & 1u));
-              if (kFold) mbar_wait(xready(sl), (slot_par >> sl & 1u));  // norm digits expanded
-              PROF_E(2);
-              ready_mask |= 1u << sl;
-            }
-            const uint64_t bd0 = smem_desc_sw128(sbase + SmemPlan::kR + sl * kRTileBytes);
-            const int np = c == cpr - 1 ? np_last : kPiecesPerChunk;
-#pragma unroll
-            for (int pp = 0; pp < kPiecesPerChunk; ++pp) {  // static buffer / phase (see the epilogue)
-              if (pp >= np) break;  // all-padding pieces of the last chunk are never computed
-              const uint32_t buf = mw * kNB + (pp & 1);
-              PROF_B(); mbar_wait(tempty(buf), (((pp >> 1) ^ (ph_t >> (pp & 1))) & 1) ^ 1); PROF_E(0);
-              tc_fence_after();
-              // rows kPiece*pp.. of the chunk: SWIZZLE_128B core groups of 8 rows x 128 B
-              const uint64_t bd = bd0 + pp * (kPiece * kDim >> 4);
-#ifdef TID_NOMMA  // timing experiment only: no MMAs (the commit still signals the buffer)
-              if (kFold) mma_commit(tfull(buf)); else
-#endif
-              if (kFold)  // + norm-term K-step: rows kPiece*pp.. of the 32-B-wide tile
-                mma_piece_fold_ts(tmem_base + buf * kPiece, at, bd, tmem_base + kAxCol,
-                                  smem_desc_sw32(sbase + SmemPlan::kX + sl * kXTileBytes) + pp * (kPiece * kXDim >> 4),
-                                  tfull(buf));
-              else
-                mma_piece<kIdescI8>(tmem_base + buf * kPiece, ad, bd, tfull(buf));
-            }
-            ph_t ^= use_parity(np);
+        if (lane == 0) {
+          for (int sl = 0; sl < nslots; ++sl) {
+            PROF_B(); mbar_wait_sleep(rempty(sl), (slot_par >> sl & 1u) ^ 1); PROF_E(0);
+            mbar_expect_tx(rfull(sl), kRTileBytes + kColBytes);
+            const int s = sl / cpr, c = sl % cpr;
+            const int64_t ref = J.ref_first + s;
+            tma_load_3d(sbase + SmemPlan::kR + sl * kRTileBytes, &rmap, rfull(sl), 0, c * kBN,
+                        static_cast<int>(p.ref_map_base + ref));
+            bulk_load(sbase + SmemPlan::kCol + sl * kColBytes, p.colkey + (ref * cpr + c) * kColInts, kColBytes,
+                      rfull(sl));
           }
         }
-        if (s == J.nr - 1) {  // this warp's release of query tile t (covers all its prior MMAs)
-          const uint32_t gq = qctr + t;
-          if (waited <= t) {  // never touched tile t: still wait for it so the phase order holds
-            if (kFold) mbar_wait(tqfull(gq % kTQ), (gq / kTQ) & 1);
-            else mbar_wait(qfull(gq % kQStages), (gq / kQStages) & 1);
-            waited = t + 1;
-          }
-          mma_commit(kFold ? tqempty(gq % kTQ) : qempty(gq % kQStages));
-        }
-        if (++g == kNG) g = 0;
-        if (++s == J.nr) { s = 0; ++t; }
-      }
-      for (int sl = 0; sl < nslots; ++sl) {
-        if (!(ready_mask >> sl & 1u)) {  // keep rempty / xready phases ordered
-          mbar_wait(rfull(sl), (slot_par >> sl & 1u));
-          if (kFold) mbar_wait(xready(sl), (slot_par >> sl & 1u));
-        }
-        mma_commit(rempty(sl));
-        slot_par ^= 1u << sl;
-      }
-      qctr += J.nq * T;
-    }
-  } else {
-    // ===================== epilogue: TMEM -> registers -> top-2 -> ratio -> count =====================
-    // Each piece (64 columns) is fetched with one x64 TMEM load and its buffer released as soon
-    // as the load has landed, so the MMA of the group's next-but-one piece overlaps the scan; the
-    // 3 groups (3 epilogue warps per SMSP) hide each other's load latency.
-    const int ew = warp - kFirstEpiWarp;  // 0 .. 4*kNG-1
-    const int g = ew >> 2;                // group: units u with u % kNG == g
-    const int quarter = warp & 3;         // TMEM lanes 32*quarter .. +31 (hardware restriction)
-    const uint32_t taddr_q = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16);
-    const int row_in_tile = quarter * 32 + lane;
-    const int nq_ld = T * kBM;
-    const bool ratio32 = p.num2 <= 511u && p.den2 <= 511u;  // den^2 * d fits 32 bits (d <= 8,323,200)
-    uint32_t slot_par = 0;                // bit sl = phase parity of reference slot sl
-    const int np_last = piece_count_last(p.m, cpr);
-    uint32_t ph_t = 0;                    // bit b: phase flip of TMEM buffer b (see the MMA warps)
-    uint32_t v[64];
-
-    for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
-      const Job J = decode_job(p, j);
-      const int nslots = J.nr * cpr;
-      const int U = J.nq * T * J.nr;
-      // column keys of every slot of the job (also orders this warp's rempty arrivals)
-      PROF_B();
-      for (int sl = 0; sl < nslots; ++sl) mbar_wait(rfull(sl), slot_par >> sl & 1u);
-      if constexpr (kFold) {
-        // the fifth MMA K-step's B operand, expanded here from the column terms W (HBM keeps only W:
+        __syncwarp();
+        if constexpr (kFold) {
+        // the fifth MMA K-step's B operand, expanded by this warp from the column terms W (HBM keeps only W:
         // 4 B per keypoint instead of 32 B of digits).  Column i of a slot: 32 u8 digits of
         // E = floor(W / 2) against the constant operand a = (255 x 15, 1, 255 x 15, 1):
         // E = 255 * (sum of the 30 "255"-weighted digits) + d15 + d31, filled greedily (255, 255, ...,
@@ -704,7 +584,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         // 254 > max E = 1,048,576).  Padding columns (W < 0) get zero digits.  Both 16-byte halves of
         // the constant operand are equal, so the SWIZZLE_32B placement of a row's two halves does not
         // change the product: rows are written plainly, 32 B each.
-        for (int x = ew * 32 + lane; x < nslots * kBN; x += kEpiWarps * 32) {
+        for (int sl = 0; sl < nslots; ++sl) mbar_wait(rfull(sl), slot_par >> sl & 1u);  // column terms landed
+        for (int x = lane; x < nslots * kBN; x += 32) {
           const int sl = x / kBN, col = x % kBN;
           int W;
           asm volatile("ld.shared.s32 %0, [%1];" : "=r"(W) : "r"(sbase + SmemPlan::kCol + sl * kColBytes + col * 4));
@@ -740,6 +621,138 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         if (lane == 0)
           for (int sl = 0; sl < nslots; ++sl) mbar_arrive(xready(sl));
       }
+        slot_par ^= (1u << nslots) - 1u;
+        const int ntiles = J.nq * T;
+        if (lane == 0) {
+          // TMA tile t+1 into shared memory while tile t is copied to its TMEM slot (the MMAs read A
+          // from TMEM, so each query tile crosses the shared-memory port once, not once per piece)
+          auto issue = [&](int t) {
+            const uint32_t gq = qctr + t, st = gq % kQStages;
+            PROF_B(); mbar_wait_sleep(qempty(st), ((gq / kQStages) & 1) ^ 1); PROF_E(1);
+            mbar_expect_tx(qfull(st), kQTileBytes);
+            tma_load_3d(sbase + SmemPlan::kQ + st * kQTileBytes, &qmap, qfull(st), 0, (t % T) * kBM, J.q_first + t / T);
+          };
+          if (ntiles > 0) issue(0);
+          for (int t = 0; t < ntiles; ++t) {
+            if (t + 1 < ntiles) issue(t + 1);
+            const uint32_t gq = qctr + t, st = gq % kQStages, sl = gq % kTQ;
+            mbar_wait(qfull(st), (gq / kQStages) & 1);
+            mbar_wait_sleep(tqempty(sl), ((gq / kTQ) & 1) ^ 1);
+            tc_fence_after();
+            const uint64_t sd = smem_desc_sw128(sbase + SmemPlan::kQ + st * kQTileBytes);
+#pragma unroll
+            for (int k = 0; k < kDim / kXDim; ++k) tmem_cp_128x256b(tmem_base + kTQBase + sl * kQCols + 8 * k, sd + 2 * k);
+            commit_one(tqfull(sl));
+            commit_one(qempty(st));
+          }
+          qctr += ntiles;
+        }
+      }
+    }
+  } else if (warp < kFirstEpiWarp) {
+    // ===================== MMA issuers: warp mw serves epilogue group mw =====================
+    // Issuing tcgen05.mma costs the issuing SMSP throughput, so the kNG issuers sit on SMSPs 1-3.
+    // Warp mw issues the pieces of the units u with u % kNG == mw, in order, into its group's two
+    // 64-column buffers (whole warp, one elected lane).  Every warp commits the release of every
+    // query tile (waiting for tiles it never used, so the stage phases stay in order).
+    const int mw = warp - kFirstMmaWarp;
+    const int np_last = kSkip ? piece_count_last(p.m, cpr) : kPiecesPerChunk;
+    uint32_t ph_t = 0;  // bit b: phase flip of this group's TMEM buffer b (chunks with an odd use count)
+    uint32_t qctr = 0;
+    if (kFold) mbar_wait(axfull, 0);  // constant norm-term operand in TMEM
+    uint32_t slot_par = 0;  // bit sl = phase parity of reference slot sl
+    for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
+      const Job J = decode_job(p, j);
+      const int nslots = J.nr * cpr;
+      const int U = J.nq * T * J.nr;
+      uint32_t ready_mask = 0;
+      int waited = 0, t = 0, s = 0, g = 0;
+      for (int u = 0; u < U; ++u) {
+        if (g == mw) {
+          while (waited <= t) {
+            const uint32_t gq = qctr + waited;
+            PROF_B();
+            mbar_wait(tqfull(gq % kTQ), (gq / kTQ) & 1);
+            PROF_E(1);
+            ++waited;
+          }
+          const uint32_t at = tmem_base + kTQBase + ((qctr + t) % kTQ) * kQCols;  // A (query tile) in TMEM
+          for (int c = 0; c < cpr; ++c) {
+            const int sl = s * cpr + c;
+            if (!(ready_mask >> sl & 1u)) {
+              PROF_B(); mbar_wait(rfull(sl), (slot_par >> sl & 1u));
+              if (kFold) mbar_wait(xready(sl), (slot_par >> sl & 1u));  // norm digits expanded
+              PROF_E(2);
+              ready_mask |= 1u << sl;
+            }
+            const uint64_t bd0 = smem_desc_sw128(sbase + SmemPlan::kR + sl * kRTileBytes);
+            const int np = c == cpr - 1 ? np_last : kPiecesPerChunk;
+#pragma unroll
+            for (int pp = 0; pp < kPiecesPerChunk; ++pp) {  // static buffer / phase (see the epilogue)
+              if (kSkip && pp >= np) break;  // all-padding pieces of the last chunk are never computed
+              const uint32_t buf = mw * kNB + (pp & 1);
+              PROF_B(); mbar_wait(tempty(buf), (((pp >> 1) ^ (ph_t >> (pp & 1))) & 1) ^ 1); PROF_E(0);
+              tc_fence_after();
+              // rows kPiece*pp.. of the chunk: SWIZZLE_128B core groups of 8 rows x 128 B
+              const uint64_t bd = bd0 + pp * (kPiece * kDim >> 4);
+#ifdef TID_NOMMA  // timing experiment only: no MMAs (the commit still signals the buffer)
+              if (kFold) mma_commit(tfull(buf)); else
+#endif
+              if (kFold)  // + norm-term K-step: rows kPiece*pp.. of the 32-B-wide tile
+                mma_piece_fold_ts(tmem_base + buf * kPiece, at, bd, tmem_base + kAxCol,
+                                  smem_desc_sw32(sbase + SmemPlan::kX + sl * kXTileBytes) + pp * (kPiece * kXDim >> 4),
+                                  tfull(buf));
+              else
+                mma_piece_ts(tmem_base + buf * kPiece, at, bd, tfull(buf));
+            }
+            if (kSkip) ph_t ^= use_parity(np);
+          }
+        }
+        if (s == J.nr - 1) {  // this warp's release of query tile t (covers all its prior MMAs)
+          const uint32_t gq = qctr + t;
+          if (waited <= t) {  // never touched tile t: still wait for it so the phase order holds
+            mbar_wait(tqfull(gq % kTQ), (gq / kTQ) & 1);
+            waited = t + 1;
+          }
+          mma_commit(tqempty(gq % kTQ));
+        }
+        if (++g == kNG) g = 0;
+        if (++s == J.nr) { s = 0; ++t; }
+      }
+      for (int sl = 0; sl < nslots; ++sl) {
+        if (!(ready_mask >> sl & 1u)) {  // keep rempty / xready phases ordered
+          mbar_wait(rfull(sl), (slot_par >> sl & 1u));
+          if (kFold) mbar_wait(xready(sl), (slot_par >> sl & 1u));
+        }
+        mma_commit(rempty(sl));
+        slot_par ^= 1u << sl;
+      }
+      qctr += J.nq * T;
+    }
+  } else {
+    // ===================== epilogue: TMEM -> registers -> top-2 -> ratio -> count =====================
+    // Each piece (64 columns) is fetched with one x64 TMEM load and its buffer released as soon
+    // as the load has landed, so the MMA of the group's next-but-one piece overlaps the scan; the
+    // 3 groups (3 epilogue warps per SMSP) hide each other's load latency.
+    const int ew = warp - kFirstEpiWarp;  // 0 .. 4*kNG-1
+    const int g = ew >> 2;                // group: units u with u % kNG == g
+    const int quarter = warp & 3;         // TMEM lanes 32*quarter .. +31 (hardware restriction)
+    const uint32_t taddr_q = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16);
+    const int row_in_tile = quarter * 32 + lane;
+    const int nq_ld = T * kBM;
+    const bool ratio32 = p.num2 <= 511u && p.den2 <= 511u;  // den^2 * d fits 32 bits (d <= 8,323,200)
+    uint32_t slot_par = 0;                // bit sl = phase parity of reference slot sl
+    const int np_last = kSkip ? piece_count_last(p.m, cpr) : kPiecesPerChunk;
+    uint32_t ph_t = 0;                    // bit b: phase flip of TMEM buffer b (see the MMA warps)
+    uint32_t v[64];
+
+    for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
+      const Job J = decode_job(p, j);
+      const int nslots = J.nr * cpr;
+      const int U = J.nq * T * J.nr;
+      // column keys of every slot of the job (also orders this warp's rempty arrivals)
+      PROF_B();
+      for (int sl = 0; sl < nslots; ++sl) mbar_wait(rfull(sl), slot_par >> sl & 1u);
       PROF_E(4);
       // own units u = g, g + kNG, ...; unit u = (tile t = u / nr, reference s = u % nr), and
       // t = (query qi - q_first) * T + tq.  Tracked incrementally (no divisions per unit).
@@ -771,7 +784,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             const int np = c == cpr - 1 ? np_last : kPiecesPerChunk;
 #pragma unroll
             for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
-              if (pp >= np) break;  // all-padding pieces (m not a multiple of 64 x 4) are not computed
+              if (kSkip && pp >= np) break;  // all-padding pieces (m not a multiple of 64 x 4) are not computed
               const uint32_t buf = g * kNB + (pp & 1);
               PROF_B(); mbar_wait(tfull(buf), ((pp >> 1) ^ (ph_t >> (pp & 1))) & 1); PROF_E(0);
               tc_fence_after();
@@ -784,7 +797,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               __syncwarp();
               if (lane == 0) mbar_arrive(tempty(buf));
               PROF_B();
-              if (kpc >= kBN) {  // full chunk (the common case): no masking
+              if (kpc >= (pp + 1) * kPiece) {  // every column of the piece is real (the common case)
 #ifndef TID_NOSCAN
                 scan32_fold<false>(v, 32, R, T1, T2);
                 scan32_fold<false>(v + 32, 32, R, T1, T2);
@@ -795,7 +808,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               }
               PROF_E(1);
             }
-            ph_t ^= use_parity(np);
+            if (kSkip) ph_t ^= use_parity(np);
             PROF_B();
             int x1, x2;
             finish_fold(R, T1, T2, x1, x2);
@@ -848,7 +861,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           const int np = c == cpr - 1 ? np_last : kPiecesPerChunk;
 #pragma unroll
           for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
-            if (pp >= np) break;
+            if (kSkip && pp >= np) break;
             const uint32_t buf = g * kNB + (pp & 1);
             PROF_B(); mbar_wait(tfull(buf), ((pp >> 1) ^ (ph_t >> (pp & 1))) & 1); PROF_E(0);
             tc_fence_after();
@@ -869,7 +882,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               PROF_E(1);
             }
           }
-          ph_t ^= use_parity(np);
+          if (kSkip) ph_t ^= use_parity(np);
           PROF_B();
           int k1, k2;
           finish_partition(R, T1, T2, k1, k2);
@@ -955,18 +968,18 @@ cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CU
   int dev = 0;
   cudaGetDevice(&dev);
   if (dev >= 64 || !(attr_set >> dev & 1)) {
-    cudaError_t e = cudaFuncSetAttribute(match_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         static_cast<int>(SmemPlan::kAlloc));
-    if (e != cudaSuccess) return e;
-    e = cudaFuncSetAttribute(match_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             static_cast<int>(SmemPlan::kAlloc));
-    if (e != cudaSuccess) return e;
+    for (auto k : {match_kernel<true, false>, match_kernel<true, true>, match_kernel<false, false>,
+                   match_kernel<false, true>}) {
+      cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                           static_cast<int>(SmemPlan::kAlloc));
+      if (e != cudaSuccess) return e;
+    }
     if (dev < 64) attr_set |= uint64_t(1) << dev;
   }
-  if (fold)
-    match_kernel<true><<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, p);
-  else
-    match_kernel<false><<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, p);
+  const bool skip = piece_count_last(p.m, p.cpr) < kPiecesPerChunk;
+  auto kern = fold ? (skip ? match_kernel<true, true> : match_kernel<true, false>)
+                   : (skip ? match_kernel<false, true> : match_kernel<false, false>);
+  kern<<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, p);
   return cudaGetLastError();
 }
 

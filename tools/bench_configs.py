@@ -20,25 +20,34 @@ sys.path.insert(0, ROOT)
 
 import tidgen  # noqa: E402
 import paper_conf_icpp_wangzll21_b200 as tid  # noqa: E402
+from bench import ClockSampler  # noqa: E402  (nvidia-smi clocks during each timed region)
 
 
 def log(*a):
     print(*a, file=sys.stderr, flush=True)
 
 
+LAST_CLOCKS = {}
+
+
 def timed(fn, reps, warm=3):
+    """CUDA-event times (ms) of `reps` calls after `warm` untimed ones; nvidia-smi clocks sampled
+    during the timed calls land in LAST_CLOCKS (added to every JSON record)."""
     import torch
     for _ in range(warm):
         fn()
     torch.cuda.synchronize()
     ts = []
-    for _ in range(reps):
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record()
-        fn()
-        e1.record()
-        e1.synchronize()
-        ts.append(e0.elapsed_time(e1))
+    with ClockSampler(torch.cuda.current_device()) as clk:
+        for _ in range(reps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            fn()
+            e1.record()
+            e1.synchronize()
+            ts.append(e0.elapsed_time(e1))
+    LAST_CLOCKS.clear()
+    LAST_CLOCKS.update(clk.summary())
     return ts
 
 
@@ -75,7 +84,8 @@ def search_case(name, B, n, R, m, k, reps, hbm_budget=0, host_budget=0, chunk=0)
            "e2e_p50_ms": statistics.median(ts_e2e), "e2e_comparisons_per_s": B * R / (statistics.median(ts_e2e) / 1e3),
            "match_kernel_ms_per_search": st["match_ms"] / reps if st["match_launches"] else None,
            "h2d_GBps": (st["h2d_bytes"] / (sum(ts) / 1e3) / 1e9) if st["h2d_bytes"] else 0.0,
-           "planted_top1": top1, "info": idx.info()}
+           "planted_top1": top1, "info": idx.info(), "clocks": dict(LAST_CLOCKS),
+           "tensor_tops_int8": 2.0 * B * R * n * m * 128 / (p50 / 1e3) / 1e12}
     idx.close()
     print(json.dumps(out), flush=True)
     return out
@@ -93,7 +103,8 @@ def verify_case(P=4096, n=1000, m=1000, reps=10):
     c = cnt.cpu().numpy()
     out = {"case": "C2 verify", "pairs": P, "query_kp": n, "ref_kp": m, "p50_ms": statistics.median(ts),
            "comparisons_per_s": P / (statistics.median(ts) / 1e3), "p50_ms_with_nn": statistics.median(ts_nn),
-           "positives_mean_count": float(c[pos].mean()), "negatives_mean_count": float(c[~pos].mean())}
+           "positives_mean_count": float(c[pos].mean()), "negatives_mean_count": float(c[~pos].mean()),
+           "tensor_tops_int8": 2.0 * P * n * m * 128 / (statistics.median(ts) / 1e3) / 1e12, "clocks": dict(LAST_CLOCKS)}
     idx.close()
     print(json.dumps(out), flush=True)
 
@@ -136,6 +147,12 @@ def main():
     if "sweep" in what:
         for B in (1, 8, 64, 256):
             search_case(f"sweep B={B}", B, 1000, 100_000, 256, 5, reps=5 if B >= 64 else 20)
+    if "table7" in what:
+        # B200 analogue of the speed half of Table 7: reference budget m
+        # and query budget n at B = 256
+        for m, n in ((768, 768), (512, 768), (384, 768), (256, 768), (384, 1024), (384, 512), (384, 384)):
+            R = int(os.environ.get("T7_REFS", "30000"))
+            search_case(f"table7 m={m} n={n}", 256, n, R, m, 5, reps=3)
     if "host" in what:
         R = int(os.environ.get("HOST_REFS", "1000000"))
         rb = 256 * 128
