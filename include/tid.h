@@ -175,6 +175,43 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
                       uint32_t* counts_out, int32_t* nn_out, void* stream);
 
 /*
+ * Post-match verification: one-to-one verification followed by the
+ * paper's outlier removal, "the geometric verification is performed to remove the outliers that
+ * may be mismatched" (§3.1) and "edge feature removing" (§4.1).  The paper
+ * defines neither step; the readings (R14-R16) are:
+ *   edge-feature removal: a good match (ratio test passed) is dropped when its query keypoint or
+ *     its nearest reference keypoint lies within `border` px of its image's edge (x < border,
+ *     y < border, x >= width - border or y >= height - border);
+ *   geometric verification: a 2-D similarity X = a x - b y + tx, Y = b x + a y + ty from query to
+ *     reference coordinates, fitted exactly to 2 matches per hypothesis; a match is an inlier
+ *     when its squared reprojection error is < inlier_px^2; RANSAC over `iterations` hypotheses
+ *     drawn with a counter-based generator (splitmix64 of seed, pair index and hypothesis
+ *     index), or every pair of matches when iterations == 0; the best hypothesis has the most
+ *     inliers, ties to the earliest.  Matches are taken in query-keypoint order.  Geometry is
+ *     IEEE fp64 with every operation rounded separately, so results are deterministic.
+ * Arguments as tid_verify, plus:
+ *   q_xy : float [P][n][2] query keypoint (x, y) in pixels; r_xy : float [P][m][2] (host or device).
+ *   counts_out  (nullable) uint32 [P]: ratio-test matches (= tid_verify's counts);
+ *   good_out    uint32 [P]: matches left after edge-feature removal;
+ *   inliers_out uint32 [P]: inliers of the best hypothesis (0 when fewer than 2 matches remain);
+ *   model_out   (nullable) double [P][4]: (a, b, tx, ty) of the best hypothesis (zeros if none).
+ * Errors: TID_EINVAL (null pointers, inlier_px <= 0, border < 0, iterations < 0, as tid_verify).
+ */
+typedef struct {
+  float border;                      /* edge margin in pixels (0 = only points outside the image)   */
+  float query_width, query_height;   /* query image extent in pixels                                  */
+  float ref_width, ref_height;       /* reference image extent in pixels                              */
+  float inlier_px;                   /* inlier threshold on the reprojection distance, pixels (> 0)  */
+  int32_t iterations;                /* RANSAC hypotheses; 0 = exhaustive over all match pairs        */
+  uint64_t seed;                     /* generator seed                                                */
+} tid_geom_params;
+
+tid_status tid_verify_geometric(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t* r, int32_t m,
+                                int64_t P, const int32_t* n_q, const int32_t* m_r, const float* q_xy,
+                                const float* r_xy, const tid_geom_params* params, uint32_t* counts_out,
+                                uint32_t* good_out, uint32_t* inliers_out, double* model_out, void* stream);
+
+/*
  * Shard merge: merge G ranked lists per query into one.
  *   ids_in/counts_in : [G][B][k] (int64 / int32), host or device, each list in rank order.
  *   ids_out/counts_out : [B][k] in (count desc, id asc) order.

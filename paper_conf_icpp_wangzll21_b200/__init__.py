@@ -26,7 +26,8 @@ STATUS = {0: "TID_OK", -1: "TID_EINVAL", -2: "TID_ENOMEM", -3: "TID_ECUDA", -4: 
 EXPORTS = ("tid_index_create", "tid_index_destroy", "tid_add_references", "tid_search", "tid_search_counts",
            "tid_verify", "tid_merge_topk", "tid_nccl_unique_id", "tid_get_info", "tid_profile", "tid_get_stats",
            "tid_set_tuning", "tid_delete_references", "tid_update_references", "tid_index_save", "tid_index_load",
-           "tid_f16_prepare", "tid_f16_search_counts", "tid_host_tier_map", "tid_last_error")
+           "tid_f16_prepare", "tid_f16_search_counts", "tid_host_tier_map", "tid_verify_geometric",
+           "tid_last_error")
 
 
 class TidError(RuntimeError):
@@ -54,6 +55,12 @@ class Info(ctypes.Structure):
 class Stats(ctypes.Structure):
     _fields_ = [("match_launches", ctypes.c_int64), ("match_ms", ctypes.c_double),
                 ("kernel_launches", ctypes.c_int64), ("h2d_bytes", ctypes.c_int64), ("d2h_bytes", ctypes.c_int64)]
+
+
+class GeomParams(ctypes.Structure):
+    _fields_ = [("border", ctypes.c_float), ("query_width", ctypes.c_float), ("query_height", ctypes.c_float),
+                ("ref_width", ctypes.c_float), ("ref_height", ctypes.c_float), ("inlier_px", ctypes.c_float),
+                ("iterations", ctypes.c_int32), ("seed", ctypes.c_uint64)]
 
 
 class Tuning(ctypes.Structure):
@@ -94,6 +101,7 @@ def load_library(path: str = LIB_PATH):
     lib.tid_f16_prepare.argtypes = [vp, vp, i64, i32, ctypes.c_float, vp, vp]
     lib.tid_f16_search_counts.argtypes = [vp, vp, i32, i64, vp, i32, i64, vp, vp]
     lib.tid_host_tier_map.argtypes = [vp, i64, P(ctypes.POINTER(ctypes.c_uint8)), P(i64)]
+    lib.tid_verify_geometric.argtypes = [vp, vp, i32, vp, i32, i64, vp, vp, vp, vp, P(GeomParams), vp, vp, vp, vp, vp]
     lib.tid_last_error.restype = ctypes.c_char_p
     for name in EXPORTS[:-1]:
         getattr(lib, name).restype = ctypes.c_int
@@ -321,6 +329,30 @@ class Index:
         np_ = None if nn is None else _out_ptr(nn, (P, n, 4), np.int32, self.device, "nn")
         _check(self._lib.tid_verify(self._h, qp, n, rp, m, P, nqp, mrp, cp, np_, _stream(q, r, counts)))
         return counts, nn
+
+    def verify_geometric(self, q, r, q_xy, r_xy, *, border=0.0, query_size=(1e9, 1e9), ref_size=(1e9, 1e9),
+                         inlier_px=3.0, iterations=256, seed=2021, n_q=None, m_r=None, want_model=True):
+        """Row f4: verify pairs (q, r) like ``verify`` then edge-feature removal + 2-point similarity
+        RANSAC on the keypoint coordinates q_xy float [P][n][2], r_xy float [P][m][2].
+        Returns (counts, good, inliers) uint32 [P] and the model float64 [P][4] (a, b, tx, ty)."""
+        P, n, _ = _shape(q)
+        P2, m, _ = _shape(r)
+        assert P == P2
+        qp, k1 = _ptr(q, np.uint8)
+        rp, k2 = _ptr(r, np.uint8)
+        nqp, k3 = _ptr(n_q, np.int32)
+        mrp, k4 = _ptr(m_r, np.int32)
+        qx, k5 = _ptr(q_xy, np.float32)
+        rx, k6 = _ptr(r_xy, np.float32)
+        if _shape(q_xy) != (P, n, 2) or _shape(r_xy) != (P, m, 2):
+            raise ValueError("q_xy must be [P][n][2] and r_xy [P][m][2]")
+        gp = GeomParams(border, query_size[0], query_size[1], ref_size[0], ref_size[1], inlier_px, iterations, seed)
+        counts, good, inl = np.empty(P, np.uint32), np.empty(P, np.uint32), np.empty(P, np.uint32)
+        model = np.empty((P, 4), np.float64) if want_model else None
+        _check(self._lib.tid_verify_geometric(self._h, qp, n, rp, m, P, nqp, mrp, qx, rx, ctypes.byref(gp),
+                                              counts.ctypes.data, good.ctypes.data, inl.ctypes.data,
+                                              None if model is None else model.ctypes.data, _stream(q, r)))
+        return counts, good, inl, model
 
     def merge_topk(self, ids, counts):
         """ids int64 / counts int32 [G][B][k] (each list ranked) -> merged [B][k]."""

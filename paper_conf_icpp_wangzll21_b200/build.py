@@ -9,7 +9,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libtid.so")
-SOURCES = [os.path.join(CSRC, f) for f in ("tid_api.cu", "tid_kernels.cu", "tid_f16.cu")]
+SOURCES = [os.path.join(CSRC, f) for f in ("tid_api.cu", "tid_kernels.cu", "tid_f16.cu", "tid_geom.cu")]
 DEPS = SOURCES + [os.path.join(CSRC, "tid_kernels.cuh"), os.path.join(ROOT, "include", "tid.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",

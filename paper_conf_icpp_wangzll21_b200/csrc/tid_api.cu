@@ -285,6 +285,7 @@ struct tid_index {
   DevBuf stage_desc[2], stage_colkey[2], stage_kp[2];
   DevBuf ws_qs;                   // shifted queries q' = q ^ 0x80 (search)
   DevBuf ws_rtot;                 // collective reference count (all-reduce)
+  DevBuf ws_geo_nn, ws_geo_cnt, ws_geo_xy, ws_geo_out;  // f4 post-match verification
   int64_t* h_rtot = nullptr;      // pinned host copy of it
   DevBuf ws_f16q, ws_f16r, ws_f16nq, ws_f16nr, ws_f16in;  // f1 float path
   int64_t host_chunk = 0;
@@ -790,7 +791,8 @@ tid_status tid_index_destroy(tid_index* idx) {
   DevBuf* bufs[] = {&idx->ws_q, &idx->ws_nq, &idx->ws_nvalid, &idx->ws_counts, &idx->ws_cand, &idx->ws_keys,
                     &idx->ws_gather, &idx->ws_ids, &idx->ws_cnts, &idx->ws_r, &idx->ws_colkey, &idx->ws_nn,
                     &idx->ws_kp, &idx->ws_mr, &idx->stage_desc[0], &idx->stage_desc[1], &idx->stage_colkey[0],
-                    &idx->stage_colkey[1], &idx->stage_kp[0], &idx->stage_kp[1], &idx->ws_qs, &idx->ws_f16q, &idx->ws_f16r, &idx->ws_f16nq,
+                    &idx->stage_colkey[1], &idx->stage_kp[0], &idx->stage_kp[1], &idx->ws_qs, &idx->ws_geo_nn, &idx->ws_geo_cnt,
+                    &idx->ws_geo_xy, &idx->ws_geo_out, &idx->ws_f16q, &idx->ws_f16r, &idx->ws_f16nq,
                     &idx->ws_f16nr, &idx->ws_f16in};
   for (DevBuf* b : bufs) b->release();
   for (auto& pr : idx->prof_ev) { cudaEventDestroy(pr.first); cudaEventDestroy(pr.second); }
@@ -1369,6 +1371,73 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
   bool host_out = false;
   if (!dev_counts) TRY(copy_out(idx, counts_out, counts, static_cast<size_t>(P) * 4, s, &host_out));
   if (nn_out && !dev_nn) TRY(copy_out(idx, nn_out, nn, static_cast<size_t>(P) * n * 16, s, &host_out));
+  if (host_out) CU(cudaStreamSynchronize(s));
+  CU(cudaGetLastError());
+  return TID_OK;
+}
+
+tid_status tid_verify_geometric(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t* r, int32_t m, int64_t P,
+                                const int32_t* n_q, const int32_t* m_r, const float* q_xy, const float* r_xy,
+                                const tid_geom_params* gp, uint32_t* counts_out, uint32_t* good_out,
+                                uint32_t* inliers_out, double* model_out, void* stream) {
+  if (!idx) return fail(TID_EINVAL, "null index");
+  if (!q_xy || !r_xy || !gp || !good_out || !inliers_out) return fail(TID_EINVAL, "null argument");
+  if (!(gp->inlier_px > 0.0f) || !(gp->border >= 0.0f)) return fail(TID_EINVAL, "inlier_px must be > 0, border >= 0");
+  if (gp->iterations < 0) return fail(TID_EINVAL, "iterations < 0");
+  if (P < 1 || P > (1LL << 31) - 1 || n < 1 || m < 2) return fail(TID_EINVAL, "bad P / n / m");
+  TRY(set_device(idx));
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  CallGuard guard(idx, s);
+  // 1) one-to-one verification (a3-a5): exact (d1, i1, d2, i2) of every query row, into the workspace
+  TRY(idx->ws_geo_nn.ensure(static_cast<size_t>(P) * n * 16, "geometric nn"));
+  TRY(idx->ws_geo_cnt.ensure(static_cast<size_t>(P) * 4 * 4, "geometric counts"));
+  uint32_t* dcnt = idx->ws_geo_cnt.as<uint32_t>();
+  uint32_t* dgood = dcnt + P;
+  uint32_t* dinl = dcnt + 2 * P;
+  TRY(tid_verify(idx, q, n, r, m, P, n_q, m_r, dcnt, idx->ws_geo_nn.as<int32_t>(), s));
+  // 2) coordinates and per-pair counts on the device
+  const size_t qb = static_cast<size_t>(P) * n * 8, rb = static_cast<size_t>(P) * m * 8;
+  TRY(idx->ws_geo_xy.ensure(qb + rb + static_cast<size_t>(P) * 8 + 64, "keypoint coordinates"));
+  float* dq = idx->ws_geo_xy.as<float>();
+  float* dr = reinterpret_cast<float*>(idx->ws_geo_xy.as<uint8_t>() + qb);
+  TRY(copy_in(idx, dq, q_xy, qb, s));
+  TRY(copy_in(idx, dr, r_xy, rb, s));
+  const int32_t* dnq = nullptr;
+  const int32_t* dmr = nullptr;
+  int32_t* dvalid = reinterpret_cast<int32_t*>(idx->ws_geo_xy.as<uint8_t>() + qb + rb);
+  if (n_q) {
+    TRY(copy_in(idx, dvalid, n_q, static_cast<size_t>(P) * 4, s));
+    dnq = dvalid;
+  }
+  if (m_r) {
+    TRY(copy_in(idx, dvalid + P, m_r, static_cast<size_t>(P) * 4, s));
+    dmr = dvalid + P;
+  }
+  // 3) edge-feature removal + RANSAC per pair (f4)
+  GeomParams g{};
+  g.border = gp->border;
+  g.qw = gp->query_width;
+  g.qh = gp->query_height;
+  g.rw = gp->ref_width;
+  g.rh = gp->ref_height;
+  g.thr = gp->inlier_px;
+  g.iters = gp->iterations;
+  g.seed = gp->seed;
+  g.num2 = idx->cfg.ratio_num * idx->cfg.ratio_num;
+  g.den2 = idx->cfg.ratio_den * idx->cfg.ratio_den;
+  double* dmodel = nullptr;
+  const bool dev_model = model_out && is_device_ptr(model_out);
+  if (model_out) {
+    TRY(idx->ws_geo_out.ensure(static_cast<size_t>(P) * 32, "geometric models"));
+    dmodel = dev_model ? model_out : idx->ws_geo_out.as<double>();
+  }
+  CU(launch_geometric(idx->ws_geo_nn.as<int32_t>(), n, m, P, dnq, dmr, dq, dr, g, dgood, dinl, dmodel, s));
+  count_kernel(idx);
+  bool host_out = false;
+  if (counts_out) TRY(copy_out(idx, counts_out, dcnt, static_cast<size_t>(P) * 4, s, &host_out));
+  TRY(copy_out(idx, good_out, dgood, static_cast<size_t>(P) * 4, s, &host_out));
+  TRY(copy_out(idx, inliers_out, dinl, static_cast<size_t>(P) * 4, s, &host_out));
+  if (model_out && !dev_model) TRY(copy_out(idx, model_out, dmodel, static_cast<size_t>(P) * 32, s, &host_out));
   if (host_out) CU(cudaStreamSynchronize(s));
   CU(cudaGetLastError());
   return TID_OK;

@@ -123,6 +123,19 @@ void launch_merge(const uint64_t* cand, int32_t L, int64_t B, int32_t k, int64_t
 void launch_pack_lists(const int64_t* ids, const int32_t* counts, int64_t n, uint64_t* keys, cudaStream_t s);
 size_t match_smem_bytes();
 
+// f4 post-match verification (tid_geom.cu): edge-feature removal + 2-point similarity RANSAC
+struct GeomParams {
+  float border, qw, qh, rw, rh;  // edge margin (px) and the query / reference image extents
+  float thr;                     // inlier threshold on the reprojection distance (px)
+  int32_t iters;                 // hypotheses; <= 0: every pair (exhaustive)
+  uint64_t seed;
+  uint32_t num2, den2;           // ratio test den2 * d1 < num2 * d2
+};
+// nn [P][n][4] int32 (d1, i1, d2, i2) from the verify kernel; coordinates [P][n][2] / [P][m][2] float.
+cudaError_t launch_geometric(const int32_t* nn, int32_t n, int32_t m, int64_t P, const int32_t* n_q,
+                             const int32_t* m_r, const float* q_xy, const float* r_xy, const GeomParams& g,
+                             uint32_t* good, uint32_t* inl, double* model, cudaStream_t s);
+
 // f1 float path (tid_f16.cu)
 size_t f16_smem_bytes();
 cudaError_t launch_f16_prepare(const uint8_t* sift, int64_t rows, int32_t rootsift, float scale, void* out,

@@ -1,4 +1,5 @@
-"""Run one search with a -DTID_PROF build of libtid and print the per-role cycle buckets."""
+"""Run one search (or, with `verify` as the first argument, one C2 verification of 4,096 pairs
+n = m = 1000) with a -DTID_PROF build of libtid (TID_LIB=...) and print the per-role cycle buckets."""
 import ctypes
 import os
 import sys
@@ -9,14 +10,21 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import tidgen  # noqa: E402
 import paper_conf_icpp_wangzll21_b200 as tid  # noqa: E402
 
-R, B, n, m = int(sys.argv[1]) if len(sys.argv) > 1 else 20000, 256, 1000, 256
-refs, _ = tidgen.refs(0, R, m)
-qs, _ = tidgen.queries(0, B, n, R_total=R, m=m)
-idx = tid.Index(ref_kp=m)
-idx.add_references(refs)
-idx.search(qs, 5)
-idx.profile(True)
-idx.search(qs, 5)
+if len(sys.argv) > 1 and sys.argv[1] == "verify":
+    Q, Rr, _ = tidgen.pairs(4096, 1000, 1000)
+    idx = tid.Index(ref_kp=256, query_kp_max=1000)
+    idx.verify(Q, Rr, want_nn=False)
+    idx.profile(True)
+    idx.verify(Q, Rr, want_nn=False)
+else:
+    R, B, n, m = int(sys.argv[1]) if len(sys.argv) > 1 else 20000, 256, 1000, 256
+    refs, _ = tidgen.refs(0, R, m)
+    qs, _ = tidgen.queries(0, B, n, R_total=R, m=m)
+    idx = tid.Index(ref_kp=m)
+    idx.add_references(refs)
+    idx.search(qs, 5)
+    idx.profile(True)
+    idx.search(qs, 5)
 st = idx.stats()
 lib = tid.load_library()
 buf = np.zeros(148 * 32 * 8, np.uint64)
