@@ -74,7 +74,16 @@ typedef struct {
   int32_t  cache_policy;       /* 0 = fill: HBM first, then the host tier (ids in insertion order);
                                   1 = FIFO (§6.1): every new batch enters HBM and the
                                   oldest batches are swapped out to the host tier when HBM is full */
-  int32_t  reserved;
+  int32_t  descriptor;         /* 0 = u8 SIFT, exact integer path (default);
+                                  1 = the paper's float path (SURVEY row f1, §4.2, §5.1
+                                  P:555-576): u8 SIFT given to add/search is converted on the GPU
+                                  to [RootSIFT] x f16_scale in fp16 and stored that way (2 B per
+                                  value + 8 KiB of norm terms per reference); matching on
+                                  tcgen05.mma.kind::f16 (see tid_f16_search_counts for the
+                                  arithmetic and the +-1 count acceptance).  ref_kp <= 256;
+                                  save / load and tid_verify stay on the u8 path.              */
+  float    f16_scale;          /* descriptor 1: scale factor before the fp16 conversion (0 = 1)  */
+  int32_t  f16_rootsift;       /* descriptor 1: 1 = RootSIFT (L1-normalise, sqrt) first          */
 } tid_config;
 
 /* Create an index on cfg->device.  Allocates the HBM arena lazily (on first add).
@@ -108,7 +117,8 @@ tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t
  * rather than pageable host memory, Table 5): appends `count` references that live in
  * the host tier and returns, in *desc_out, a pointer to their pinned storage
  * u8 [count][ref_kp][128] (initialised to zeros = references that match nothing), which the
- * caller fills in place — no staging copy.  Every reference has ref_kp keypoints.  Contents are
+ * caller fills in place — no staging copy (descriptor 1: fp16 [count][ref_kp][128] values,
+ * already RootSIFT / scaled).  Every reference has ref_kp keypoints.  Contents are
  * read when a search streams the tier, so they must be written before the next search; the
  * pointer stays valid until tid_index_destroy.  first_local_id as in tid_add_references.
  * Errors: TID_EINVAL (count < 1, null desc_out), TID_ENOMEM (host budget exceeded),

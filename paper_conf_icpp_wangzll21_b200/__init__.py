@@ -41,7 +41,8 @@ class Config(ctypes.Structure):
                 ("query_kp_max", ctypes.c_int32), ("ratio_num", ctypes.c_uint32), ("ratio_den", ctypes.c_uint32),
                 ("hbm_budget_bytes", ctypes.c_uint64), ("host_budget_bytes", ctypes.c_uint64),
                 ("id_base", ctypes.c_int64), ("rank", ctypes.c_int32), ("world_size", ctypes.c_int32),
-                ("nccl_unique_id", ctypes.c_void_p), ("cache_policy", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("nccl_unique_id", ctypes.c_void_p), ("cache_policy", ctypes.c_int32), ("descriptor", ctypes.c_int32),
+                ("f16_scale", ctypes.c_float), ("f16_rootsift", ctypes.c_int32)]
 
 
 class Info(ctypes.Structure):
@@ -186,13 +187,18 @@ class Index:
 
     def __init__(self, ref_kp: int = 256, query_kp_max: int = 1024, ratio=(4, 5), device: int = 0,
                  hbm_budget_bytes: int = 0, host_budget_bytes: int = 0, id_base: int = 0, rank: int = 0,
-                 world_size: int = 1, nccl_id: bytes | None = None, cache_policy: str = "fill"):
+                 world_size: int = 1, nccl_id: bytes | None = None, cache_policy: str = "fill",
+                 descriptor: str = "u8", f16_scale: float = 1.0, f16_rootsift: bool = True):
+        """descriptor "u8": exact integer path; "f16": the float path (RootSIFT / scaled SIFT stored
+        in fp16, tcgen05 kind::f16) — add/search still take u8 SIFT, converted on the GPU."""
         self._lib = load_library()
         self._id_buf = ctypes.create_string_buffer(nccl_id, 128) if nccl_id is not None else None
         cfg = Config(device, 128, ref_kp, query_kp_max, ratio[0], ratio[1], hbm_budget_bytes, host_budget_bytes,
                      id_base, rank, world_size,
                      ctypes.cast(self._id_buf, ctypes.c_void_p) if self._id_buf is not None else None,
-                     {"fill": 0, "fifo": 1}[cache_policy], 0)
+                     {"fill": 0, "fifo": 1}[cache_policy], {"u8": 0, "f16": 1}[descriptor], f16_scale,
+                     1 if f16_rootsift else 0)
+        self.descriptor = descriptor
         h = ctypes.c_void_p()
         _check(self._lib.tid_index_create(ctypes.byref(cfg), ctypes.byref(h)))
         self._h = h
@@ -234,7 +240,10 @@ class Index:
         ptr = ctypes.POINTER(ctypes.c_uint8)()
         first = ctypes.c_int64()
         _check(self._lib.tid_host_tier_map(self._h, count, ctypes.byref(ptr), ctypes.byref(first)))
-        view = np.ctypeslib.as_array(ptr, shape=(count, self.ref_kp, 128))
+        if self.descriptor == "f16":  # fp16 values [count][ref_kp][128]
+            view = np.ctypeslib.as_array(ptr, shape=(count, self.ref_kp, 256)).view(np.float16)
+        else:
+            view = np.ctypeslib.as_array(ptr, shape=(count, self.ref_kp, 128))
         return first.value, view
 
     def delete(self, local_ids):

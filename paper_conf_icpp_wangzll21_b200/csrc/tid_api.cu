@@ -8,6 +8,7 @@
 #include <dlfcn.h>
 
 #include <algorithm>
+#include <cmath>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
@@ -254,6 +255,7 @@ struct Segment {
   bool on_host = false;
   uint8_t* desc = nullptr;    // [cap][m][128]: device (HBM) or pinned host
   int32_t* colkey = nullptr;  // device, HBM segments only: [cap][cpr][256] column terms W (search)
+  uint16_t* xop = nullptr;    // device, HBM segments of a float (f1) index: [cap][256][16] fp16 norm terms
   int64_t cap = 0, count = 0, first = 0;
   std::vector<int32_t> kp;    // keypoint count per reference (0 = deleted / empty)
 };
@@ -265,7 +267,11 @@ struct tid_index {
   int device = 0;
   int num_sms = 148;
   int cpr = 1;                    // chunks per reference = ceil(ref_kp / 256)
-  int64_t ref_bytes = 0;          // bytes per stored reference
+  bool f16 = false;               // descriptor 1: the float path (RootSIFT / scaled SIFT in fp16, row f1)
+  float f16_c = 0.0f, f16_scale = 1.0f;  // the index's norm-term constant C and the fp16 scale factor
+  int32_t f16_rootsift = 1;
+  int64_t ref_bytes = 0;          // bytes per stored reference (u8, or fp16 for a float index)
+  int64_t in_bytes = 0;           // bytes per reference of the caller's u8 input (ref_kp * 128)
   int64_t hbm_ref_bytes = 0;      // HBM bytes per resident reference (descriptors + norm digits + column terms)
   uint64_t hbm_budget = 0, host_budget = 0;
   std::vector<Segment> segs;      // id order; HBM and host segments may interleave (FIFO policy)
@@ -286,6 +292,7 @@ struct tid_index {
   DevBuf ws_qs;                   // shifted queries q' = q ^ 0x80 (search)
   DevBuf ws_rtot;                 // collective reference count (all-reduce)
   DevBuf ws_geo_nn, ws_geo_cnt, ws_geo_xy, ws_geo_out;  // f4 post-match verification
+  DevBuf ws_u8, ws_f16c, ws_f16kp, ws_f16rows, stage_xop[2];  // f1 index: conversion staging, C, xop inputs
   int64_t* h_rtot = nullptr;      // pinned host copy of it
   DevBuf ws_f16q, ws_f16r, ws_f16nq, ws_f16nr, ws_f16in;  // f1 float path
   int64_t host_chunk = 0;
@@ -413,6 +420,9 @@ tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const ui
   return TID_OK;
 }
 
+tid_status f16_norm_terms(tid_index* idx, const void* refs16, int64_t count, const int32_t* kp_dev, uint16_t* xop,
+                          cudaStream_t s);
+
 // A run of consecutive local ids [first, first + cnt) inside one segment (offset `off`), inside one
 // count window.  Host-tier pieces are at most host_chunk references (one staging buffer).
 struct Piece {
@@ -450,12 +460,50 @@ tid_status run_pass(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, in
                     uint32_t* counts, cudaStream_t s, OnWindow on_window) {
   const int T = static_cast<int>(ceil_div(n, kBM));
   const int64_t R = idx->n_hbm + idx->n_host;
-  TRY(idx->ws_nq.ensure(static_cast<size_t>(B) * T * kBM * 4, "query norms"));
-  TRY(idx->ws_qs.ensure(static_cast<size_t>(B) * n * kDim, "shifted queries"));
-  launch_query_prep(dq, B, n, T, idx->ws_nq.as<int32_t>(), idx->ws_qs.as<uint8_t>(), s);
-  count_kernel(idx);
   CUtensorMap qmap;
-  TRY(make_map(&qmap, idx->ws_qs.p, B, n, kBM));
+  if (idx->f16) {  // row f1: queries -> [RootSIFT] x scale -> fp16, fp32 squared norms N_Q
+    TRY(idx->ws_f16q.ensure(static_cast<size_t>(B) * n * kDim * 2, "f16 queries"));
+    TRY(idx->ws_f16nq.ensure(static_cast<size_t>(B) * T * kBM * 4, "f16 query norms"));
+    CU(launch_f16_prepare(dq, B * n, idx->f16_rootsift, idx->f16_scale, idx->ws_f16q.p, s));
+    CU(launch_f16_norms(idx->ws_f16q.p, B, n, T * kBM, 0.0f, idx->ws_f16nq.as<float>(), s));
+    count_kernel(idx, 2);
+    TRY(make_map_f16(&qmap, idx->ws_f16q.p, B, n, kBM));
+  } else {
+    TRY(idx->ws_nq.ensure(static_cast<size_t>(B) * T * kBM * 4, "query norms"));
+    TRY(idx->ws_qs.ensure(static_cast<size_t>(B) * n * kDim, "shifted queries"));
+    launch_query_prep(dq, B, n, T, idx->ws_nq.as<int32_t>(), idx->ws_qs.as<uint8_t>(), s);
+    count_kernel(idx);
+    TRY(make_map(&qmap, idx->ws_qs.p, B, n, kBM));
+  }
+  // row f1: one kind::f16 match launch over `cnt` references starting at map index `base`
+  auto launch_f16 = [&](const void* rbase, const void* xbase, int64_t map_count, int64_t base, int64_t cnt,
+                        int64_t col0) -> tid_status {
+    CUtensorMap rmap, xmap;
+    TRY(make_map_f16(&rmap, rbase, map_count, idx->cfg.ref_kp, kBN));
+    TRY(make_xmap(&xmap, xbase, map_count, kBN));
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    if (idx->prof) {
+      if (idx->prof_used == idx->prof_ev.size()) {
+        cudaEvent_t a, b;
+        CU(cudaEventCreate(&a));
+        CU(cudaEventCreate(&b));
+        idx->prof_ev.push_back({a, b});
+      }
+      e0 = idx->prof_ev[idx->prof_used].first;
+      e1 = idx->prof_ev[idx->prof_used].second;
+      ++idx->prof_used;
+      CU(cudaEventRecord(e0, s));
+    }
+    CU(launch_f16_match(qmap, rmap, xmap, idx->ws_f16c.as<float>(), idx->ws_f16nq.as<float>(), static_cast<int32_t>(B),
+                        n, T, cnt, idx->cfg.ratio_num * idx->cfg.ratio_num, idx->cfg.ratio_den * idx->cfg.ratio_den,
+                        counts, idx->num_sms, s, W, col0, base, nvalid));
+    if (idx->prof) {
+      CU(cudaEventRecord(e1, s));
+      idx->stats.match_launches++;
+      count_kernel(idx);
+    }
+    return TID_OK;
+  };
   const std::vector<Piece> pieces = plan_pieces(idx, W);
   std::vector<int64_t> next_host(pieces.size() + 1, -1);  // index of the next host piece after i
   for (int64_t i = static_cast<int64_t>(pieces.size()) - 1, nh = -1; i >= 0; --i) {
@@ -470,7 +518,10 @@ tid_status run_pass(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, in
   if (first_host >= 0) {
     for (int b = 0; b < 2; ++b) {
       TRY(idx->stage_desc[b].ensure(static_cast<size_t>(chunk * rb), "host-tier staging"));
-      TRY(idx->stage_colkey[b].ensure(static_cast<size_t>(chunk) * idx->cpr * kColBytes, "staging keys"));
+      if (idx->f16)
+        TRY(idx->stage_xop[b].ensure(static_cast<size_t>(chunk) * kBN * 16 * 2, "staging norm terms"));
+      else
+        TRY(idx->stage_colkey[b].ensure(static_cast<size_t>(chunk) * idx->cpr * kColBytes, "staging keys"));
       TRY(idx->stage_kp[b].ensure(static_cast<size_t>(chunk) * 4, "staging kp"));
     }
     // the copy stream must not overwrite staging buffers still read by a previous call
@@ -504,6 +555,15 @@ tid_status run_pass(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, in
       const int b = host_buf[i];
       if (next_host[i] >= 0) TRY(issue_copy(next_host[i]));  // prefetch the next chunk while this one computes
       CU(cudaStreamWaitEvent(s, idx->ev_h2d[b], 0));
+      if (idx->f16) {
+        TRY(f16_norm_terms(idx, idx->stage_desc[b].p, pc.cnt, idx->stage_kp[b].as<int32_t>(),
+                           idx->stage_xop[b].as<uint16_t>(), s));
+        count_kernel(idx, 2);
+        TRY(launch_f16(idx->stage_desc[b].p, idx->stage_xop[b].p, chunk, 0, pc.cnt, pc.first - w0));
+        CU(cudaEventRecord(idx->ev_free[b], s));
+        if (i + 1 == pieces.size() || pieces[i + 1].win != pc.win) TRY(on_window(w0, std::min(W, R - w0)));
+        continue;
+      }
       RefPrepParams rp{};
       rp.desc = idx->stage_desc[b].as<uint8_t>();
       rp.src = nullptr;
@@ -518,6 +578,8 @@ tid_status run_pass(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, in
       TRY(launch_search_range(idx, qmap, idx->stage_desc[b].as<uint8_t>(), chunk, 0, rp.colkey, pc.cnt, B,
                               n, T, nvalid, counts, W, pc.first - w0, s));
       CU(cudaEventRecord(idx->ev_free[b], s));
+    } else if (idx->f16) {
+      TRY(launch_f16(pc.sg->desc, pc.sg->xop, pc.sg->cap, pc.off, pc.cnt, pc.first - w0));
     } else {
       TRY(launch_search_range(idx, qmap, pc.sg->desc, pc.sg->cap, pc.off,
                               pc.sg->colkey + pc.off * idx->cpr * kColInts, pc.cnt, B, n, T, nvalid, counts, W,
@@ -570,11 +632,14 @@ tid_status alloc_segment(tid_index* idx, bool on_host, int64_t cap, Segment* out
     idx->host_alloc += cap * rb;
   } else {
     cudaError_t e1 = cudaMalloc(&sg.desc, static_cast<size_t>(cap * rb));
-    cudaError_t e2 = e1 == cudaSuccess ? cudaMalloc(&sg.colkey, static_cast<size_t>(cap) * idx->cpr * kColBytes) : e1;
+    cudaError_t e2 = e1 != cudaSuccess ? e1
+                     : idx->f16 ? cudaMalloc(&sg.xop, static_cast<size_t>(cap) * kBN * 16 * 2)
+                                : cudaMalloc(&sg.colkey, static_cast<size_t>(cap) * idx->cpr * kColBytes);
     if (e1 != cudaSuccess || e2 != cudaSuccess) {
       cudaGetLastError();
       if (sg.desc) cudaFree(sg.desc);
       if (sg.colkey) cudaFree(sg.colkey);
+      if (sg.xop) cudaFree(sg.xop);
       return fail(TID_ENOMEM, "HBM arena allocation of %lld references failed", static_cast<long long>(cap));
     }
     idx->hbm_alloc += cap * idx->hbm_ref_bytes;
@@ -590,17 +655,50 @@ void free_segment(tid_index* idx, Segment& sg) {
   } else {
     if (sg.desc) cudaFree(sg.desc);
     if (sg.colkey) cudaFree(sg.colkey);
+    if (sg.xop) cudaFree(sg.xop);
     idx->hbm_alloc -= sg.cap * idx->hbm_ref_bytes;
   }
   sg.desc = nullptr;
   sg.colkey = nullptr;
+  sg.xop = nullptr;
 }
 
 // Ingest `take` references (host or device `src`, kp_host per reference) into HBM segment sg at
 // position `pos`: copy, zero padding rows, N_R -> packed column keys (Alg. 1 step 1).
+// Float index (descriptor 1): u8 SIFT rows (host or device) -> [RootSIFT] x scale -> fp16 at dst
+// (device), on the legacy stream.  Unaligned or host input goes through the u8 staging buffer.
+tid_status convert_f16(tid_index* idx, const uint8_t* src, bool src_dev, int64_t count, void* dst) {
+  const size_t ib = static_cast<size_t>(count) * idx->in_bytes;
+  const uint8_t* din = src;
+  if (!src_dev || reinterpret_cast<uintptr_t>(src) % 16) {
+    TRY(idx->ws_u8.ensure(ib, "u8 staging"));
+    CU(cudaMemcpy(idx->ws_u8.p, src, ib, cudaMemcpyDefault));
+    din = idx->ws_u8.as<uint8_t>();
+  }
+  CU(launch_f16_prepare(din, count * idx->cfg.ref_kp, idx->f16_rootsift, idx->f16_scale, dst, nullptr));
+  return TID_OK;
+}
+
+// Float index: norm-term rows (fixed C, per-reference keypoint counts) of `count` stored fp16 references.
+tid_status f16_norm_terms(tid_index* idx, const void* refs16, int64_t count, const int32_t* kp_dev, uint16_t* xop,
+                          cudaStream_t s) {
+  TRY(idx->ws_f16rows.ensure(static_cast<size_t>(count) * idx->cfg.ref_kp * 4, "f16 reference norms"));
+  CU(launch_f16_xop_fixed(refs16, count, idx->cfg.ref_kp, kp_dev, idx->f16_c, idx->ws_f16rows.as<float>(), xop, s));
+  return TID_OK;
+}
+
 tid_status ingest_hbm(tid_index* idx, Segment& sg, int64_t pos, const uint8_t* src, bool src_dev,
                       const int32_t* kp_host, int64_t take) {
   const int64_t rb = idx->ref_bytes;
+  if (idx->f16) {  // row f1: convert on the GPU, then the norm terms with the index's constant C
+    TRY(convert_f16(idx, src, src_dev, take, sg.desc + pos * rb));
+    TRY(idx->ws_kp.ensure(static_cast<size_t>(take) * 4, "kp staging"));
+    CU(cudaMemcpy(idx->ws_kp.p, kp_host, static_cast<size_t>(take) * 4, cudaMemcpyHostToDevice));
+    TRY(f16_norm_terms(idx, sg.desc + pos * rb, take, idx->ws_kp.as<int32_t>(),
+                       sg.xop + static_cast<size_t>(pos) * kBN * 16, nullptr));
+    CU(cudaStreamSynchronize(nullptr));
+    return TID_OK;
+  }
   uint8_t* dst = sg.desc + pos * rb;
   RefPrepParams rp{};
   rp.desc = dst;
@@ -725,6 +823,10 @@ tid_status tid_index_create(const tid_config* cfg, tid_index** out) {
     return fail(TID_EINVAL, "rank %d / world_size %d invalid", cfg->rank, cfg->world_size);
   if (cfg->world_size > 1 && !cfg->nccl_unique_id) return fail(TID_EINVAL, "world_size > 1 needs nccl_unique_id");
   if (cfg->id_base < 0) return fail(TID_EINVAL, "id_base must be >= 0");
+  if (cfg->descriptor != 0 && cfg->descriptor != 1) return fail(TID_EINVAL, "descriptor must be 0 (u8) or 1 (fp16)");
+  if (cfg->descriptor == 1 && cfg->ref_kp > kBN)
+    return fail(TID_EINVAL, "descriptor 1 (float path): ref_kp=%d > 256", cfg->ref_kp);
+  if (cfg->descriptor == 1 && !(cfg->f16_scale >= 0.0f)) return fail(TID_EINVAL, "f16_scale must be >= 0");
 
   int ndev = 0;
   CU(cudaGetDeviceCount(&ndev));
@@ -742,8 +844,24 @@ tid_status tid_index_create(const tid_config* cfg, tid_index** out) {
   idx->device = cfg->device;
   idx->num_sms = prop.multiProcessorCount;
   idx->cpr = static_cast<int>(ceil_div(cfg->ref_kp, kBN));
-  idx->ref_bytes = static_cast<int64_t>(cfg->ref_kp) * kDim;
+  idx->in_bytes = static_cast<int64_t>(cfg->ref_kp) * kDim;
+  idx->ref_bytes = idx->in_bytes;
   idx->hbm_ref_bytes = idx->ref_bytes + static_cast<int64_t>(idx->cpr) * kColBytes;
+  if (cfg->descriptor == 1) {  // row f1: fp16 storage + 256 x 16 fp16 norm terms per reference
+    idx->f16 = true;
+    idx->f16_scale = cfg->f16_scale > 0.0f ? cfg->f16_scale : 1.0f;
+    idx->f16_rootsift = cfg->f16_rootsift ? 1 : 0;
+    idx->ref_bytes = 2 * idx->in_bytes;
+    idx->hbm_ref_bytes = idx->ref_bytes + static_cast<int64_t>(kBN) * 16 * 2;
+    // C: the smallest power of two >= half the largest N_R the index can hold, so X = C + q.r - N_R/2
+    // >= 0 for every reference: RootSIFT rows have unit norm (x (1 + 2^-11)^2 after
+    // fp16 rounding), raw SIFT at most 128 * 255^2; both times scale^2.
+    const double s2 = static_cast<double>(idx->f16_scale) * idx->f16_scale;
+    const double bound = (idx->f16_rootsift ? 1.0 + 1.0 / 512 : 128.0 * 255 * 255) * s2 / 2;
+    int e = 0;
+    std::frexp(bound, &e);
+    idx->f16_c = static_cast<float>(std::ldexp(1.0, e));
+  }
   size_t free_b = 0, total_b = 0;
   cudaMemGetInfo(&free_b, &total_b);
   const uint64_t reserve = 8ull << 30;
@@ -763,6 +881,13 @@ tid_status tid_index_create(const tid_config* cfg, tid_index** out) {
   if (e != cudaSuccess) {
     tid_index_destroy(idx);
     return fail(TID_ECUDA, "stream/event creation: %s", cudaGetErrorString(e));
+  }
+  if (idx->f16) {
+    if (idx->ws_f16c.ensure(4, "f16 constant") != TID_OK ||
+        cudaMemcpy(idx->ws_f16c.p, &idx->f16_c, 4, cudaMemcpyHostToDevice) != cudaSuccess) {
+      tid_index_destroy(idx);
+      return fail(TID_ENOMEM, "f16 constant allocation failed");
+    }
   }
   if (cfg->world_size > 1 || cfg->nccl_unique_id) {  // a 1-rank communicator exercises the same path
     ncclUniqueId id;
@@ -792,6 +917,7 @@ tid_status tid_index_destroy(tid_index* idx) {
                     &idx->ws_gather, &idx->ws_ids, &idx->ws_cnts, &idx->ws_r, &idx->ws_colkey, &idx->ws_nn,
                     &idx->ws_kp, &idx->ws_mr, &idx->stage_desc[0], &idx->stage_desc[1], &idx->stage_colkey[0],
                     &idx->stage_colkey[1], &idx->stage_kp[0], &idx->stage_kp[1], &idx->ws_qs, &idx->ws_geo_nn, &idx->ws_geo_cnt,
+                    &idx->ws_u8, &idx->ws_f16c, &idx->ws_f16kp, &idx->ws_f16rows, &idx->stage_xop[0], &idx->stage_xop[1],
                     &idx->ws_geo_xy, &idx->ws_geo_out, &idx->ws_f16q, &idx->ws_f16r, &idx->ws_f16nq,
                     &idx->ws_f16nr, &idx->ws_f16in};
   for (DevBuf* b : bufs) b->release();
@@ -898,7 +1024,7 @@ tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t
       sg = &idx->segs.back();
     }
     const int64_t take = std::min(to_hbm - done, sg->cap - sg->count);
-    TRY_TX(ingest_hbm(idx, *sg, sg->count, desc + done * rb, dev_in, kp.data() + done, take));
+    TRY_TX(ingest_hbm(idx, *sg, sg->count, desc + done * idx->in_bytes, dev_in, kp.data() + done, take));
     sg->kp.insert(sg->kp.end(), kp.begin() + done, kp.begin() + done + take);
     sg->count += take;
     idx->n_hbm += take;
@@ -919,9 +1045,20 @@ tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t
       sg = &idx->segs.back();
     }
     const int64_t take = std::min(to_host - hdone, sg->cap - sg->count);
-    if (cudaMemcpy(sg->desc + sg->count * rb, desc + (to_hbm + hdone) * rb, static_cast<size_t>(take * rb),
-                   cudaMemcpyDefault) != cudaSuccess)
+    if (idx->f16) {  // convert on the GPU, then into the pinned tier (fp16)
+      for (int64_t o = 0; o < take;) {
+        const int64_t c = std::min<int64_t>(take - o, 8192);
+        TRY_TX(idx->ws_f16r.ensure(static_cast<size_t>(c * rb), "f16 conversion"));
+        TRY_TX(convert_f16(idx, desc + (to_hbm + hdone + o) * idx->in_bytes, dev_in, c, idx->ws_f16r.p));
+        if (cudaMemcpy(sg->desc + (sg->count + o) * rb, idx->ws_f16r.p, static_cast<size_t>(c * rb),
+                       cudaMemcpyDeviceToHost) != cudaSuccess)
+          return rollback(fail(TID_ECUDA, "host-tier copy: %s", cudaGetErrorString(cudaGetLastError())));
+        o += c;
+      }
+    } else if (cudaMemcpy(sg->desc + sg->count * rb, desc + (to_hbm + hdone) * rb, static_cast<size_t>(take * rb),
+                          cudaMemcpyDefault) != cudaSuccess) {
       return rollback(fail(TID_ECUDA, "host-tier copy: %s", cudaGetErrorString(cudaGetLastError())));
+    }
     sg->kp.insert(sg->kp.end(), kp.begin() + to_hbm + hdone, kp.begin() + to_hbm + hdone + take);
     sg->count += take;
     idx->n_host += take;
@@ -976,7 +1113,13 @@ tid_status tid_delete_references(tid_index* idx, const int64_t* local_ids, int64
     int64_t off;
     Segment* sg = find_segment(idx, id, &off);
     sg->kp[off] = 0;  // no keypoints: every column becomes padding -> count 0
-    if (!sg->on_host) {
+    if (!sg->on_host && idx->f16) {
+      TRY(idx->ws_kp.ensure(4, "kp"));
+      CU(cudaMemcpy(idx->ws_kp.p, &zero, 4, cudaMemcpyHostToDevice));
+      TRY(f16_norm_terms(idx, sg->desc + off * idx->ref_bytes, 1, idx->ws_kp.as<int32_t>(),
+                         sg->xop + static_cast<size_t>(off) * kBN * 16, nullptr));
+      CU(cudaStreamSynchronize(nullptr));
+    } else if (!sg->on_host) {
       RefPrepParams rp{};
       rp.desc = sg->desc + off * idx->ref_bytes;
       rp.src = nullptr;
@@ -1018,10 +1161,14 @@ tid_status tid_update_references(tid_index* idx, const int64_t* local_ids, const
   for (int64_t i = 0; i < count; ++i) {
     int64_t off;
     Segment* sg = find_segment(idx, ids[i], &off);
-    if (sg->on_host) {
+    if (sg->on_host && idx->f16) {
+      TRY(idx->ws_f16r.ensure(static_cast<size_t>(rb), "f16 conversion"));
+      TRY(convert_f16(idx, desc + i * idx->in_bytes, dev_in, 1, idx->ws_f16r.p));
+      CU(cudaMemcpy(sg->desc + off * rb, idx->ws_f16r.p, static_cast<size_t>(rb), cudaMemcpyDeviceToHost));
+    } else if (sg->on_host) {
       CU(cudaMemcpy(sg->desc + off * rb, desc + i * rb, static_cast<size_t>(rb), cudaMemcpyDefault));
     } else {
-      TRY(ingest_hbm(idx, *sg, off, desc + i * rb, dev_in, &kp[i], 1));
+      TRY(ingest_hbm(idx, *sg, off, desc + i * idx->in_bytes, dev_in, &kp[i], 1));
     }
     sg->kp[off] = kp[i];
     idx->dead[static_cast<size_t>(ids[i])] = 0;
@@ -1035,6 +1182,7 @@ tid_status tid_update_references(tid_index* idx, const int64_t* local_ids, const
 tid_status tid_index_save(const tid_index* cidx, const char* path) {
   tid_index* idx = const_cast<tid_index*>(cidx);
   if (!idx || !path) return fail(TID_EINVAL, "null argument");
+  if (idx->f16) return fail(TID_EUNSUPPORTED, "save: float (descriptor 1) indexes are not persisted");
   TRY(set_device(idx));
   CU(cudaEventSynchronize(idx->ev_last));
   FILE* f = fopen(path, "wb");
@@ -1070,6 +1218,7 @@ tid_status tid_index_save(const tid_index* cidx, const char* path) {
 
 tid_status tid_index_load(tid_index* idx, const char* path, int64_t* first_local_id) {
   if (!idx || !path) return fail(TID_EINVAL, "null argument");
+  if (idx->f16) return fail(TID_EUNSUPPORTED, "load: float (descriptor 1) indexes are not persisted");
   FILE* f = fopen(path, "rb");
   if (!f) return fail(TID_EINVAL, "cannot open %s", path);
   char magic[4];

@@ -195,7 +195,8 @@ __global__ void __launch_bounds__(kThreads, 1)
     match_f16_kernel(const __grid_constant__ CUtensorMap qmap, const __grid_constant__ CUtensorMap rmap,
                      const __grid_constant__ CUtensorMap xmap, const float* __restrict__ cterm,
                      const float* __restrict__ nq_all, int32_t B, int32_t n, int32_t T, int64_t R, int32_t q_per_job,
-                     uint32_t num2, uint32_t den2, uint32_t* __restrict__ counts) {
+                     uint32_t num2, uint32_t den2, uint32_t* __restrict__ counts, int64_t ldc, int64_t col0,
+                     int64_t rbase, const int32_t* __restrict__ n_valid) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const uint32_t sb = su32(smem);
@@ -242,9 +243,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int q0 = static_cast<int>(j % qchunks) * q_per_job, nq = min(q_per_job, B - q0);
         bar_wait(rempty, (rc & 1) ^ 1);
         bar_expect(rfull, 2 * kRHalf + kXTile);
-        tma3(sb + Plan::kR, &rmap, rfull, 0, 0, static_cast<int>(r));
-        tma3(sb + Plan::kR + kRHalf, &rmap, rfull, 64, 0, static_cast<int>(r));
-        tma3(sb + Plan::kX, &xmap, rfull, 0, 0, static_cast<int>(r));
+        tma3(sb + Plan::kR, &rmap, rfull, 0, 0, static_cast<int>(rbase + r));
+        tma3(sb + Plan::kR + kRHalf, &rmap, rfull, 64, 0, static_cast<int>(rbase + r));
+        tma3(sb + Plan::kX, &xmap, rfull, 0, 0, static_cast<int>(rbase + r));
         for (int t = 0; t < nq * T; ++t, ++qc) {
           const int st = qc % kStages;
           bar_wait(qempty(st), ((qc / kStages) & 1) ^ 1);
@@ -301,9 +302,10 @@ __global__ void __launch_bounds__(kThreads, 1)
       bar_wait(rfull, rc & 1);
       uint32_t cnt = 0;
       int qi = q0, tt = 0;  // query and tile of unit t (no divisions per unit)
+      int nv = n_valid ? min(n_valid[qi], n) : n;
       for (int t = 0; t < nq * T; ++t, ++uc) {
         const int row = tt * kBM + row_in_tile;
-        const bool valid = row < n;
+        const bool valid = row < nv;
         const float nqv = nq_all[static_cast<int64_t>(qi) * T * kBM + row];
         int Rm[16];
 #pragma unroll
@@ -354,10 +356,11 @@ __global__ void __launch_bounds__(kThreads, 1)
         const bool pass = valid && x2 >= 0 && double(den2) * d1 < double(num2) * d2;
         cnt += __popc(__ballot_sync(0xffffffffu, pass) & 0x33333333u);  // one thread per row
         if (++tt == T) {
-          if (lane == 0 && cnt) atomicAdd(counts + static_cast<int64_t>(qi) * R + r, cnt);
+          if (lane == 0 && cnt) atomicAdd(counts + static_cast<int64_t>(qi) * ldc + col0 + r, cnt);
           cnt = 0;
           tt = 0;
           ++qi;
+          if (t + 1 < nq * T) nv = n_valid ? min(n_valid[qi], n) : n;
         }
       }
       __syncwarp();
@@ -401,27 +404,34 @@ __global__ void nr_rows_kernel(const __half* __restrict__ x, int64_t rows, float
   float mx = row < rows ? acc : 0.0f;
 #pragma unroll
   for (int o = 8; o < 32; o <<= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
-  if ((threadIdx.x & 31) == 0) atomicMax(max_bits, __float_as_uint(mx));
+  if ((threadIdx.x & 31) == 0 && max_bits) atomicMax(max_bits, __float_as_uint(mx));
 }
 
 // Norm-term rows [R][256][16] fp16: (h1, h2, h3, 0 ...) with h1 + h2 + h3 = C - N_R / 2 (three
 // fp16 terms of the fp32 value, 33 significant bits), C = smallest power of two >= max N_R / 2;
 // rows >= m: h1 = -inf.  Also writes C.  One thread per row (32 contiguous bytes out).
+// fixed_c > 0: the index's constant (a bound on every N_R / 2 it can hold) instead of
+// the launch's maximum; kp (nullable): rows >= kp[ref] are padding (h1 = -inf) like rows >= m.
 __global__ void xop_kernel(const float* __restrict__ nr, int64_t R, int32_t m, const uint32_t* __restrict__ max_bits,
-                           __half* __restrict__ xop, float* __restrict__ cterm) {
+                           __half* __restrict__ xop, float* __restrict__ cterm, float fixed_c,
+                           const int32_t* __restrict__ kp) {
   const int64_t g = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
   if (g >= R * kBN) return;
-  int e;
-  frexpf(0.5f * __uint_as_float(*max_bits), &e);
-  const float C = ldexpf(1.0f, e);  // > max N_R / 2 (or 1 if all norms are 0)
-  if (g == 0) *cterm = C;
+  float C = fixed_c;
+  if (!(C > 0.0f)) {
+    int e;
+    frexpf(0.5f * __uint_as_float(*max_bits), &e);
+    C = ldexpf(1.0f, e);  // > max N_R / 2 (or 1 if all norms are 0)
+  }
+  if (g == 0 && cterm) *cterm = C;
   const int64_t ref = g / kBN;
-  const int row = static_cast<int>(g % kBN);
+  const int row0 = static_cast<int>(g % kBN);
+  const int row = (kp && row0 >= kp[ref]) ? kBN : row0;  // padding rows of a ragged reference
   __half h[kXH];
 #pragma unroll
   for (int i = 0; i < kXH; ++i) h[i] = __float2half_rn(0.0f);
   if (row < m) {
-    const float val = C - 0.5f * nr[ref * m + row];
+    const float val = C - 0.5f * nr[ref * m + row0];
     h[0] = __float2half_rn(val);
     const float r1 = val - __half2float(h[0]);
     h[1] = __float2half_rn(r1);
@@ -429,7 +439,7 @@ __global__ void xop_kernel(const float* __restrict__ nr, int64_t R, int32_t m, c
   } else {
     h[0] = __ushort_as_half(0xFC00u);  // -inf
   }
-  uint4* dst = reinterpret_cast<uint4*>(xop + g * kXH);
+  uint4* dst = reinterpret_cast<uint4*>(xop + g * kXH);  // (ref, row0)
   const uint4* src = reinterpret_cast<const uint4*>(h);
   dst[0] = src[0];
   dst[1] = src[1];
@@ -514,13 +524,26 @@ cudaError_t launch_f16_xop(const void* r, int64_t R, int32_t m, uint32_t* scratc
   f16::nr_rows_kernel<<<static_cast<unsigned>((rows * 8 + 255) / 256), 256, 0, s>>>(static_cast<const __half*>(r),
                                                                                    rows, nr, scratch);
   f16::xop_kernel<<<static_cast<unsigned>((R * kBN + 255) / 256), 256, 0, s>>>(nr, R, m, scratch,
-                                                                               static_cast<__half*>(xop), cterm);
+                                                                               static_cast<__half*>(xop), cterm, 0.0f,
+                                                                               nullptr);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_f16_xop_fixed(const void* r, int64_t R, int32_t m, const int32_t* kp, float C, float* nr, void* xop,
+                                 cudaStream_t s) {
+  if (R <= 0) return cudaSuccess;
+  const int64_t rows = R * m;
+  f16::nr_rows_kernel<<<static_cast<unsigned>((rows * 8 + 255) / 256), 256, 0, s>>>(static_cast<const __half*>(r),
+                                                                                   rows, nr, nullptr);
+  f16::xop_kernel<<<static_cast<unsigned>((R * kBN + 255) / 256), 256, 0, s>>>(nr, R, m, nullptr,
+                                                                               static_cast<__half*>(xop), nullptr, C, kp);
   return cudaGetLastError();
 }
 
 cudaError_t launch_f16_match(const CUtensorMap& qmap, const CUtensorMap& rmap, const CUtensorMap& xmap,
                              const float* cterm, const float* nq, int32_t B, int32_t n, int32_t T, int64_t R,
-                             uint32_t num2, uint32_t den2, uint32_t* counts, int num_sms, cudaStream_t s) {
+                             uint32_t num2, uint32_t den2, uint32_t* counts, int num_sms, cudaStream_t s, int64_t ldc,
+                             int64_t col0, int64_t rbase, const int32_t* n_valid) {
   cudaError_t e = cudaFuncSetAttribute(f16::match_f16_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(f16::Plan::kAlloc));
   if (e != cudaSuccess) return e;
@@ -529,8 +552,8 @@ cudaError_t launch_f16_match(const CUtensorMap& qmap, const CUtensorMap& rmap, c
   while (R * ((B + qpj - 1) / qpj) < 2LL * num_sms && qpj > 1) qpj = (qpj + 1) / 2;
   const int64_t jobs = R * ((B + qpj - 1) / qpj);
   const int grid = static_cast<int>(jobs < num_sms ? jobs : num_sms);
-  f16::match_f16_kernel<<<grid, f16::kThreads, f16::Plan::kAlloc, s>>>(qmap, rmap, xmap, cterm, nq, B, n, T, R, qpj,
-                                                                        num2, den2, counts);
+  f16::match_f16_kernel<<<grid, f16::kThreads, f16::Plan::kAlloc, s>>>(
+      qmap, rmap, xmap, cterm, nq, B, n, T, R, qpj, num2, den2, counts, ldc > 0 ? ldc : R, col0, rbase, n_valid);
   return cudaGetLastError();
 }
 

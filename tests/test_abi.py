@@ -67,7 +67,29 @@ def test_config_struct_matches_header():
     fields = re.findall(r"^\s*(?:const\s+)?\w+\*?\s+\*?(\w+)(?:,\s*(\w+))?;", body, re.M)
     names = [x for f in fields for x in f if x]
     assert names == [f for f, _ in tid.Config._fields_]
-    assert ctypes.sizeof(tid.Config) == 72
+
+
+def test_struct_sizes_match_the_c_compiler(tmp_path):
+    """Every struct the binding mirrors has the size and field offsets gcc gives the header's."""
+    import paper_conf_icpp_wangzll21_b200 as tid
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    structs = {"tid_config": tid.Config, "tid_info": tid.Info, "tid_stats": tid.Stats, "tid_tuning": tid.Tuning,
+               "tid_geom_params": tid.GeomParams}
+    lines = ['#include <stdio.h>', '#include <stddef.h>', '#include "tid.h"', "int main(void) {"]
+    for cname, py in structs.items():
+        lines.append(f'  printf("{cname} %zu\\n", sizeof({cname}));')
+        for f, _ in py._fields_:
+            lines.append(f'  printf("{cname}.{f} %zu\\n", offsetof({cname}, {f}));')
+    lines.append("  return 0;\n}")
+    src = tmp_path / "sizes.c"
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "sizes"
+    subprocess.check_call(["gcc", "-I", os.path.join(root, "include"), str(src), "-o", str(exe)])
+    got = dict(l.split() for l in subprocess.check_output([str(exe)], text=True).splitlines())
+    for cname, py in structs.items():
+        assert int(got[cname]) == ctypes.sizeof(py), cname
+        for f, _ in py._fields_:
+            assert int(got[f"{cname}.{f}"]) == getattr(py, f).offset, (cname, f)
 
 
 def test_plain_c_example_compiles_and_links(tmp_path):

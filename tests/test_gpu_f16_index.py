@@ -1,0 +1,99 @@
+"""GPU parity of the float path stored in the index (descriptor "f16"): u8 SIFT
+converted on the GPU to RootSIFT (or scaled SIFT) fp16 at ingest and per search, matched on
+tcgen05.mma.kind::f16 through the same windows / top-k / host tier / merge machinery as the
+integer path.  Expected values come from the float64 oracle on the same fp16 values (and, where
+the fp16 values make every fp32 step exact, from the exact integer oracle)."""
+import numpy as np
+import pytest
+
+import oracle
+import tidgen
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def tid():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    from paper_conf_icpp_wangzll21_b200 import build
+    build.build()
+    import paper_conf_icpp_wangzll21_b200 as t
+    return t
+
+
+def test_f16_index_rootsift_parity(tid):
+    """RootSIFT fp16 index, 64 queries x 2,000 references: every count within +-1 of the float64
+    oracle on the same fp16 values for >= 99.9 % of pairs; the planted target ranks first; the
+    returned top-k is the (count desc, id asc) ranking of the index's own count matrix; Eq. 2
+     of the GPU's own fp16 values is small."""
+    B, n, R, m, k = 64, 1000, 2000, 256, 5
+    refs, _ = tidgen.refs(0, R, m)
+    qs, tg = tidgen.queries(0, B, n, R_total=R, m=m)
+    with tid.Index(ref_kp=m, query_kp_max=1024, descriptor="f16") as idx:
+        idx.add_references(refs)
+        counts = idx.search_counts(qs).astype(np.int64)
+        ids, cnt = idx.search(qs, k)
+        q16 = idx.f16_prepare(qs, True, 1.0)
+        r16 = idx.f16_prepare(refs, True, 1.0)
+        info = idx.info()
+    assert info["hbm_bytes_per_reference"] == m * 128 * 2 + 256 * 16 * 2
+    want = oracle.f16_search_counts_c(q16, r16).astype(np.int64)
+    d = np.abs(counts - want)
+    assert np.mean(d <= 1) >= 0.999 and d.max() <= 2, (np.mean(d <= 1), d.max())
+    np.testing.assert_array_equal(ids[:, 0], tg)
+    e_ids, e_cnt = oracle.topk(counts, k)
+    np.testing.assert_array_equal(ids, e_ids)
+    np.testing.assert_array_equal(cnt, e_cnt)
+    rq, rr = oracle.rootsift(qs[0, :300]), oracle.rootsift(refs[0])
+    e = oracle.compression_error(rq, rr, q16[0, :300].astype(np.float64), r16[0].astype(np.float64))
+    assert 0 < e < 1e-3
+
+
+@pytest.mark.parametrize("host", [False, True])
+def test_f16_index_scaled_sift_exact(tid, host):
+    """Raw SIFT x 2^-7 in fp16 is exact and so is every fp32 step of the kind::f16 path: the float
+    index must reproduce the exact integer oracle bit for bit — with ragged kp and n_q, deleted
+    references, several count windows and (host=True) a streamed pinned host tier."""
+    R, m, n, B, k = 70, 200, 300, 3, 6
+    refs, kp = tidgen.refs(0, R, m, kp_min=60, pad_byte=31)
+    qs, _ = tidgen.queries(0, B, n, R_total=R, m=m, kp_min=60, n_planted=50)
+    n_q = np.array([300, 131, 7], np.int32)
+    rb = m * 128 * 2
+    kw = dict(hbm_budget_bytes=20 * rb, host_budget_bytes=100 * rb) if host else {}
+    with tid.Index(ref_kp=m, query_kp_max=512, descriptor="f16", f16_rootsift=False, f16_scale=2.0 ** -7,
+                   **kw) as idx:
+        idx.add_references(refs, kp)
+        if host:
+            assert idx.info()["host_references"] == R - 20
+        idx.set_tuning(window_refs=17, host_chunk_refs=9)
+        idx.delete([4, 33])
+        counts = idx.search_counts(qs, n_q=n_q).astype(np.int64)
+        ids, cnt = idx.search(qs, k, n_q=n_q)
+    want = oracle.search_counts(qs, refs, n_q=n_q, kp=kp)
+    want[:, [4, 33]] = 0
+    np.testing.assert_array_equal(counts, want)
+    c = want.copy()
+    c[:, [4, 33]] = -1
+    e_ids, e_cnt = oracle.np_rank(c, k)
+    np.testing.assert_array_equal(ids, e_ids)
+    np.testing.assert_array_equal(cnt, e_cnt)
+
+
+def test_f16_index_host_tier_map_and_equals_resident(tid):
+    """A float index's host tier filled in place (fp16 values) searches exactly like the same
+    references resident in HBM (same kernel, same fp16 values)."""
+    R, m, n, B = 40, 256, 400, 2
+    refs, _ = tidgen.refs(5, R, m)
+    qs, _ = tidgen.queries(5, B, n, R_total=R, m=m)
+    with tid.Index(ref_kp=m, descriptor="f16") as res:
+        res.add_references(refs)
+        c_res = res.search_counts(qs)
+        r16 = res.f16_prepare(refs, True, 1.0)
+    with tid.Index(ref_kp=m, descriptor="f16", host_budget_bytes=R * m * 256) as idx:
+        first, view = idx.host_tier_map(R)
+        view[:] = r16
+        idx.set_tuning(host_chunk_refs=16)
+        c_host = idx.search_counts(qs)
+    np.testing.assert_array_equal(c_host, c_res)
