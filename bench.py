@@ -497,10 +497,11 @@ def main():
             "kernel": "match_f16_kernel" if f1 else "match_kernel", "kernel_ms": match_ms,
             "kernel_share_of_step": (st["match_ms"] / args.steps) / ms_per_step,
             "frac_of_nominal": achieved / (2250.0 if f1 else 4500.0),
-            "algorithmic_ops": "2*n*m*128 per (query, reference) pair; the kernel also runs a 5th (norm-term) "
-                               "K-step, +25% tensor work not counted here",
+            "algorithmic_ops": "2*n*m*128 per (query, reference) pair; the kernel also runs a "
+                               + ("9th (norm-term) K = 16 step, +12.5%" if f1 else "5th (norm-term) K-step, +25%")
+                               + " tensor work not counted here",
             "binding_note": "the fused epilogue (TMEM loads + two-partition top-2 on the ALU pipe) limits the kernel "
-                            "below the tensor peak; see DESIGN.md section 7",
+                            "below the tensor peak; see DESIGN.md sections 6-8",
             "pipes_ncu": pipes_from_profile(traffic)}
 
     # CPU oracle on rank 0's host cores, after every timed region (the other ranks wait)

@@ -27,6 +27,12 @@
 
 #include <climits>
 
+// Timing-experiment switches that skip work and give WRONG results (skeleton timings in DESIGN.md):
+// refused unless the build says it is an experiment.
+#if (defined(TID_NOSCAN) || defined(TID_NOMMA) || defined(TID_NOLOAD)) && !defined(TID_EXPERIMENT)
+#error "TID_NOSCAN / TID_NOMMA / TID_NOLOAD skip work (wrong results): timing experiments only, add -DTID_EXPERIMENT"
+#endif
+
 namespace tid {
 namespace f16 {
 

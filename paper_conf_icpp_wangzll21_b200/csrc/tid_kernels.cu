@@ -4,6 +4,12 @@
 
 #include <climits>
 
+// Timing-experiment switches that skip work and give WRONG results (skeleton timings in DESIGN.md):
+// refused unless the build says it is an experiment.
+#if (defined(TID_NOSCAN) || defined(TID_NOMMA) || defined(TID_NOLOAD)) && !defined(TID_EXPERIMENT)
+#error "TID_NOSCAN / TID_NOMMA / TID_NOLOAD skip work (wrong results): timing experiments only, add -DTID_EXPERIMENT"
+#endif
+
 namespace tid {
 
 // ------------------------------------------------------------------ PTX helpers (sm_100a)
@@ -782,50 +788,6 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             // so buffer and phase are compile-time functions of pp (fully unrolled)
             static_assert(kNB == 2 && kPiecesPerChunk == 4, "static buffer / phase schedule");
             const int np = c == cpr - 1 ? np_last : kPiecesPerChunk;
-#ifdef TID_PIPE
-            // Software-pipelined TMEM reads: the chunk's pieces are read as 32-column halves, the
-            // next half's tcgen05.ld in flight while this half is scanned; a piece's buffer is
-            // released as soon as both its halves have landed (before its second half is scanned).
-            {
-              uint32_t ha[32], hb[32];
-              auto bufp = [&](int pp) { return static_cast<uint32_t>(g * kNB + (pp & 1)); };
-              auto parp = [&](int pp) { return static_cast<uint32_t>(((pp >> 1) ^ (ph_t >> (pp & 1))) & 1); };
-              mbar_wait(tfull(bufp(0)), parp(0));
-              tc_fence_after();
-              tmem_ld32(taddr_q + bufp(0) * kPiece, ha);
-              tmem_wait_ld();
-              reg_fence(ha);
-#pragma unroll
-              for (int k = 0; k < 2 * kPiecesPerChunk; ++k) {
-                const int pp = k >> 1;
-                if (kSkip && pp >= np) break;
-                uint32_t(&cur)[32] = (k & 1) ? hb : ha;
-                uint32_t(&nxt)[32] = (k & 1) ? ha : hb;
-                const int kn = k + 1;
-                const bool more = kn < 2 * kPiecesPerChunk && (!kSkip || (kn >> 1) < np);
-                if (more) {
-                  if ((kn & 1) == 0) {  // first half of the next piece: its accumulator must be complete
-                    mbar_wait(tfull(bufp(kn >> 1)), parp(kn >> 1));
-                    tc_fence_after();
-                  }
-                  tmem_ld32(taddr_q + bufp(kn >> 1) * kPiece + (kn & 1) * 32, nxt);
-                }
-                const int lim = kpc - pp * kPiece - (k & 1) * 32;
-                if (lim >= 32) scan32_fold<false>(cur, 32, R, T1, T2);
-                else scan32_fold<true>(cur, lim, R, T1, T2);
-                if (more) {
-                  tmem_wait_ld();
-                  reg_fence(nxt);
-                  if (kn & 1) {  // both halves of piece kn >> 1 are in registers: buffer free
-                    tc_fence_before();
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(tempty(bufp(kn >> 1)));
-                  }
-                }
-              }
-            }
-            if (false)
-#endif
 #pragma unroll
             for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
               if (kSkip && pp >= np) break;  // all-padding pieces (m not a multiple of 64 x 4) are not computed
