@@ -1420,39 +1420,21 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
   const uint8_t* dq;
   const int32_t* dnv;
   TRY(stage_queries(idx, q, n_q, n, P, &dq, &dnv, s));
-  // references: device copy (host input) and packed column keys
+  // references: read in place on the device (a host or unaligned buffer is copied); their keys
+  // N_R * 256 + i and the masking of rows >= m_r happen inside the match kernel
   const uint8_t* dr = r;
   const size_t rbytes = static_cast<size_t>(P) * m * kDim;
-  const bool r_dev = is_device_ptr(r);
-  TRY(idx->ws_colkey.ensure(static_cast<size_t>(P) * cpr * kColBytes, "pair keys"));
-  RefPrepParams rp{};
-  rp.m = m;
-  rp.cpr = cpr;
-  rp.count = P;
-  rp.colkey = idx->ws_colkey.as<int32_t>();
+  if (!is_device_ptr(r) || reinterpret_cast<uintptr_t>(r) % 16) {
+    TRY(idx->ws_r.ensure(rbytes, "pair references"));
+    TRY(copy_in(idx, idx->ws_r.p, r, rbytes, s));
+    dr = idx->ws_r.as<uint8_t>();
+  }
+  const int32_t* dmr = nullptr;
   if (m_r) {
     TRY(idx->ws_mr.ensure(static_cast<size_t>(P) * 4, "m_r"));
     TRY(copy_in(idx, idx->ws_mr.p, m_r, static_cast<size_t>(P) * 4, s));
-    rp.kp = idx->ws_mr.as<int32_t>();
+    dmr = idx->ws_mr.as<int32_t>();
   }
-  if (!r_dev || m_r) {
-    // host input, or masked rows to zero: work on our own copy
-    TRY(idx->ws_r.ensure(rbytes, "pair references"));
-    if (r_dev) {
-      rp.src = r;  // copy + zero rows >= m_r
-    } else {
-      TRY(copy_in(idx, idx->ws_r.p, r, rbytes, s));
-      rp.src = nullptr;
-    }
-    rp.desc = idx->ws_r.as<uint8_t>();
-    dr = idx->ws_r.as<uint8_t>();
-  } else {
-    if (reinterpret_cast<uintptr_t>(r) % 16) return fail(TID_EINVAL, "r must be 16-byte aligned");
-    rp.desc = nullptr;  // read-only: keys only
-    rp.src = r;
-  }
-  launch_ref_prep(rp, s);
-  count_kernel(idx);
   TRY(idx->ws_nq.ensure(static_cast<size_t>(P) * T * kBM * 4, "query norms"));
   launch_query_prep(dq, P, n, T, idx->ws_nq.as<int32_t>(), nullptr, s);
   count_kernel(idx);
@@ -1485,7 +1467,8 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
   p.n_qchunks = 1;
   p.n_refs = P;
   p.ref_map_base = 0;
-  p.colkey = idx->ws_colkey.as<int32_t>();
+  p.colkey = nullptr;  // computed in the kernel
+  p.m_valid = dmr;
   p.nq = idx->ws_nq.as<int32_t>();
   p.n_valid = dnv;
   p.n_rows = n;

@@ -538,7 +538,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     for (int i = 0; i < kMaxSlots; ++i) {
       mbar_init(rfull(i), 1);
       mbar_init(rempty(i), kNG + kEpiWarps);
-      mbar_init(xready(i), 1);  // search: the producer warp expanded the slot's norm digits
+      mbar_init(xready(i), 1);  // search: the producer warp expanded the slot's norm digits; verify: the
+                                // epilogue computed the keys and masked rows beyond m_r
     }
     for (int i = 0; i < kTmemBufs; ++i) { mbar_init(tfull(i), 1); mbar_init(tempty(i), 4); }
     fence_barrier_init();
@@ -571,13 +572,14 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         if (lane == 0) {
           for (int sl = 0; sl < nslots; ++sl) {
             PROF_B(); mbar_wait_sleep(rempty(sl), (slot_par >> sl & 1u) ^ 1); PROF_E(0);
-            mbar_expect_tx(rfull(sl), kRTileBytes + kColBytes);
+            mbar_expect_tx(rfull(sl), kRTileBytes + (kFold ? kColBytes : 0u));
             const int s = sl / cpr, c = sl % cpr;
             const int64_t ref = J.ref_first + s;
             tma_load_3d(sbase + SmemPlan::kR + sl * kRTileBytes, &rmap, rfull(sl), 0, c * kBN,
                         static_cast<int>(p.ref_map_base + ref));
-            bulk_load(sbase + SmemPlan::kCol + sl * kColBytes, p.colkey + (ref * cpr + c) * kColInts, kColBytes,
-                      rfull(sl));
+            if (kFold)  // search: the stored column terms W (verify computes its keys on chip)
+              bulk_load(sbase + SmemPlan::kCol + sl * kColBytes, p.colkey + (ref * cpr + c) * kColInts, kColBytes,
+                        rfull(sl));
           }
         }
         __syncwarp();
@@ -687,7 +689,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             const int sl = s * cpr + c;
             if (!(ready_mask >> sl & 1u)) {
               PROF_B(); mbar_wait(rfull(sl), (slot_par >> sl & 1u));
-              if (kFold) mbar_wait(xready(sl), (slot_par >> sl & 1u));  // norm digits expanded
+              // search: norm digits expanded; verify with m_r: rows beyond m_r zeroed
+              if (kFold || p.m_valid) mbar_wait(xready(sl), (slot_par >> sl & 1u));
               PROF_E(2);
               ready_mask |= 1u << sl;
             }
@@ -728,7 +731,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
       for (int sl = 0; sl < nslots; ++sl) {
         if (!(ready_mask >> sl & 1u)) {  // keep rempty / xready phases ordered
           mbar_wait(rfull(sl), (slot_par >> sl & 1u));
-          if (kFold) mbar_wait(xready(sl), (slot_par >> sl & 1u));
+          if (kFold || p.m_valid) mbar_wait(xready(sl), (slot_par >> sl & 1u));
         }
         mma_commit(rempty(sl));
         slot_par ^= 1u << sl;
@@ -757,8 +760,44 @@ __global__ void __launch_bounds__(kNumThreads, 1)
       const int nslots = J.nr * cpr;
       const int U = J.nq * T * J.nr;
       // column keys of every slot of the job (also orders this warp's rempty arrivals)
+      const int mcap = (!kFold && p.m_valid) ? min(p.m_valid[J.ref_first], p.m) : p.m;  // issued before the wait
       PROF_B();
       for (int sl = 0; sl < nslots; ++sl) mbar_wait(rfull(sl), slot_par >> sl & 1u);
+      if constexpr (!kFold) {
+        // verify: the packed column keys N_R * 256 + i (Alg. 1 step 1) computed here from the
+        // reference tile already in shared memory (no separate pass over the references in HBM).
+        // A row's 128 bytes stay within its 128-byte line under SWIZZLE_128B, so the sum over its
+        // eight 16-byte chunks does not depend on their order.  Rows >= min(m_r, m) get the sentinel.
+        for (int x = ew * 32 + lane; x < nslots * kBN; x += kEpiWarps * 32) {
+          const int sl = x / kBN, i = x % kBN;
+          const int col = (sl % cpr) * kBN + i;
+          uint32_t acc = 0;
+          const uint32_t row = sbase + SmemPlan::kR + sl * kRTileBytes + i * kDim;
+          if (col < mcap) {
+#pragma unroll
+            for (int w = 0; w < kDim / 16; ++w) {
+              const int4 x4 = lds128(row + 16 * w);
+              acc = __dp4a(static_cast<uint32_t>(x4.x), static_cast<uint32_t>(x4.x), acc);
+              acc = __dp4a(static_cast<uint32_t>(x4.y), static_cast<uint32_t>(x4.y), acc);
+              acc = __dp4a(static_cast<uint32_t>(x4.z), static_cast<uint32_t>(x4.z), acc);
+              acc = __dp4a(static_cast<uint32_t>(x4.w), static_cast<uint32_t>(x4.w), acc);
+            }
+          } else if (col < p.m) {
+            // a row beyond this pair's m_r holds the caller's bytes: zero it, so its product is 0 and
+            // the sentinel key 256 * (2^23 - 1) + i never wins (rows >= m are zero-filled by TMA)
+#pragma unroll
+            for (int w = 0; w < kDim / 16; ++w)
+              asm volatile("st.shared.v4.b32 [%0], {%1, %1, %1, %1};" ::"r"(row + 16 * w), "r"(0) : "memory");
+          }
+          const int32_t key = (col < mcap ? static_cast<int32_t>(acc) : kSentinelNorm) * 256 + i;
+          asm volatile("st.shared.s32 [%0], %1;" ::"r"(sbase + SmemPlan::kCol + sl * kColBytes + i * 4), "r"(key)
+                       : "memory");
+        }
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // zeroed rows -> tensor-core reads
+        named_bar(1, kEpiWarps * 32);  // every key of the job written before any warp scans
+        if (p.m_valid && ew == 0 && lane == 0)  // the MMA warps may read the masked tiles
+          for (int sl = 0; sl < nslots; ++sl) mbar_arrive(xready(sl));
+      }
       PROF_E(4);
       // own units u = g, g + kNG, ...; unit u = (tile t = u / nr, reference s = u % nr), and
       // t = (query qi - q_first) * T + tq.  Tracked incrementally (no divisions per unit).
@@ -1044,34 +1083,49 @@ void launch_ref_prep(const RefPrepParams& p, cudaStream_t s) {
 
 // ------------------------------------------------------------------ a2: query prep
 // N_Q per row (Alg. 1 step 2) and, for the search path, the shifted copy q' = q ^ 0x80
-// (= q - 128 as s8), one 16-byte word per thread-iteration.
+// (= q - 128 as s8).  Eight lanes per 128-byte row, one 16-byte word each, so a warp reads and
+// writes four whole rows (512 contiguous bytes) per instruction; the row sum by shuffles.
 __global__ void query_prep_kernel(const uint8_t* __restrict__ q, int64_t B, int32_t n, int32_t rows_pad,
                                   int32_t* __restrict__ nq, uint8_t* __restrict__ qs) {
+  constexpr int kRows = 4;  // rows per 8-lane group: four independent 16-byte loads in flight per lane
   const int64_t gid = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
-  if (gid >= B * rows_pad) return;
-  const int64_t b = gid / rows_pad;
-  const int row = static_cast<int>(gid % rows_pad);
-  uint32_t acc = 0;
-  if (row < n) {
-    const uint4* src = reinterpret_cast<const uint4*>(q + (b * n + row) * kDim);
-    uint4* dst = qs ? reinterpret_cast<uint4*>(qs + (b * n + row) * kDim) : nullptr;
+  const int l8 = static_cast<int>(gid & 7);
+  const int64_t g = gid >> 3;  // 8-lane group
+  const int64_t total = B * rows_pad;
+  uint4 x[kRows];
+  bool have[kRows];
 #pragma unroll
-    for (int w = 0; w < kDim / 16; ++w) {
-      const uint4 x = src[w];
-      acc = __dp4a(x.x, x.x, acc); acc = __dp4a(x.y, x.y, acc);
-      acc = __dp4a(x.z, x.z, acc); acc = __dp4a(x.w, x.w, acc);
-      if (dst) dst[w] = make_uint4(x.x ^ 0x80808080u, x.y ^ 0x80808080u, x.z ^ 0x80808080u, x.w ^ 0x80808080u);
-    }
+  for (int k = 0; k < kRows; ++k) {  // rows g + k * groups: consecutive groups read consecutive rows
+    const int64_t r = g + k * (static_cast<int64_t>(gridDim.x) * blockDim.x >> 3);
+    const int64_t b = r < total ? r / rows_pad : 0;
+    const int row = r < total ? static_cast<int>(r - b * rows_pad) : 0;
+    have[k] = r < total && row < n;
+    x[k] = have[k] ? *reinterpret_cast<const uint4*>(q + (b * n + row) * kDim + l8 * 16) : make_uint4(0, 0, 0, 0);
   }
-  nq[gid] = static_cast<int32_t>(acc);
+#pragma unroll
+  for (int k = 0; k < kRows; ++k) {
+    const int64_t r = g + k * (static_cast<int64_t>(gridDim.x) * blockDim.x >> 3);
+    uint32_t acc = 0;
+    acc = __dp4a(x[k].x, x[k].x, acc); acc = __dp4a(x[k].y, x[k].y, acc);
+    acc = __dp4a(x[k].z, x[k].z, acc); acc = __dp4a(x[k].w, x[k].w, acc);
+    if (qs && have[k]) {
+      const int64_t b = r / rows_pad;
+      const int row = static_cast<int>(r - b * rows_pad);
+      *reinterpret_cast<uint4*>(qs + (b * n + row) * kDim + l8 * 16) = make_uint4(
+          x[k].x ^ 0x80808080u, x[k].y ^ 0x80808080u, x[k].z ^ 0x80808080u, x[k].w ^ 0x80808080u);
+    }
+#pragma unroll
+    for (int o = 1; o < 8; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (r < total && l8 == 0) nq[r] = static_cast<int32_t>(acc);
+  }
 }
 
 void launch_query_prep(const uint8_t* q, int64_t B, int32_t n, int32_t tiles_per_q, int32_t* nq, uint8_t* qs,
                        cudaStream_t s) {
   const int32_t rows_pad = tiles_per_q * kBM;
-  const int64_t total = B * rows_pad;
-  if (total == 0) return;
-  query_prep_kernel<<<static_cast<unsigned>((total + 255) / 256), 256, 0, s>>>(q, B, n, rows_pad, nq, qs);
+  const int64_t groups = (B * rows_pad + 3) / 4;  // 4 rows per 8-lane group
+  if (B * rows_pad == 0) return;
+  query_prep_kernel<<<static_cast<unsigned>((groups * 8 + 255) / 256), 256, 0, s>>>(q, B, n, rows_pad, nq, qs);
 }
 
 // ------------------------------------------------------------------ a6: top-k of the count matrix

@@ -79,6 +79,7 @@ struct MatchParams {
   const int32_t* colkey;     // [n_refs][cpr*256] packed column keys (launch-relative)
   const int32_t* nq;         // [num_q][tiles_per_q*128] squared query norms
   const int32_t* n_valid;    // [num_q] valid query rows (nullable = n_rows)
+  const int32_t* m_valid;    // verify: [P] valid reference rows per pair (nullable = m)
   int32_t n_rows;            // stored rows per query (n)
   uint32_t* counts;          // search: [num_q][ldc] (+ col0); verify: [num_q]
   int64_t ldc;

@@ -31,4 +31,32 @@ with tid.Index(query_kp_max=1024) as idx:
     q16, r16 = idx.f16_prepare(Qf, False, 2.0 ** -7), idx.f16_prepare(Rr, False, 2.0 ** -7)
     fc = idx.f16_search_counts(q16, r16)
 assert np.array_equal(fc.astype(np.int64), oracle.search_counts(Qf, Rr))
+# round 2: several count windows + deletes, verify with ragged m_r (rows masked in the kernel),
+# the float index (fp16 storage + host tier), post-match verification (f4)
+with tid.Index(ref_kp=256, query_kp_max=1024) as idx:
+    idx.add_references(refs, kp)
+    idx.set_tuning(window_refs=4)
+    idx.delete([2])
+    ids, cn = idx.search(qs, 4)
+c2 = oracle.search_counts(qs, refs, kp=kp)
+c2[:, 2] = -1
+assert np.array_equal(ids, oracle.np_rank(c2, 4)[0])
+m_r = np.array([300, 17, 2], np.int32)
+with tid.Index(ref_kp=256) as idx:
+    vc, nn = idx.verify(Q, R, m_r=m_r)
+assert np.array_equal(vc.astype(np.int64), oracle.verify(Q, R, m_r=m_r)[0])
+with tid.Index(ref_kp=200, descriptor="f16", f16_rootsift=False, f16_scale=2.0 ** -7,
+               hbm_budget_bytes=2 * 200 * 256, host_budget_bytes=8 * 200 * 256) as idx:
+    idx.set_tuning(host_chunk_refs=2)
+    idx.add_references(Rr)
+    fc2 = idx.search_counts(Qf)
+assert np.array_equal(fc2.astype(np.int64), oracle.search_counts(Qf, Rr))
+rng = np.random.default_rng(1)
+qxy = (rng.random((3, 200, 2)) * 100).astype(np.float32)
+rxy = (rng.random((3, 300, 2)) * 100).astype(np.float32)
+with tid.Index(ref_kp=256) as idx:
+    _, g, inl, mdl = idx.verify_geometric(Q, R, qxy, rxy, iterations=64, inlier_px=5.0)
+_, onn = oracle.verify(Q, R)
+eg, ei, em = oracle.geometric(onn, qxy, rxy, iterations=64, inlier_px=5.0)
+assert np.array_equal(g.astype(np.int64), eg) and np.array_equal(inl.astype(np.int64), ei)
 print("sanitize run ok")
