@@ -262,7 +262,8 @@ __device__ __forceinline__ void reg_fence64(uint32_t (&v)[64]) {
 
 // ------------------------------------------------------------------ optional cycle accounting
 // Built only with -DTID_PROF (experiments): per-warp clock64 buckets, read back with
-// tid_debug_read_prof().  Buckets: epilogue 0 wait-accumulator 1 scan 2 finalise 4 wait-keys;
+// tid_debug_read_prof().  Buckets: epilogue 0 wait-accumulator 1 scan 2 finalise 3 TMEM load + release
+// (search) 4 wait-keys 5 unit tail: ratio test, count, next unit (search);
 // MMA 0 wait-free-accumulator 1 wait-query 2 wait-ref; producer 0 wait-ref-slot 1 wait-query-stage;
 // 7 = whole loop.
 #ifdef TID_PROF
@@ -486,6 +487,34 @@ __device__ __forceinline__ uint32_t use_parity(int np) {
   return (((np + 1) >> 1) & 1u) | (((np >> 1) & 1u) << 1);
 }
 
+// The fifth MMA K-step's B operand for one reference column: 32 u8 digits of E = floor(W / 2)
+// against the constant operand a = (255 x 15, 1, 255 x 15, 1), i.e. E = 255 * (sum of the 30
+// "255"-weighted digits) + d15 + d31.  The 30 weighted digits (positions 0..14, 16..30, ranks
+// 0..29) are filled greedily: rank k holds clamp(hi - 255 k, 0, 255) with hi = E / 255 <= 4,112,
+// so ranks < q = hi / 255 are 255, rank q holds hi mod 255 and the rest 0; d15 = E mod 255,
+// d31 = 0 (capacity 7,650 * 255 + 254 > max E = 1,048,576).  Padding columns (W < 0): zeros.
+// Built as 8 rank words, then moved into position order with byte permutes.
+__device__ __forceinline__ void norm_digits(int32_t W, uint32_t (&w8)[8]) {
+  const uint32_t E = W > 0 ? static_cast<uint32_t>(W) >> 1 : 0u;
+  const uint32_t hi = E / 255u, lo = E - 255u * hi;
+  const uint32_t q = hi / 255u, rem = hi - 255u * q;
+  uint32_t rk[8];  // rank words: byte b of rk[i] = digit of rank 4 i + b
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int d = static_cast<int>(q) - 4 * i;  // full bytes in this word
+    rk[i] = d >= 4 ? 0xFFFFFFFFu
+                   : (d < 0 ? 0u : ((d == 0 ? 0u : (0xFFFFFFFFu >> (32 - 8 * d))) | (rem << (8 * d))));
+  }
+  w8[0] = rk[0];
+  w8[1] = rk[1];
+  w8[2] = rk[2];
+  w8[3] = (rk[3] & 0x00FFFFFFu) | (lo << 24);              // ranks 12..14, then position 15 = lo
+  w8[4] = __byte_perm(rk[3], rk[4], 0x6543);                // ranks 15..18
+  w8[5] = __byte_perm(rk[4], rk[5], 0x6543);                // ranks 19..22
+  w8[6] = __byte_perm(rk[5], rk[6], 0x6543);                // ranks 23..26
+  w8[7] = __byte_perm(rk[6], rk[7], 0x6543) & 0x00FFFFFFu;  // ranks 27..29, position 31 = 0
+}
+
 // ------------------------------------------------------------------ fused match kernel
 // One persistent CTA per SM.  A job = (up to kNG = 3 references resident in SMEM, fewer chunks'
 // worth for m > 256) x (range of query tiles streamed through a kQStages ring; search: copied
@@ -538,8 +567,9 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     for (int i = 0; i < kMaxSlots; ++i) {
       mbar_init(rfull(i), 1);
       mbar_init(rempty(i), kNG + kEpiWarps);
-      mbar_init(xready(i), 1);  // search: the producer warp expanded the slot's norm digits; verify: the
-                                // epilogue computed the keys and masked rows beyond m_r
+      // search: the kNG MMA warps expanded the slot's norm digits; verify: the epilogue computed the
+      // keys and masked rows beyond m_r (one arrival)
+      mbar_init(xready(i), kFold ? kNG : 1);
     }
     for (int i = 0; i < kTmemBufs; ++i) { mbar_init(tfull(i), 1); mbar_init(tempty(i), 4); }
     fence_barrier_init();
@@ -583,52 +613,6 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           }
         }
         __syncwarp();
-        if constexpr (kFold) {
-        // the fifth MMA K-step's B operand, expanded by this warp from the column terms W (HBM keeps only W:
-        // 4 B per keypoint instead of 32 B of digits).  Column i of a slot: 32 u8 digits of
-        // E = floor(W / 2) against the constant operand a = (255 x 15, 1, 255 x 15, 1):
-        // E = 255 * (sum of the 30 "255"-weighted digits) + d15 + d31, filled greedily (255, 255, ...,
-        // rest, 0, ...) in positions 0..14, 16..30 and d15 = E mod 255, d31 = 0 (capacity 7,650 * 255 +
-        // 254 > max E = 1,048,576).  Padding columns (W < 0) get zero digits.  Both 16-byte halves of
-        // the constant operand are equal, so the SWIZZLE_32B placement of a row's two halves does not
-        // change the product: rows are written plainly, 32 B each.
-        for (int sl = 0; sl < nslots; ++sl) mbar_wait(rfull(sl), slot_par >> sl & 1u);  // column terms landed
-        for (int x = lane; x < nslots * kBN; x += 32) {
-          const int sl = x / kBN, col = x % kBN;
-          int W;
-          asm volatile("ld.shared.s32 %0, [%1];" : "=r"(W) : "r"(sbase + SmemPlan::kCol + sl * kColBytes + col * 4));
-          const uint32_t E = W > 0 ? static_cast<uint32_t>(W) >> 1 : 0u;
-          const uint32_t hi = E / 255u, lo = E - 255u * (E / 255u);
-          uint32_t w8[8];
-#pragma unroll
-          for (int wi = 0; wi < 8; ++wi) {
-            uint32_t word = 0;
-#pragma unroll
-            for (int bi = 0; bi < 4; ++bi) {
-              const int t = wi * 4 + bi;                          // digit position 0..31
-              const int rank = t < 15 ? t : (t < 31 && t > 15 ? t - 1 : -1);  // order among the 30 "255" digits
-              uint32_t dg;
-              if (t == 15) dg = lo;
-              else if (t == 31) dg = 0u;
-              else {
-                const int32_t rest = static_cast<int32_t>(hi) - 255 * rank;
-                dg = rest <= 0 ? 0u : (rest >= 255 ? 255u : static_cast<uint32_t>(rest));
-              }
-              word |= dg << (8 * bi);
-            }
-            w8[wi] = word;
-          }
-          const uint32_t dst = sbase + SmemPlan::kX + sl * kXTileBytes + col * kXDim;
-          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst), "r"(w8[0]), "r"(w8[1]), "r"(w8[2]),
-                       "r"(w8[3]) : "memory");
-          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst + 16), "r"(w8[4]), "r"(w8[5]), "r"(w8[6]),
-                       "r"(w8[7]) : "memory");
-        }
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> tensor-core reads
-        __syncwarp();
-        if (lane == 0)
-          for (int sl = 0; sl < nslots; ++sl) mbar_arrive(xready(sl));
-      }
         slot_par ^= (1u << nslots) - 1u;
         const int ntiles = J.nq * T;
         if (lane == 0) {
@@ -673,6 +657,29 @@ __global__ void __launch_bounds__(kNumThreads, 1)
       const Job J = decode_job(p, j);
       const int nslots = J.nr * cpr;
       const int U = J.nq * T * J.nr;
+      if constexpr (kFold) {
+        // the norm digits of the job's slots, expanded by the kNG MMA warps (HBM keeps only the column
+        // terms W: 4 B per keypoint instead of 32 B of digits); both 16-byte halves of the constant
+        // operand are equal, so the SWIZZLE_32B placement of a row's halves does not matter and rows
+        // are written plainly, 32 B each
+        for (int sl = 0; sl < nslots; ++sl) mbar_wait(rfull(sl), slot_par >> sl & 1u);
+        for (int x = mw * 32 + lane; x < nslots * kBN; x += kNG * 32) {
+          const int sl = x / kBN, col = x % kBN;
+          int W;
+          asm volatile("ld.shared.s32 %0, [%1];" : "=r"(W) : "r"(sbase + SmemPlan::kCol + sl * kColBytes + col * 4));
+          uint32_t w8[8];
+          norm_digits(W, w8);
+          const uint32_t dst = sbase + SmemPlan::kX + sl * kXTileBytes + col * kXDim;
+          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst), "r"(w8[0]), "r"(w8[1]), "r"(w8[2]),
+                       "r"(w8[3]) : "memory");
+          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst + 16), "r"(w8[4]), "r"(w8[5]), "r"(w8[6]),
+                       "r"(w8[7]) : "memory");
+        }
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> tensor-core reads
+        __syncwarp();
+        if (lane == 0)
+          for (int sl = 0; sl < nslots; ++sl) mbar_arrive(xready(sl));
+      }
       uint32_t ready_mask = 0;
       int waited = 0, t = 0, s = 0, g = 0;
       for (int u = 0; u < U; ++u) {
@@ -832,6 +839,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               if (kSkip && pp >= np) break;  // all-padding pieces (m not a multiple of 64 x 4) are not computed
               const uint32_t buf = g * kNB + (pp & 1);
               PROF_B(); mbar_wait(tfull(buf), ((pp >> 1) ^ (ph_t >> (pp & 1))) & 1); PROF_E(0);
+              PROF_B();
               tc_fence_after();
 #ifndef TID_NOLOAD  // timing experiment only: scan stale registers (wrong results)
               tmem_ld64(taddr_q + buf * kPiece, v);
@@ -841,6 +849,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               tc_fence_before();  // the piece is in registers: buffer free
               __syncwarp();
               if (lane == 0) mbar_arrive(tempty(buf));
+              PROF_E(3);
               PROF_B();
               if (kpc >= (pp + 1) * kPiece) {  // every column of the piece is real (the common case)
 #ifndef TID_NOSCAN
@@ -861,6 +870,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             G1 = max(G1, x1);
             PROF_E(2);
           }
+          PROF_B();
           // d = N_Q - 2X - p, p in {0, 1}: decide the ratio test from the bounds
           const bool real2 = G2 > INT_MIN;
           bool undecided = false;
@@ -976,6 +986,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           }
           cnt = 0;
         }
+        if constexpr (kFold) { PROF_E(5); }
         u += kNG; s = ns; tq = ntq;
         if (nqi != qi && has_next) {
           qi = nqi;

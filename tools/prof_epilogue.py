@@ -32,7 +32,7 @@ lib.tid_debug_read_prof(buf.ctypes.data, ctypes.c_size_t(buf.nbytes))
 buf = buf.reshape(148, 32, 8).astype(np.float64)
 nw = (tid.load_library() and 0) or None
 print("match kernel ms", st["match_ms"], "launches", st["match_launches"])
-names = {0: "producer", 1: "mma", 2: "mma", 3: "mma", 4: "mma"}
+names = {0: "producer", 1: "mma", 2: "mma", 3: "mma"}
 for w in range(0, 32):
     if buf[:, w, 7].sum() == 0:
         continue
