@@ -389,9 +389,8 @@ def main():
         CONFIGS[args.config] = (B, n, Rg, m, k)
     nccl_id = None
     if world > 1:
-        obj = [tid.nccl_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(obj, src=0)
-        nccl_id = obj[0]
+        from paper_conf_icpp_wangzll21_b200.dist import exchange_nccl_id
+        nccl_id = exchange_nccl_id(tid.nccl_unique_id)  # rank 0 creates it, the process group broadcasts it
     c5 = None
     if args.config == "c5":
         idx, refs, start, Rg, c5 = build_c5(args, tid, tidgen, torch, dist, world, rank, local, nccl_id, m)
