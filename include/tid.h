@@ -78,9 +78,9 @@ typedef struct {
                                   1 = the paper's float path (SURVEY row f1, §4.2, §5.1
                                   P:555-576): u8 SIFT given to add/search is converted on the GPU
                                   to [RootSIFT] x f16_scale in fp16 and stored that way (2 B per
-                                  value + 8 KiB of norm terms per reference); matching on
+                                  value + 8 KiB of norm terms per 256 keypoints); matching on
                                   tcgen05.mma.kind::f16 (see tid_f16_search_counts for the
-                                  arithmetic and the +-1 count acceptance).  ref_kp <= 256;
+                                  arithmetic and the +-1 count acceptance).  ref_kp <= 512;
                                   save / load and tid_verify stay on the u8 path.              */
   float    f16_scale;          /* descriptor 1: scale factor before the fp16 conversion (0 = 1)  */
   int32_t  f16_rootsift;       /* descriptor 1: 1 = RootSIFT (L1-normalise, sqrt) first          */
@@ -243,7 +243,7 @@ tid_status tid_merge_topk(tid_index* idx, const int64_t* ids_in, const int32_t* 
  *   P:527-530) and round to nearest even.  Computed in fp32 on the GPU.
  *
  * tid_f16_search_counts: good-match counts of B fp16 queries [B][n][128] against R fp16 references
- *   [R][m][128] (host or device; n <= query_kp_max, 2 <= m <= 256) -> counts_out uint32 [B][R].
+ *   [R][m][128] (host or device; n <= query_kp_max, 2 <= m <= 512) -> counts_out uint32 [B][R].
  *   The product q.r runs on tcgen05.mma.kind::f16 with fp32 accumulation; a ninth K-step adds
  *   C - N_R / 2 (N_R in fp32 from the fp16 values, split into three fp16 terms; C = power of two
  *   >= max N_R / 2), so d = N_Q + 2C - 2 X with X = C + q.r - N_R / 2 >= 0 read straight from the

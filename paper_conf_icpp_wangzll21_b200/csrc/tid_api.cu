@@ -480,7 +480,7 @@ tid_status run_pass(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, in
                         int64_t col0) -> tid_status {
     CUtensorMap rmap, xmap;
     TRY(make_map_f16(&rmap, rbase, map_count, idx->cfg.ref_kp, kBN));
-    TRY(make_xmap(&xmap, xbase, map_count, kBN));
+    TRY(make_xmap(&xmap, xbase, map_count, static_cast<int64_t>(kBN) * idx->cpr));
     cudaEvent_t e0 = nullptr, e1 = nullptr;
     if (idx->prof) {
       if (idx->prof_used == idx->prof_ev.size()) {
@@ -496,7 +496,7 @@ tid_status run_pass(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, in
     }
     CU(launch_f16_match(qmap, rmap, xmap, idx->ws_f16c.as<float>(), idx->ws_f16nq.as<float>(), static_cast<int32_t>(B),
                         n, T, cnt, idx->cfg.ratio_num * idx->cfg.ratio_num, idx->cfg.ratio_den * idx->cfg.ratio_den,
-                        counts, idx->num_sms, s, W, col0, base, nvalid));
+                        counts, idx->num_sms, s, W, col0, base, nvalid, idx->cpr));
     if (idx->prof) {
       CU(cudaEventRecord(e1, s));
       idx->stats.match_launches++;
@@ -519,7 +519,7 @@ tid_status run_pass(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, in
     for (int b = 0; b < 2; ++b) {
       TRY(idx->stage_desc[b].ensure(static_cast<size_t>(chunk * rb), "host-tier staging"));
       if (idx->f16)
-        TRY(idx->stage_xop[b].ensure(static_cast<size_t>(chunk) * kBN * 16 * 2, "staging norm terms"));
+        TRY(idx->stage_xop[b].ensure(static_cast<size_t>(chunk) * kBN * idx->cpr * 16 * 2, "staging norm terms"));
       else
         TRY(idx->stage_colkey[b].ensure(static_cast<size_t>(chunk) * idx->cpr * kColBytes, "staging keys"));
       TRY(idx->stage_kp[b].ensure(static_cast<size_t>(chunk) * 4, "staging kp"));
@@ -633,7 +633,7 @@ tid_status alloc_segment(tid_index* idx, bool on_host, int64_t cap, Segment* out
   } else {
     cudaError_t e1 = cudaMalloc(&sg.desc, static_cast<size_t>(cap * rb));
     cudaError_t e2 = e1 != cudaSuccess ? e1
-                     : idx->f16 ? cudaMalloc(&sg.xop, static_cast<size_t>(cap) * kBN * 16 * 2)
+                     : idx->f16 ? cudaMalloc(&sg.xop, static_cast<size_t>(cap) * kBN * idx->cpr * 16 * 2)
                                 : cudaMalloc(&sg.colkey, static_cast<size_t>(cap) * idx->cpr * kColBytes);
     if (e1 != cudaSuccess || e2 != cudaSuccess) {
       cudaGetLastError();
@@ -695,7 +695,7 @@ tid_status ingest_hbm(tid_index* idx, Segment& sg, int64_t pos, const uint8_t* s
     TRY(idx->ws_kp.ensure(static_cast<size_t>(take) * 4, "kp staging"));
     CU(cudaMemcpy(idx->ws_kp.p, kp_host, static_cast<size_t>(take) * 4, cudaMemcpyHostToDevice));
     TRY(f16_norm_terms(idx, sg.desc + pos * rb, take, idx->ws_kp.as<int32_t>(),
-                       sg.xop + static_cast<size_t>(pos) * kBN * 16, nullptr));
+                       sg.xop + static_cast<size_t>(pos) * kBN * idx->cpr * 16, nullptr));
     CU(cudaStreamSynchronize(nullptr));
     return TID_OK;
   }
@@ -824,8 +824,8 @@ tid_status tid_index_create(const tid_config* cfg, tid_index** out) {
   if (cfg->world_size > 1 && !cfg->nccl_unique_id) return fail(TID_EINVAL, "world_size > 1 needs nccl_unique_id");
   if (cfg->id_base < 0) return fail(TID_EINVAL, "id_base must be >= 0");
   if (cfg->descriptor != 0 && cfg->descriptor != 1) return fail(TID_EINVAL, "descriptor must be 0 (u8) or 1 (fp16)");
-  if (cfg->descriptor == 1 && cfg->ref_kp > kBN)
-    return fail(TID_EINVAL, "descriptor 1 (float path): ref_kp=%d > 256", cfg->ref_kp);
+  if (cfg->descriptor == 1 && cfg->ref_kp > 2 * kBN)
+    return fail(TID_EINVAL, "descriptor 1 (float path): ref_kp=%d > 512", cfg->ref_kp);
   if (cfg->descriptor == 1 && !(cfg->f16_scale >= 0.0f)) return fail(TID_EINVAL, "f16_scale must be >= 0");
 
   int ndev = 0;
@@ -852,7 +852,7 @@ tid_status tid_index_create(const tid_config* cfg, tid_index** out) {
     idx->f16_scale = cfg->f16_scale > 0.0f ? cfg->f16_scale : 1.0f;
     idx->f16_rootsift = cfg->f16_rootsift ? 1 : 0;
     idx->ref_bytes = 2 * idx->in_bytes;
-    idx->hbm_ref_bytes = idx->ref_bytes + static_cast<int64_t>(kBN) * 16 * 2;
+    idx->hbm_ref_bytes = idx->ref_bytes + static_cast<int64_t>(kBN) * idx->cpr * 16 * 2;
     // C: the smallest power of two >= half the largest N_R the index can hold, so X = C + q.r - N_R/2
     // >= 0 for every reference: RootSIFT rows have unit norm (x (1 + 2^-11)^2 after
     // fp16 rounding), raw SIFT at most 128 * 255^2; both times scale^2.
@@ -1117,7 +1117,7 @@ tid_status tid_delete_references(tid_index* idx, const int64_t* local_ids, int64
       TRY(idx->ws_kp.ensure(4, "kp"));
       CU(cudaMemcpy(idx->ws_kp.p, &zero, 4, cudaMemcpyHostToDevice));
       TRY(f16_norm_terms(idx, sg->desc + off * idx->ref_bytes, 1, idx->ws_kp.as<int32_t>(),
-                         sg->xop + static_cast<size_t>(off) * kBN * 16, nullptr));
+                         sg->xop + static_cast<size_t>(off) * kBN * idx->cpr * 16, nullptr));
       CU(cudaStreamSynchronize(nullptr));
     } else if (!sg->on_host) {
       RefPrepParams rp{};
@@ -1641,7 +1641,7 @@ tid_status tid_f16_search_counts(tid_index* idx, const uint16_t* q, int32_t n, i
                                  int32_t m, int64_t R, uint32_t* counts_out, void* stream) {
   if (!idx || !q || !r || !counts_out) return fail(TID_EINVAL, "null argument");
   if (n < 1 || n > idx->cfg.query_kp_max) return fail(TID_EINVAL, "n=%d outside 1..query_kp_max", n);
-  if (m < 2 || m > kBN) return fail(TID_EINVAL, "m=%d outside 2..256 (float path)", m);
+  if (m < 2 || m > 2 * kBN) return fail(TID_EINVAL, "m=%d outside 2..512 (float path)", m);
   if (B < 1 || R < 1) return fail(TID_EINVAL, "B and R must be >= 1");
   if (B > (1LL << 30) || R > (1LL << 31) - 1) return fail(TID_EINVAL, "B or R too large");
   TRY(set_device(idx));
@@ -1663,7 +1663,8 @@ tid_status tid_f16_search_counts(tid_index* idx, const uint16_t* q, int32_t n, i
   }
   TRY(idx->ws_f16nq.ensure(static_cast<size_t>(B) * T * kBM * 4, "f16 query norms"));
   // norm-term operand (R x 256 rows x 32 B) + the scalars max N_R (bits) and C
-  const size_t xb = static_cast<size_t>(R) * kBN * 32;
+  const int fcpr = static_cast<int>(ceil_div(m, kBN));  // 256-row chunks per reference (1 or 2)
+  const size_t xb = static_cast<size_t>(R) * kBN * fcpr * 32;
   TRY(idx->ws_f16nr.ensure(xb + 256 + static_cast<size_t>(R) * m * 4, "f16 reference norm terms"));
   uint8_t* xop = idx->ws_f16nr.as<uint8_t>();
   uint32_t* nrmax = reinterpret_cast<uint32_t*>(xop + xb);
@@ -1679,10 +1680,10 @@ tid_status tid_f16_search_counts(tid_index* idx, const uint16_t* q, int32_t n, i
   CUtensorMap qmap, rmap, xmap;
   TRY(make_map_f16(&qmap, dq, B, n, kBM));
   TRY(make_map_f16(&rmap, dr, R, m, kBN));
-  TRY(make_xmap(&xmap, xop, R, kBN));  // 32-B rows, SWIZZLE_32B (same geometry as the u8 norm digits)
+  TRY(make_xmap(&xmap, xop, R, static_cast<int64_t>(kBN) * fcpr));  // 32-B rows, SWIZZLE_32B
   CU(launch_f16_match(qmap, rmap, xmap, cterm, idx->ws_f16nq.as<float>(), static_cast<int32_t>(B), n, T, R,
                       idx->cfg.ratio_num * idx->cfg.ratio_num, idx->cfg.ratio_den * idx->cfg.ratio_den, counts,
-                      idx->num_sms, s));
+                      idx->num_sms, s, 0, 0, 0, nullptr, fcpr));
   count_kernel(idx);
   if (!dev_counts) {
     bool host_out = false;

@@ -41,31 +41,32 @@ constexpr int kThreads = 32 * (2 + kEpi);
 constexpr int kHalfBytes = 128;                     // one SWIZZLE_128B row = 64 fp16
 constexpr uint32_t kRHalf = kBN * kHalfBytes;       // 32 KiB: 256 reference rows x 64 fp16
 constexpr uint32_t kQHalf = kBM * kHalfBytes;       // 16 KiB: 128 query rows x 64 fp16
-constexpr int kStages = 4;
 constexpr int kXH = 16;                             // fp16 per norm-term row (one K = 16 step, 32 B)
 constexpr uint32_t kXTile = kBN * kXH * 2;          // 8 KiB: 256 reference rows x 16 fp16
-#ifndef TID_F16_N
-#define TID_F16_N 128
-#endif
-// MMA pieces of kFN columns through kFNB = 512 / kFN TMEM buffers: with N = 128 the MMA can run
-// 1.5 units ahead of the epilogue instead of one (the A tile is re-read per piece: more shared-
-// memory operand traffic, which the measurement decides)
-constexpr int kFN = TID_F16_N;
-constexpr int kFPieces = kBN / kFN;                 // pieces per unit
+// MMA pieces of kFN = 128 columns through kFNB = 4 TMEM buffers (512 columns): a reference chunk
+// of 256 keypoints is 2 pieces; global piece gp of the CTA uses buffer gp % 4 with phase
+// (gp / 4) & 1, so with one chunk per reference the MMA runs up to 1.5 units ahead of the epilogue.
+constexpr int kFN = 128;
+constexpr int kFPieces = kBN / kFN;                 // pieces per 256-column chunk
 constexpr int kFNB = 512 / kFN;                     // TMEM buffers
-static_assert(kFNB % kFPieces == 0 && (kFNB / kFPieces) == 2, "two units of pieces in flight");
 
+// Shared-memory plan for references of kCpr 256-row chunks (m <= 256 kCpr): the resident reference
+// (kCpr x 64 KiB) and its norm-term tiles, a ring of query tiles (4 stages for one chunk, 2 for two:
+// 227 KiB in all), the constant operand, barriers.
+template <int kCpr>
 struct Plan {
-  static constexpr uint32_t kR = 0;                            // 2 halves
-  static constexpr uint32_t kQ = kR + 2 * kRHalf;              // kStages x 2 halves
-  static constexpr uint32_t kX = kQ + kStages * 2 * kQHalf;    // norm-term tile (SWIZZLE_32B)
-  static constexpr uint32_t kAx = kX + kXTile;                 // constant A operand (ones)
+  static constexpr int kStages = kCpr == 1 ? 4 : 2;
+  static constexpr uint32_t kR = 0;                                   // kCpr chunks x 2 K-halves
+  static constexpr uint32_t kQ = kR + kCpr * 2 * kRHalf;              // kStages x 2 halves
+  static constexpr uint32_t kX = kQ + kStages * 2 * kQHalf;           // kCpr norm-term tiles (SWIZZLE_32B)
+  static constexpr uint32_t kAx = kX + kCpr * kXTile;                 // constant A operand (ones)
   static constexpr uint32_t kBar = kAx + kBM * kXH * 2;
   static constexpr uint32_t kQFull = kBar, kQEmpty = kBar + 8 * kStages;
   static constexpr uint32_t kRFull = kQEmpty + 8 * kStages, kREmpty = kRFull + 8;
   static constexpr uint32_t kTFull = kREmpty + 8, kTEmpty = kTFull + 8 * kFNB;
   static constexpr uint32_t kTmemPtr = kTEmpty + 8 * kFNB;
   static constexpr uint32_t kAlloc = kTmemPtr + 16 + 1024;
+  static_assert(kAlloc <= 227 * 1024, "shared memory");
 };
 
 __device__ __forceinline__ uint32_t su32(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
@@ -151,23 +152,6 @@ __device__ __forceinline__ void ld16x64(uint32_t taddr, uint32_t (&v)[64]) {
   for (int i = 0; i < 64; ++i) asm volatile("" : "+r"(v[i]));
 }
 
-// Two x64 loads (columns [0, 128) and [128, 256) of the same 16 lanes) with one wait.
-__device__ __forceinline__ void ld16x64x2(uint32_t taddr, uint32_t (&v)[64], uint32_t (&w)[64]) {
-  asm volatile(
-      "tcgen05.ld.sync.aligned.16x64b.x64.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
-      "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32,%33,%34,%35,%36,%37,%38,%39,%40,%41,%42,%43,%44,"
-      "%45,%46,%47,%48,%49,%50,%51,%52,%53,%54,%55,%56,%57,%58,%59,%60,%61,%62,%63}, [%64];"
-      : F16_OUT32(v), F16_OUT32((v + 32)) : "r"(taddr));
-  asm volatile(
-      "tcgen05.ld.sync.aligned.16x64b.x64.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
-      "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32,%33,%34,%35,%36,%37,%38,%39,%40,%41,%42,%43,%44,"
-      "%45,%46,%47,%48,%49,%50,%51,%52,%53,%54,%55,%56,%57,%58,%59,%60,%61,%62,%63}, [%64];"
-      : F16_OUT32(w), F16_OUT32((w + 32)) : "r"(taddr + 128));
-  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-#pragma unroll
-  for (int i = 0; i < 64; ++i) asm volatile("" : "+r"(v[i]), "+r"(w[i]));
-}
-
 // Two-partition top-2 of the largest values (see tid_kernels.cu): P = 16-register halves of a
 // 32-register block, P' = position mod 16; R[b] = P' maxima, T1 >= T2 = two largest P maxima.
 __device__ __forceinline__ int mx3(int a, int b, int c) { return __vimax3_s32(a, b, c); }
@@ -197,25 +181,28 @@ __device__ __forceinline__ void finish(const int (&R)[16], int T1, int T2, int& 
   x2 = mx3(T2, sr, sc);
 }
 
+template <int kCpr>
 __global__ void __launch_bounds__(kThreads, 1)
     match_f16_kernel(const __grid_constant__ CUtensorMap qmap, const __grid_constant__ CUtensorMap rmap,
                      const __grid_constant__ CUtensorMap xmap, const float* __restrict__ cterm,
                      const float* __restrict__ nq_all, int32_t B, int32_t n, int32_t T, int64_t R, int32_t q_per_job,
                      uint32_t num2, uint32_t den2, uint32_t* __restrict__ counts, int64_t ldc, int64_t col0,
                      int64_t rbase, const int32_t* __restrict__ n_valid) {
+  using P = Plan<kCpr>;
+  constexpr int kStages = P::kStages;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const uint32_t sb = su32(smem);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  auto qfull = [&](int i) { return sb + Plan::kQFull + 8 * i; };
-  auto qempty = [&](int i) { return sb + Plan::kQEmpty + 8 * i; };
-  const uint32_t rfull = sb + Plan::kRFull, rempty = sb + Plan::kREmpty;
-  auto tfull = [&](int i) { return sb + Plan::kTFull + 8 * i; };
-  auto tempty = [&](int i) { return sb + Plan::kTEmpty + 8 * i; };
-  uint32_t* tptr = reinterpret_cast<uint32_t*>(smem + Plan::kTmemPtr);
+  auto qfull = [&](int i) { return sb + P::kQFull + 8 * i; };
+  auto qempty = [&](int i) { return sb + P::kQEmpty + 8 * i; };
+  const uint32_t rfull = sb + P::kRFull, rempty = sb + P::kREmpty;
+  auto tfull = [&](int i) { return sb + P::kTFull + 8 * i; };
+  auto tempty = [&](int i) { return sb + P::kTEmpty + 8 * i; };
+  uint32_t* tptr = reinterpret_cast<uint32_t*>(smem + P::kTmemPtr);
   {  // constant A operand of the norm-term step: every row (1, 1, 1, 0 x 5) in both 16-B halves,
      // so the SWIZZLE_32B layout does not matter
-    uint32_t* ax = reinterpret_cast<uint32_t*>(smem + Plan::kAx);
+    uint32_t* ax = reinterpret_cast<uint32_t*>(smem + P::kAx);
     const uint32_t one2 = 0x3C003C00u, one0 = 0x00003C00u;  // fp16 pairs (1, 1), (1, 0)
     for (int i = threadIdx.x; i < kBM * kXH / 2; i += blockDim.x) {
       const int w = i & 3;  // 32-bit word within a 16-B half
@@ -248,44 +235,50 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int64_t r = j / qchunks;
         const int q0 = static_cast<int>(j % qchunks) * q_per_job, nq = min(q_per_job, B - q0);
         bar_wait(rempty, (rc & 1) ^ 1);
-        bar_expect(rfull, 2 * kRHalf + kXTile);
-        tma3(sb + Plan::kR, &rmap, rfull, 0, 0, static_cast<int>(rbase + r));
-        tma3(sb + Plan::kR + kRHalf, &rmap, rfull, 64, 0, static_cast<int>(rbase + r));
-        tma3(sb + Plan::kX, &xmap, rfull, 0, 0, static_cast<int>(rbase + r));
+        bar_expect(rfull, kCpr * (2 * kRHalf + kXTile));
+#pragma unroll
+        for (int c = 0; c < kCpr; ++c) {  // chunk c: reference rows 256 c .. (both K-halves) + norm terms
+          tma3(sb + P::kR + c * 2 * kRHalf, &rmap, rfull, 0, c * kBN, static_cast<int>(rbase + r));
+          tma3(sb + P::kR + c * 2 * kRHalf + kRHalf, &rmap, rfull, 64, c * kBN, static_cast<int>(rbase + r));
+          tma3(sb + P::kX + c * kXTile, &xmap, rfull, 0, c * kBN, static_cast<int>(rbase + r));
+        }
         for (int t = 0; t < nq * T; ++t, ++qc) {
           const int st = qc % kStages;
           bar_wait(qempty(st), ((qc / kStages) & 1) ^ 1);
           bar_expect(qfull(st), 2 * kQHalf);
-          const uint32_t dst = sb + Plan::kQ + st * 2 * kQHalf;
+          const uint32_t dst = sb + P::kQ + st * 2 * kQHalf;
           tma3(dst, &qmap, qfull(st), 0, (t % T) * kBM, q0 + t / T);
           tma3(dst + kQHalf, &qmap, qfull(st), 64, (t % T) * kBM, q0 + t / T);
         }
       }
     }
   } else if (warp == 1) {
-    uint32_t qc = 0, rc = 0, uc = 0;
-    const uint64_t ax = desc32(sb + Plan::kAx), bx = desc32(sb + Plan::kX);
+    uint32_t qc = 0, rc = 0, gp = 0;  // gp: global piece counter (buffer gp % 4, phase (gp / 4) & 1)
+    const uint64_t ax = desc32(sb + P::kAx);
     for (int64_t j = blockIdx.x; j < n_jobs; j += gridDim.x, ++rc) {
       const int q0 = static_cast<int>(j % qchunks) * q_per_job, nq = min(q_per_job, B - q0);
       bar_wait(rfull, rc & 1);
-      const uint64_t b0 = desc128(sb + Plan::kR), b1 = desc128(sb + Plan::kR + kRHalf);
-      for (int t = 0; t < nq * T; ++t, ++qc, ++uc) {
+      for (int t = 0; t < nq * T; ++t, ++qc) {
         const int st = qc % kStages;
         bar_wait(qfull(st), (qc / kStages) & 1);
-        const uint32_t qa = sb + Plan::kQ + st * 2 * kQHalf;
-        // unit uc uses buffers kFPieces * (uc & 1) + h, each once per two units (static phases)
+        const uint32_t qa = sb + P::kQ + st * 2 * kQHalf;
 #pragma unroll
-        for (int h = 0; h < kFPieces; ++h) {
-          const int buf = kFPieces * (uc & 1) + h;
-          bar_wait(tempty(buf), ((uc >> 1) & 1) ^ 1);
-          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        for (int c = 0; c < kCpr; ++c) {
+          const uint64_t b0 = desc128(sb + P::kR + c * 2 * kRHalf), b1 = desc128(sb + P::kR + c * 2 * kRHalf + kRHalf);
+          const uint64_t bx = desc32(sb + P::kX + c * kXTile);
+#pragma unroll
+          for (int h = 0; h < kFPieces; ++h, ++gp) {
+            const int buf = gp % kFNB;
+            bar_wait(tempty(buf), ((gp / kFNB) & 1) ^ 1);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 #ifdef TID_NOMMA  // timing experiment only
-          commit(tfull(buf));
+            commit(tfull(buf));
 #else
-          // reference rows kFN * h.. : SWIZZLE_128B 8-row groups of 1 KiB / SWIZZLE_32B groups of 256 B
-          mma_unit(tmem + buf * kFN, desc128(qa), desc128(qa + kQHalf), b0 + h * (kFN * 128 >> 4),
-                   b1 + h * (kFN * 128 >> 4), ax, bx + h * (kFN * 32 >> 4), tfull(buf));
+            // reference rows kFN * h.. : SWIZZLE_128B 8-row groups of 1 KiB / SWIZZLE_32B groups of 256 B
+            mma_unit(tmem + buf * kFN, desc128(qa), desc128(qa + kQHalf), b0 + h * (kFN * 128 >> 4),
+                     b1 + h * (kFN * 128 >> 4), ax, bx + h * (kFN * 32 >> 4), tfull(buf));
 #endif
+          }
         }
         commit(qempty(st));
       }
@@ -297,11 +290,8 @@ __global__ void __launch_bounds__(kThreads, 1)
     const uint32_t tq = tmem + (static_cast<uint32_t>(quarter * 32 + 16 * half) << 16);
     const int row_in_tile = quarter * 32 + 16 * half + (lane >> 2) + 8 * (lane & 1);
     const double c2 = 2.0 * static_cast<double>(*cterm);
-    uint32_t rc = 0, uc = 0;
+    uint32_t rc = 0, gp = 0;
     uint32_t v[64];
-#if TID_F16_N == 256
-    uint32_t w[64];
-#endif
     for (int64_t j = blockIdx.x; j < n_jobs; j += gridDim.x, ++rc) {
       const int64_t r = j / qchunks;
       const int q0 = static_cast<int>(j % qchunks) * q_per_job, nq = min(q_per_job, B - q0);
@@ -309,7 +299,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       uint32_t cnt = 0;
       int qi = q0, tt = 0;  // query and tile of unit t (no divisions per unit)
       int nv = n_valid ? min(n_valid[qi], n) : n;
-      for (int t = 0; t < nq * T; ++t, ++uc) {
+      for (int t = 0; t < nq * T; ++t) {
         const int row = tt * kBM + row_in_tile;
         const bool valid = row < nv;
         const float nqv = nq_all[static_cast<int64_t>(qi) * T * kBM + row];
@@ -317,26 +307,12 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
         for (int b = 0; b < 16; ++b) Rm[b] = INT_MIN;
         int T1 = INT_MIN, T2 = INT_MIN;
-#if TID_F16_N == 256
-        const int buf = uc & 1;
-        bar_wait(tfull(buf), (uc >> 1) & 1);
-        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        // both 128-column halves in flight at once; the buffer is free as soon as they landed
-        ld16x64x2(tq + buf * kBN, v, w);
-        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-        __syncwarp();
-        if (lane == 0) bar_arrive(tempty(buf));
-#ifndef TID_NOSCAN  // timing experiment only
-        scan32(v, Rm, T1, T2);
-        scan32(v + 32, Rm, T1, T2);
-        scan32(w, Rm, T1, T2);
-        scan32(w + 32, Rm, T1, T2);
-#endif
-#else
+        // every chunk's pieces into one two-partition state: two columns of different loads are in
+        // different P groups, two of one load differ in position mod 16, so the top-2 stays exact
 #pragma unroll
-        for (int h = 0; h < kFPieces; ++h) {  // one x64 load (128 columns) per piece
-          const int buf = kFPieces * (uc & 1) + h;
-          bar_wait(tfull(buf), (uc >> 1) & 1);
+        for (int pc = 0; pc < kCpr * kFPieces; ++pc, ++gp) {  // one x64 load (128 columns) per piece
+          const int buf = gp % kFNB;
+          bar_wait(tfull(buf), (gp / kFNB) & 1);
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
           ld16x64(tq + buf * kFN, v);
           asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
@@ -347,7 +323,6 @@ __global__ void __launch_bounds__(kThreads, 1)
           scan32(v + 32, Rm, T1, T2);
 #endif
         }
-#endif
         int x1, x2;
         finish(Rm, T1, T2, x1, x2);
         {  // merge with the partner thread holding the row's other columns
@@ -420,9 +395,9 @@ __global__ void nr_rows_kernel(const __half* __restrict__ x, int64_t rows, float
 // the launch's maximum; kp (nullable): rows >= kp[ref] are padding (h1 = -inf) like rows >= m.
 __global__ void xop_kernel(const float* __restrict__ nr, int64_t R, int32_t m, const uint32_t* __restrict__ max_bits,
                            __half* __restrict__ xop, float* __restrict__ cterm, float fixed_c,
-                           const int32_t* __restrict__ kp) {
+                           const int32_t* __restrict__ kp, int32_t rows_per_ref) {
   const int64_t g = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
-  if (g >= R * kBN) return;
+  if (g >= R * rows_per_ref) return;
   float C = fixed_c;
   if (!(C > 0.0f)) {
     int e;
@@ -430,9 +405,9 @@ __global__ void xop_kernel(const float* __restrict__ nr, int64_t R, int32_t m, c
     C = ldexpf(1.0f, e);  // > max N_R / 2 (or 1 if all norms are 0)
   }
   if (g == 0 && cterm) *cterm = C;
-  const int64_t ref = g / kBN;
-  const int row0 = static_cast<int>(g % kBN);
-  const int row = (kp && row0 >= kp[ref]) ? kBN : row0;  // padding rows of a ragged reference
+  const int64_t ref = g / rows_per_ref;
+  const int row0 = static_cast<int>(g % rows_per_ref);
+  const int row = (kp && row0 >= kp[ref]) ? rows_per_ref : row0;  // padding rows of a ragged reference
   __half h[kXH];
 #pragma unroll
   for (int i = 0; i < kXH; ++i) h[i] = __float2half_rn(0.0f);
@@ -503,7 +478,7 @@ __global__ void prepare_kernel(const uint8_t* __restrict__ sift, int64_t rows, i
 
 }  // namespace f16
 
-size_t f16_smem_bytes() { return f16::Plan::kAlloc; }
+size_t f16_smem_bytes() { return f16::Plan<1>::kAlloc; }
 
 cudaError_t launch_f16_prepare(const uint8_t* sift, int64_t rows, int32_t rootsift, float scale, void* out,
                                cudaStream_t s) {
@@ -529,9 +504,9 @@ cudaError_t launch_f16_xop(const void* r, int64_t R, int32_t m, uint32_t* scratc
   const int64_t rows = R * m;
   f16::nr_rows_kernel<<<static_cast<unsigned>((rows * 8 + 255) / 256), 256, 0, s>>>(static_cast<const __half*>(r),
                                                                                    rows, nr, scratch);
-  f16::xop_kernel<<<static_cast<unsigned>((R * kBN + 255) / 256), 256, 0, s>>>(nr, R, m, scratch,
-                                                                               static_cast<__half*>(xop), cterm, 0.0f,
-                                                                               nullptr);
+  const int32_t rows_per_ref = ((m + kBN - 1) / kBN) * kBN;
+  f16::xop_kernel<<<static_cast<unsigned>((R * rows_per_ref + 255) / 256), 256, 0, s>>>(
+      nr, R, m, scratch, static_cast<__half*>(xop), cterm, 0.0f, nullptr, rows_per_ref);
   return cudaGetLastError();
 }
 
@@ -541,25 +516,28 @@ cudaError_t launch_f16_xop_fixed(const void* r, int64_t R, int32_t m, const int3
   const int64_t rows = R * m;
   f16::nr_rows_kernel<<<static_cast<unsigned>((rows * 8 + 255) / 256), 256, 0, s>>>(static_cast<const __half*>(r),
                                                                                    rows, nr, nullptr);
-  f16::xop_kernel<<<static_cast<unsigned>((R * kBN + 255) / 256), 256, 0, s>>>(nr, R, m, nullptr,
-                                                                               static_cast<__half*>(xop), nullptr, C, kp);
+  const int32_t rows_per_ref = ((m + kBN - 1) / kBN) * kBN;
+  f16::xop_kernel<<<static_cast<unsigned>((R * rows_per_ref + 255) / 256), 256, 0, s>>>(
+      nr, R, m, nullptr, static_cast<__half*>(xop), nullptr, C, kp, rows_per_ref);
   return cudaGetLastError();
 }
 
 cudaError_t launch_f16_match(const CUtensorMap& qmap, const CUtensorMap& rmap, const CUtensorMap& xmap,
                              const float* cterm, const float* nq, int32_t B, int32_t n, int32_t T, int64_t R,
                              uint32_t num2, uint32_t den2, uint32_t* counts, int num_sms, cudaStream_t s, int64_t ldc,
-                             int64_t col0, int64_t rbase, const int32_t* n_valid) {
-  cudaError_t e = cudaFuncSetAttribute(f16::match_f16_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       static_cast<int>(f16::Plan::kAlloc));
+                             int64_t col0, int64_t rbase, const int32_t* n_valid, int32_t cpr) {
+  if (cpr < 1 || cpr > 2) return cudaErrorInvalidValue;
+  auto kern = cpr == 1 ? f16::match_f16_kernel<1> : f16::match_f16_kernel<2>;
+  const size_t smem = cpr == 1 ? f16::Plan<1>::kAlloc : f16::Plan<2>::kAlloc;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
   if (e != cudaSuccess) return e;
   // queries per job: enough jobs to fill the SMs, otherwise all queries reuse the resident reference
   int32_t qpj = B;
   while (R * ((B + qpj - 1) / qpj) < 2LL * num_sms && qpj > 1) qpj = (qpj + 1) / 2;
   const int64_t jobs = R * ((B + qpj - 1) / qpj);
   const int grid = static_cast<int>(jobs < num_sms ? jobs : num_sms);
-  f16::match_f16_kernel<<<grid, f16::kThreads, f16::Plan::kAlloc, s>>>(
-      qmap, rmap, xmap, cterm, nq, B, n, T, R, qpj, num2, den2, counts, ldc > 0 ? ldc : R, col0, rbase, n_valid);
+  kern<<<grid, f16::kThreads, smem, s>>>(qmap, rmap, xmap, cterm, nq, B, n, T, R, qpj, num2, den2, counts,
+                                       ldc > 0 ? ldc : R, col0, rbase, n_valid);
   return cudaGetLastError();
 }
 

@@ -143,14 +143,16 @@ cudaError_t launch_f16_prepare(const uint8_t* sift, int64_t rows, int32_t rootsi
                                cudaStream_t s);
 cudaError_t launch_f16_norms(const void* x, int64_t items, int32_t rows, int32_t rows_pad, float pad, float* out,
                              cudaStream_t s);
-// norm-term operand [R][256][16] fp16 of fp16 references [R][m][128] and its constant C (device scalar)
+// norm-term operand [R][256 * ceil(m / 256)][16] fp16 of fp16 references [R][m][128] (m <= 512) and its
+// constant C (device scalar)
 cudaError_t launch_f16_xop(const void* r, int64_t R, int32_t m, uint32_t* scratch, float* nr, void* xop,
                            float* cterm, cudaStream_t s);
 // counts[qi * ldc + col0 + r] for references rbase + r of the maps (ldc 0 = R)
 cudaError_t launch_f16_match(const CUtensorMap& qmap, const CUtensorMap& rmap, const CUtensorMap& xmap,
                              const float* cterm, const float* nq, int32_t B, int32_t n, int32_t T, int64_t R,
                              uint32_t num2, uint32_t den2, uint32_t* counts, int num_sms, cudaStream_t s,
-                             int64_t ldc = 0, int64_t col0 = 0, int64_t rbase = 0, const int32_t* n_valid = nullptr);
+                             int64_t ldc = 0, int64_t col0 = 0, int64_t rbase = 0, const int32_t* n_valid = nullptr,
+                             int32_t cpr = 1);
 // index path: norm-term rows with the index's fixed constant C and per-reference keypoint counts
 cudaError_t launch_f16_xop_fixed(const void* r, int64_t R, int32_t m, const int32_t* kp, float C, float* nr, void* xop,
                                  cudaStream_t s);

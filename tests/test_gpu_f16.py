@@ -102,3 +102,15 @@ def test_f16_rootsift_parity_at_scale(tid):
     assert diff.max() <= 2, diff.max()
     assert np.mean(diff <= 1) >= 0.999, np.mean(diff <= 1)
     np.testing.assert_array_equal(np.argmax(got, 1), tg)
+
+
+def test_f16_counts_two_chunk_references(tid):
+    """tid_f16_search_counts with m in (256, 512]: references of two 256-row chunks (exact on u8 SIFT
+    x 2^-7, ragged n)."""
+    Rr, _ = tidgen.refs(7, 9, 384)
+    Q, _ = tidgen.queries(7, 2, 333, R_total=9, m=384, n_planted=80)
+    s = 2.0 ** -7
+    with tid.Index(query_kp_max=1024) as idx:
+        q16, r16 = idx.f16_prepare(Q, False, s), idx.f16_prepare(Rr, False, s)
+        got = idx.f16_search_counts(q16, r16).astype(np.int64)
+    np.testing.assert_array_equal(got, oracle.search_counts(Q, Rr))

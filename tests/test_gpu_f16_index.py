@@ -51,12 +51,13 @@ def test_f16_index_rootsift_parity(tid):
     assert 0 < e < 1e-3
 
 
-@pytest.mark.parametrize("host", [False, True])
-def test_f16_index_scaled_sift_exact(tid, host):
+@pytest.mark.parametrize("host,m", [(False, 200), (True, 200), (False, 384), (True, 500)])
+def test_f16_index_scaled_sift_exact(tid, host, m):
     """Raw SIFT x 2^-7 in fp16 is exact and so is every fp32 step of the kind::f16 path: the float
     index must reproduce the exact integer oracle bit for bit — with ragged kp and n_q, deleted
-    references, several count windows and (host=True) a streamed pinned host tier."""
-    R, m, n, B, k = 70, 200, 300, 3, 6
+    references, several count windows, (host=True) a streamed pinned host tier, and references of
+    two 256-row chunks (m = 384, the paper's operating point, Table 7; m = 500)."""
+    R, n, B, k = 70, 300, 3, 6
     refs, kp = tidgen.refs(0, R, m, kp_min=60, pad_byte=31)
     qs, _ = tidgen.queries(0, B, n, R_total=R, m=m, kp_min=60, n_planted=50)
     n_q = np.array([300, 131, 7], np.int32)
@@ -97,3 +98,21 @@ def test_f16_index_host_tier_map_and_equals_resident(tid):
         idx.set_tuning(host_chunk_refs=16)
         c_host = idx.search_counts(qs)
     np.testing.assert_array_equal(c_host, c_res)
+
+
+def test_f16_index_m384_rootsift_parity(tid):
+    """The paper's final configuration (RootSIFT + FP16, m = 384 reference keypoints, n = 768 query
+    keypoints; §5.1, Table 7): counts within +-1 of the float64 oracle for >= 99.9 % of pairs and
+    the planted target first."""
+    B, n, R, m = 16, 768, 300, 384
+    refs, _ = tidgen.refs(0, R, m)
+    qs, tg = tidgen.queries(0, B, n, R_total=R, m=m)
+    with tid.Index(ref_kp=m, query_kp_max=1024, descriptor="f16") as idx:
+        idx.add_references(refs)
+        counts = idx.search_counts(qs).astype(np.int64)
+        ids, _ = idx.search(qs, 3)
+        q16, r16 = idx.f16_prepare(qs, True, 1.0), idx.f16_prepare(refs, True, 1.0)
+    want = oracle.f16_search_counts_c(q16, r16).astype(np.int64)
+    d = np.abs(counts - want)
+    assert np.mean(d <= 1) >= 0.999 and d.max() <= 2
+    np.testing.assert_array_equal(ids[:, 0], tg)
