@@ -178,14 +178,27 @@ def run_reference(args, cfg_name):
     import tidgen
     per_step_refs = 4096
     refs, _ = tidgen.refs(0, per_step_refs, m, seed=SEED)
-    qs, _ = tidgen.queries(0, 1, n, R_total=Rg * args.gpus, m=m, seed=SEED)
-    # size one step to ~6 s on this host so W + K steps finish in a few minutes
-    rate, _, cores, _ = time_oracle(qs, refs, 2.0)
+    R_total = (Rg or 10_000_000 // args.gpus) * args.gpus  # c5: the requested 10 M
+    qs, _ = tidgen.queries(0, 1, n, R_total=R_total, m=m, seed=SEED)
+    f1 = cfg_name.startswith("f1")
+    if f1:  # the float oracle on the fp16 RootSIFT values (float64 direct sums)
+        q16 = oracle.to_fp16(oracle.rootsift(qs))
+        r16 = oracle.to_fp16(oracle.rootsift(refs))
+        count = lambda S: oracle.f16_search_counts_c(q16, r16[:S])  # noqa: E731
+        cores = len(os.sched_getaffinity(0))
+        count(cores)
+        t0 = time.perf_counter()
+        count(4 * cores)
+        rate = 4 * cores / (time.perf_counter() - t0)
+    else:
+        count = lambda S: oracle.search_counts(qs, refs[:S])  # noqa: E731
+        # size one step to ~6 s on this host so W + K steps finish in a few minutes
+        rate, _, cores, _ = time_oracle(qs, refs, 2.0)
     S = int(max(cores, min(per_step_refs, rate * 6.0)))
     times = []
     for i in range(args.warmup + args.steps):
         t0 = time.perf_counter()
-        c = oracle.search_counts(qs, refs[:S])
+        c = count(S)
         oracle.topk(c, min(k, S))
         dt = time.perf_counter() - t0
         if i >= args.warmup:
@@ -194,7 +207,7 @@ def run_reference(args, cfg_name):
     sample = f"per step: 1 query (n={n}) x {S} references (m={m}) of the {cfg_name} workload + top-{k}"
     line = {"metric": METRIC, "value": value, "unit": "comparisons/s", "impl": "reference", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * statistics.mean(times),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64" if f1 else "int64",
             "data": "synthetic (tidgen: clustered u8 SIFT-like descriptors, planted matches)",
             "config": config_dict(cfg_name, args.gpus),
             "cpu_baseline": {"value": value, "unit": "comparisons/s", "cores": cores, "kind": "oracle",
