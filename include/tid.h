@@ -156,6 +156,9 @@ tid_status tid_index_load(tid_index* idx, const char* path, int64_t* first_local
  *   match_counts_out : int32 [B][k]  their good-match counts.
  * With world_size > 1 the call is collective: every rank passes the same queries
  * and receives the same merged result (one NCCL all-gather of B*k candidates).
+ * Repeated calls with the same device buffers and shape (world_size 1, references in HBM, no
+ * profiling) replay a CUDA graph captured on the second such call; any change of the index
+ * invalidates it.  Results are identical either way.
  */
 tid_status tid_search(tid_index* idx, const uint8_t* queries, const int32_t* n_q, int32_t n,
                       int64_t B, int32_t k, int64_t* ref_ids_out, int32_t* match_counts_out,

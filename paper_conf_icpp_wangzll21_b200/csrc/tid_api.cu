@@ -285,6 +285,21 @@ struct tid_index {
   // every call that touches the workspaces waits for the previous call's work (whatever stream it
   // ran on) and records this event at its end: one index may be driven from several streams
   cudaEvent_t ev_last = nullptr;
+  // CUDA-graph replay of repeated searches (device buffers, HBM-resident references): the
+  // launch-bound small-batch path (C1) costs one graph launch instead of ~5 submissions
+  uint64_t gen = 0;               // bumped by every change of the references / dead flags / tuning
+  cudaStream_t graph_stream = nullptr;
+  cudaEvent_t ev_gin = nullptr, ev_gout = nullptr;
+  struct GraphEntry {
+    const void* q; const void* nq; const void* ids; const void* cnts;
+    int32_t n, k;
+    int64_t B;
+    uint64_t gen;
+    std::vector<void*> ws;        // workspace pointers baked into the graph
+    cudaGraphExec_t exec = nullptr;
+    int uses = 0;
+  };
+  std::vector<GraphEntry> graphs;
   // workspaces
   DevBuf ws_q, ws_nq, ws_nvalid, ws_counts, ws_cand, ws_keys, ws_gather, ws_ids, ws_cnts, ws_r, ws_colkey, ws_nn,
       ws_kp, ws_mr;
@@ -874,6 +889,9 @@ tid_status tid_index_create(const tid_config* cfg, tid_index** out) {
   idx->host_chunk = 16384;
   cudaError_t e = cudaStreamCreateWithFlags(&idx->copy_stream, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&idx->ev_last, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&idx->graph_stream, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&idx->ev_gin, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&idx->ev_gout, cudaEventDisableTiming);
   for (int b = 0; b < 2 && e == cudaSuccess; ++b) {
     e = cudaEventCreateWithFlags(&idx->ev_h2d[b], cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&idx->ev_free[b], cudaEventDisableTiming);
@@ -928,6 +946,11 @@ tid_status tid_index_destroy(tid_index* idx) {
   }
   if (idx->copy_stream) cudaStreamDestroy(idx->copy_stream);
   if (idx->ev_last) cudaEventDestroy(idx->ev_last);
+  for (auto& ge : idx->graphs)
+    if (ge.exec) cudaGraphExecDestroy(ge.exec);
+  if (idx->graph_stream) cudaStreamDestroy(idx->graph_stream);
+  if (idx->ev_gin) cudaEventDestroy(idx->ev_gin);
+  if (idx->ev_gout) cudaEventDestroy(idx->ev_gout);
   if (idx->h_rtot) cudaFreeHost(idx->h_rtot);
   idx->ws_rtot.release();
   if (idx->comm) nccl().CommDestroy(idx->comm);
@@ -942,6 +965,7 @@ tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t
   if (count > 0 && !desc) return fail(TID_EINVAL, "null descriptors");
   TRY(set_device(idx));
   CallGuard guard(idx, nullptr);
+  ++idx->gen;  // segments may change (FIFO swap-outs) even if the add fails
   const int64_t first = idx->n_hbm + idx->n_host;
   if (first_local_id) *first_local_id = first;
   if (count == 0) return TID_OK;
@@ -1067,6 +1091,7 @@ tid_status tid_add_references(tid_index* idx, const uint8_t* desc, const int32_t
 #undef TRY_TX
   idx->dead.resize(static_cast<size_t>(first + count), 0);
   idx->dead_dirty = true;
+  ++idx->gen;  // cached search graphs are stale
   return TID_OK;
 }
 
@@ -1094,6 +1119,7 @@ tid_status tid_host_tier_map(tid_index* idx, int64_t count, uint8_t** desc_out, 
   idx->n_host += count;
   idx->dead.resize(static_cast<size_t>(first + count), 0);
   idx->dead_dirty = true;
+  ++idx->gen;  // cached search graphs are stale
   if (first_local_id) *first_local_id = first;
   return TID_OK;
 }
@@ -1138,6 +1164,7 @@ tid_status tid_delete_references(tid_index* idx, const int64_t* local_ids, int64
   }
   idx->any_dead = idx->any_dead || count > 0;
   idx->dead_dirty = true;
+  ++idx->gen;  // cached search graphs are stale
   return TID_OK;
 }
 
@@ -1174,6 +1201,7 @@ tid_status tid_update_references(tid_index* idx, const int64_t* local_ids, const
     idx->dead[static_cast<size_t>(ids[i])] = 0;
   }
   idx->dead_dirty = true;
+  ++idx->gen;  // cached search graphs are stale
   return TID_OK;
 }
 
@@ -1311,6 +1339,78 @@ tid_status total_references(tid_index* idx, cudaStream_t s, int64_t* out) {
 }
 }  // namespace
 
+}  // extern "C"
+
+namespace {
+// Replay of a captured search (the launch-bound small-batch path pays one graph launch instead of
+// ~5 kernel / memset submissions).  A call shape (buffers, n, B, k) is captured on its second
+// occurrence (the first sizes every workspace), on the index's own non-blocking stream, joined to
+// the caller's stream by events; the graph is replayed while the index generation (references,
+// deleted flags, tuning) and every workspace pointer it baked in are unchanged.
+std::vector<void*> graph_ws(const tid_index* idx) {
+  return {idx->ws_q.p, idx->ws_nq.p, idx->ws_nvalid.p, idx->ws_counts.p, idx->ws_cand.p, idx->ws_qs.p,
+          idx->dead_dev.p};
+}
+
+template <class Enqueue>
+tid_status search_graph(tid_index* idx, const void* q, const void* nq, int32_t n, int64_t B, int32_t k, void* ids,
+                        void* cnts, cudaStream_t s, Enqueue& enqueue) {
+  const std::vector<void*> ws = graph_ws(idx);
+  tid_index::GraphEntry* e = nullptr;
+  for (auto& ge : idx->graphs)
+    if (ge.q == q && ge.nq == nq && ge.ids == ids && ge.cnts == cnts && ge.n == n && ge.k == k && ge.B == B) {
+      e = &ge;
+      break;
+    }
+  if (e && (e->gen != idx->gen || e->ws != ws)) {  // stale: drop the graph, start over
+    if (e->exec) cudaGraphExecDestroy(e->exec);
+    e->exec = nullptr;
+    e->uses = 0;
+    e->gen = idx->gen;
+    e->ws = ws;
+  }
+  if (!e) {
+    if (idx->graphs.size() >= 8) {  // small cache: evict the oldest
+      if (idx->graphs.front().exec) cudaGraphExecDestroy(idx->graphs.front().exec);
+      idx->graphs.erase(idx->graphs.begin());
+    }
+    tid_index::GraphEntry ne;
+    ne.q = q; ne.nq = nq; ne.ids = ids; ne.cnts = cnts; ne.n = n; ne.k = k; ne.B = B;
+    ne.gen = idx->gen;
+    ne.ws = ws;
+    idx->graphs.push_back(ne);
+    e = &idx->graphs.back();
+  }
+  if (e->uses < 0 || ++e->uses < 2) return enqueue(s);  // first occurrence (or not capturable): direct
+  CU(cudaEventRecord(idx->ev_gin, s));
+  CU(cudaStreamWaitEvent(idx->graph_stream, idx->ev_gin, 0));
+  if (!e->exec) {
+    CU(cudaStreamBeginCapture(idx->graph_stream, cudaStreamCaptureModeThreadLocal));
+    const tid_status st = enqueue(idx->graph_stream);
+    cudaGraph_t g = nullptr;
+    const cudaError_t ce = cudaStreamEndCapture(idx->graph_stream, &g);
+    cudaGraphExec_t exec = nullptr;
+    const bool ok = st == TID_OK && ce == cudaSuccess && g && cudaGraphInstantiate(&exec, g, 0) == cudaSuccess;
+    if (g) cudaGraphDestroy(g);
+    if (!ok || graph_ws(idx) != ws) {  // not capturable (or a workspace moved): direct from now on
+      cudaGetLastError();
+      if (exec) cudaGraphExecDestroy(exec);
+      e->uses = -1;
+      CU(cudaEventRecord(idx->ev_gout, idx->graph_stream));
+      CU(cudaStreamWaitEvent(s, idx->ev_gout, 0));
+      return enqueue(s);
+    }
+    e->exec = exec;
+  }
+  CU(cudaGraphLaunch(e->exec, idx->graph_stream));
+  CU(cudaEventRecord(idx->ev_gout, idx->graph_stream));
+  CU(cudaStreamWaitEvent(s, idx->ev_gout, 0));
+  return TID_OK;
+}
+}  // namespace
+
+extern "C" {
+
 tid_status tid_search(tid_index* idx, const uint8_t* queries, const int32_t* n_q, int32_t n, int64_t B, int32_t k,
                       int64_t* ref_ids_out, int32_t* match_counts_out, void* stream) {
   TRY(check_search_args(idx, queries, n, B));
@@ -1327,9 +1427,6 @@ tid_status tid_search(tid_index* idx, const uint8_t* queries, const int32_t* n_q
   if (R_total == 0) return fail(TID_ESTATE, "index holds no references");
   if (k > R_total)
     return fail(TID_EINVAL, "k=%d exceeds the number of references (%lld)", k, static_cast<long long>(R_total));
-  const uint8_t* dq = nullptr;
-  const int32_t* dnv = nullptr;
-  TRY(stage_queries(idx, queries, n_q, n, B, &dq, &dnv, s));
   TRY(sync_dead(idx, s));
   TRY(idx->ws_ids.ensure(static_cast<size_t>(B) * k * 8, "ids"));
   TRY(idx->ws_cnts.ensure(static_cast<size_t>(B) * k * 4, "counts"));
@@ -1339,6 +1436,12 @@ tid_status tid_search(tid_index* idx, const uint8_t* queries, const int32_t* n_q
   const bool collective = idx->comm != nullptr;
   if (collective) TRY(idx->ws_keys.ensure(static_cast<size_t>(B) * k * 8, "local keys"));
   uint64_t* local_keys = collective ? idx->ws_keys.as<uint64_t>() : nullptr;
+  // everything from query staging to the final ranking, enqueued on stream st (also the body of a
+  // captured CUDA graph: device-only work, no host synchronisation)
+  auto enqueue = [&](cudaStream_t st) -> tid_status {
+  const uint8_t* dq = nullptr;
+  const int32_t* dnv = nullptr;
+  TRY(stage_queries(idx, queries, n_q, n, B, &dq, &dnv, st));
   if (R > 0) {
     // a6: per window, per-(query, segment) top-k of the window's counts, then merge.  One window:
     // merge the segments straight into the result (one segment, no comm: the top-k kernel
@@ -1354,7 +1457,7 @@ tid_status tid_search(tid_index* idx, const uint8_t* queries, const int32_t* n_q
     TRY(idx->ws_cand.ensure(static_cast<size_t>(B) * lists * k * 8, "top-k candidates"));
     TRY(idx->ws_counts.ensure(static_cast<size_t>(B) * W * 4, "count window"));
     uint64_t* cand = idx->ws_cand.as<uint64_t>();
-    if (nwin > 1) CU(cudaMemsetAsync(cand, 0, static_cast<size_t>(B) * lists * k * 8, s));  // empty running lists
+    if (nwin > 1) CU(cudaMemsetAsync(cand, 0, static_cast<size_t>(B) * lists * k * 8, st));  // empty running lists
     const uint8_t* dead = idx->any_dead ? idx->dead_dev.as<uint8_t>() : nullptr;
     uint32_t* counts = idx->ws_counts.as<uint32_t>();
     auto on_window = [&](int64_t w0, int64_t wlen) -> tid_status {
@@ -1362,40 +1465,50 @@ tid_status tid_search(tid_index* idx, const uint8_t* queries, const int32_t* n_q
       const bool last = w0 + wlen >= R;
       if (nwin == 1) {
         const bool direct = !collective && segs == 1;
-        launch_topk(counts, B, wlen, W, idx->cfg.id_base + w0, k, segs, dead, cand, lists, 0, s,
+        launch_topk(counts, B, wlen, W, idx->cfg.id_base + w0, k, segs, dead, cand, lists, 0, st,
                     direct ? ids : nullptr, direct ? cnts : nullptr);
         count_kernel(idx);
         if (!direct) {
           launch_merge(cand, segs, B, k, static_cast<int64_t>(lists) * k, k, local_keys, collective ? nullptr : ids,
-                       collective ? nullptr : cnts, s);
+                       collective ? nullptr : cnts, st);
           count_kernel(idx);
         }
       } else {
-        launch_topk(counts, B, wlen, W, idx->cfg.id_base + w0, k, segs, dead ? dead + w0 : nullptr, cand, lists, 1, s);
+        launch_topk(counts, B, wlen, W, idx->cfg.id_base + w0, k, segs, dead ? dead + w0 : nullptr, cand, lists, 1, st);
         // running top-k (list 0) + this window's segments -> list 0, or the result after the last window
         if (!last) {
-          launch_merge(cand, 1 + segs, B, k, static_cast<int64_t>(lists) * k, k, cand, nullptr, nullptr, s,
+          launch_merge(cand, 1 + segs, B, k, static_cast<int64_t>(lists) * k, k, cand, nullptr, nullptr, st,
                        static_cast<int64_t>(lists) * k);
         } else {
           launch_merge(cand, 1 + segs, B, k, static_cast<int64_t>(lists) * k, k, local_keys, collective ? nullptr : ids,
-                       collective ? nullptr : cnts, s);
+                       collective ? nullptr : cnts, st);
         }
         count_kernel(idx, 2);
       }
       return TID_OK;
     };
-    TRY(run_pass(idx, dq, dnv, n, B, W, counts, s, on_window));
+    TRY(run_pass(idx, dq, dnv, n, B, W, counts, st, on_window));
   } else {
     // empty shard (collective only): contribute empty candidate lists to the all-gather
-    CU(cudaMemsetAsync(local_keys, 0, static_cast<size_t>(B) * k * 8, s));
+    CU(cudaMemsetAsync(local_keys, 0, static_cast<size_t>(B) * k * 8, st));
   }
   if (collective) {
     // a9: local top-k -> NCCL all-gather over NVLink -> identical merge on every rank
     const int G = idx->cfg.world_size;
     TRY(idx->ws_gather.ensure(static_cast<size_t>(G) * B * k * 8, "gathered keys"));
-    NC(nccl().AllGather(local_keys, idx->ws_gather.p, static_cast<size_t>(B) * k, ncclUint64, idx->comm, s));
-    launch_merge(idx->ws_gather.as<uint64_t>(), G, B, k, k, B * k, nullptr, ids, cnts, s);
+    NC(nccl().AllGather(local_keys, idx->ws_gather.p, static_cast<size_t>(B) * k, ncclUint64, idx->comm, st));
+    launch_merge(idx->ws_gather.as<uint64_t>(), G, B, k, k, B * k, nullptr, ids, cnts, st);
     count_kernel(idx);
+  }
+  return TID_OK;
+  };
+  // graph path: device queries / outputs, HBM-resident references, no collective, not profiling
+  const bool graphable = !collective && idx->n_host == 0 && !idx->prof && dev_ids && dev_cnt &&
+                         is_device_ptr(queries) && (!n_q || is_device_ptr(n_q));
+  if (graphable) {
+    TRY(search_graph(idx, queries, n_q, n, B, k, ids, cnts, s, enqueue));
+  } else {
+    TRY(enqueue(s));
   }
   CU(cudaGetLastError());
   bool host_out = false;
@@ -1740,6 +1853,7 @@ tid_status tid_set_tuning(tid_index* idx, const tid_tuning* t) {
   if (t->host_chunk_refs < 0) return fail(TID_EINVAL, "host_chunk_refs < 0");
   if (t->window_refs < 0) return fail(TID_EINVAL, "window_refs < 0");
   idx->tune = *t;
+  ++idx->gen;
   if (t->host_chunk_refs > 0) idx->host_chunk = t->host_chunk_refs;
   return TID_OK;
 }

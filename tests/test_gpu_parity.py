@@ -594,3 +594,47 @@ def test_hbm_capacity_per_reference(tid):
         assert cap >= 4_900_000, cap
     with tid.Index(ref_kp=384) as idx:
         assert idx.info()["hbm_bytes_per_reference"] == 384 * 128 + 2048
+
+
+def test_search_graph_replay_tracks_index_changes(tid):
+    """Repeated device-buffer searches are replayed from a captured CUDA graph (second occurrence of
+    a call shape); any change of the index (add, delete, tuning) must invalidate it: every result
+    equals the oracle on the index as it is at that call."""
+    import torch
+    R, m, n, B, k = 40, 256, 300, 2, 4
+    refs, _ = tidgen.refs(0, R + 10, m)
+    qs, _ = tidgen.queries(0, B, n, R_total=R, m=m, n_planted=60)
+    dq = torch.from_numpy(qs).cuda()
+    ids = torch.empty((B, k), dtype=torch.int64, device="cuda")
+    cnt = torch.empty((B, k), dtype=torch.int32, device="cuda")
+
+    def check(nref, dead=()):
+        c = oracle.search_counts(qs, refs[:nref])
+        for d in dead:
+            c[:, d] = -1
+        e_ids, e_cnt = oracle.np_rank(c, k)
+        np.testing.assert_array_equal(ids.cpu().numpy(), e_ids)
+        np.testing.assert_array_equal(cnt.cpu().numpy(), e_cnt)
+
+    with tid.Index(ref_kp=m) as idx:
+        idx.add_references(refs[:R])
+        for _ in range(4):  # direct, capture, replay, replay
+            ids.fill_(-7)
+            idx.search(dq, k, out=(ids, cnt))
+            torch.cuda.synchronize()
+            check(R)
+        idx.add_references(refs[R:])
+        for _ in range(3):
+            idx.search(dq, k, out=(ids, cnt))
+            torch.cuda.synchronize()
+            check(R + 10)
+        idx.delete([0, 7])
+        for _ in range(3):
+            idx.search(dq, k, out=(ids, cnt))
+            torch.cuda.synchronize()
+            check(R + 10, dead=(0, 7))
+        idx.set_tuning(window_refs=9)
+        for _ in range(3):
+            idx.search(dq, k, out=(ids, cnt))
+            torch.cuda.synchronize()
+            check(R + 10, dead=(0, 7))
