@@ -1348,8 +1348,8 @@ namespace {
 // the caller's stream by events; the graph is replayed while the index generation (references,
 // deleted flags, tuning) and every workspace pointer it baked in are unchanged.
 std::vector<void*> graph_ws(const tid_index* idx) {
-  return {idx->ws_q.p, idx->ws_nq.p, idx->ws_nvalid.p, idx->ws_counts.p, idx->ws_cand.p, idx->ws_qs.p,
-          idx->dead_dev.p};
+  return {idx->ws_q.p,     idx->ws_nq.p,    idx->ws_nvalid.p, idx->ws_counts.p, idx->ws_cand.p,
+          idx->ws_qs.p,    idx->dead_dev.p, idx->ws_f16q.p,   idx->ws_f16nq.p,  idx->ws_f16c.p};
 }
 
 template <class Enqueue>

@@ -116,3 +116,27 @@ def test_f16_index_m384_rootsift_parity(tid):
     d = np.abs(counts - want)
     assert np.mean(d <= 1) >= 0.999 and d.max() <= 2
     np.testing.assert_array_equal(ids[:, 0], tg)
+
+
+def test_f16_index_graph_replay(tid):
+    """Repeated device-buffer searches of a float index replay a captured graph: the same answer as
+    the first (direct) call, and as the index's own count matrix ranked on the host."""
+    import torch
+    R, m, n, B, k = 30, 256, 300, 2, 4
+    refs, _ = tidgen.refs(3, R, m)
+    qs, _ = tidgen.queries(3, B, n, R_total=R, m=m)
+    dq = torch.from_numpy(qs).cuda()
+    with tid.Index(ref_kp=m, descriptor="f16") as idx:
+        idx.add_references(refs)
+        c = idx.search_counts(qs).astype(np.int64)
+        outs = []
+        for _ in range(4):
+            o = (torch.empty((B, k), dtype=torch.int64, device="cuda"), torch.empty((B, k), dtype=torch.int32, device="cuda"))
+            ids, cnt = o
+            idx.search(dq, k, out=(ids, cnt))
+            torch.cuda.synchronize()
+            outs.append((ids.cpu().numpy(), cnt.cpu().numpy()))
+    e_ids, e_cnt = oracle.topk(c, k)
+    for ids, cnt in outs:
+        np.testing.assert_array_equal(ids, e_ids)
+        np.testing.assert_array_equal(cnt, e_cnt)
