@@ -130,9 +130,10 @@ def test_f16_index_graph_replay(tid):
         idx.add_references(refs)
         c = idx.search_counts(qs).astype(np.int64)
         outs = []
-        for _ in range(4):
-            o = (torch.empty((B, k), dtype=torch.int64, device="cuda"), torch.empty((B, k), dtype=torch.int32, device="cuda"))
-            ids, cnt = o
+        ids = torch.empty((B, k), dtype=torch.int64, device="cuda")
+        cnt = torch.empty((B, k), dtype=torch.int32, device="cuda")
+        for _ in range(4):  # same buffers: direct, capture, replay, replay
+            ids.fill_(-5)
             idx.search(dq, k, out=(ids, cnt))
             torch.cuda.synchronize()
             outs.append((ids.cpu().numpy(), cnt.cpu().numpy()))
