@@ -360,10 +360,13 @@ tid_status copy_out(tid_index* idx, void* dst, const void* src, size_t bytes, cu
   return TID_OK;
 }
 
-// Choose job decomposition of a search launch: refs per job G and queries per job.
-void plan_search(const tid_index* idx, int64_t n_refs, int64_t B, int T, int* G_out, int* qpj_out) {
+// Choose job decomposition of a search launch: refs per job G, queries per job, slot banks.
+// Small batches (one chunk per reference, B * T <= 16 query tiles per job) use two banks of 2 slots:
+// a job is short there, and the next job's references then load while this one runs.
+void plan_search(const tid_index* idx, int64_t n_refs, int64_t B, int T, int* G_out, int* qpj_out, int* banks_out) {
+  const int banks = (idx->cpr == 1 && B * T <= 16 && idx->tune.refs_per_job == 0) ? 2 : 1;
   // refs per job: one per epilogue group (group g <-> resident reference g), fewer for m > 256
-  const int max_g = std::min(kMaxSlots / idx->cpr, kNG);
+  const int max_g = std::min(kMaxSlots / banks / idx->cpr, kNG);
   int G = idx->tune.refs_per_job > 0 ? std::min(idx->tune.refs_per_job, max_g) : max_g;
   const int64_t target_jobs = 2LL * idx->num_sms;
   // spread small reference sets over more CTAs (fewer resident refs per job)
@@ -372,9 +375,9 @@ void plan_search(const tid_index* idx, int64_t n_refs, int64_t B, int T, int* G_
   int qpj = static_cast<int>(B);
   // still too few jobs: split the query batch too (each job then re-reads its refs)
   while (groups * ceil_div(B, qpj) < target_jobs && qpj > 1) qpj = (qpj + 1) / 2;
-  (void)T;
   *G_out = G;
   *qpj_out = qpj;
+  *banks_out = banks;
 }
 
 tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const uint8_t* rbase, int64_t map_count, int64_t ref_map_base, const int32_t* colkey, int64_t n_refs, int64_t B,
@@ -389,9 +392,10 @@ tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const ui
   p.qs = idx->ws_qs.as<uint8_t>();
   p.rdesc = rbase;
   p.m = idx->cfg.ref_kp;
-  int G, qpj;
-  plan_search(idx, n_refs, B, T, &G, &qpj);
+  int G, qpj, banks;
+  plan_search(idx, n_refs, B, T, &G, &qpj, &banks);
   p.refs_per_job = G;
+  p.slot_banks = banks;
   p.cpr = idx->cpr;
   p.tiles_per_q = T;
   p.num_q = static_cast<int32_t>(B);

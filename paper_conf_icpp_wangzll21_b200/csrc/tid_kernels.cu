@@ -596,24 +596,26 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     {
       uint32_t qctr = 0;
       uint32_t slot_par = 0;  // bit sl = phase parity of reference slot sl
-      for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
+      uint32_t jc = 0;        // this CTA's job count: slot bank (jc & 1) when p.slot_banks == 2
+      for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x, ++jc) {
         const Job J = decode_job(p, j);
         const int nslots = J.nr * cpr;
+        const int b0 = p.slot_banks == 2 ? static_cast<int>(jc & 1u) * (kMaxSlots / 2) : 0;
         if (lane == 0) {
           for (int sl = 0; sl < nslots; ++sl) {
-            PROF_B(); mbar_wait_sleep(rempty(sl), (slot_par >> sl & 1u) ^ 1); PROF_E(0);
-            mbar_expect_tx(rfull(sl), kRTileBytes + (kFold ? kColBytes : 0u));
+            PROF_B(); mbar_wait_sleep(rempty(b0 + sl), (slot_par >> (b0 + sl) & 1u) ^ 1); PROF_E(0);
+            mbar_expect_tx(rfull(b0 + sl), kRTileBytes + (kFold ? kColBytes : 0u));
             const int s = sl / cpr, c = sl % cpr;
             const int64_t ref = J.ref_first + s;
-            tma_load_3d(sbase + SmemPlan::kR + sl * kRTileBytes, &rmap, rfull(sl), 0, c * kBN,
+            tma_load_3d(sbase + SmemPlan::kR + (b0 + sl) * kRTileBytes, &rmap, rfull(b0 + sl), 0, c * kBN,
                         static_cast<int>(p.ref_map_base + ref));
             if (kFold)  // search: the stored column terms W (verify computes its keys on chip)
-              bulk_load(sbase + SmemPlan::kCol + sl * kColBytes, p.colkey + (ref * cpr + c) * kColInts, kColBytes,
-                        rfull(sl));
+              bulk_load(sbase + SmemPlan::kCol + (b0 + sl) * kColBytes, p.colkey + (ref * cpr + c) * kColInts, kColBytes,
+                        rfull(b0 + sl));
           }
         }
         __syncwarp();
-        slot_par ^= (1u << nslots) - 1u;
+        slot_par ^= ((1u << nslots) - 1u) << b0;
         const int ntiles = J.nq * T;
         if (lane == 0) {
           // TMA tile t+1 into shared memory while tile t is copied to its TMEM slot (the MMAs read A
@@ -653,23 +655,25 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     uint32_t qctr = 0;
     if (kFold) mbar_wait(axfull, 0);  // constant norm-term operand in TMEM
     uint32_t slot_par = 0;  // bit sl = phase parity of reference slot sl
-    for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
+    uint32_t jc = 0;
+    for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x, ++jc) {
       const Job J = decode_job(p, j);
       const int nslots = J.nr * cpr;
+      const int b0 = p.slot_banks == 2 ? static_cast<int>(jc & 1u) * (kMaxSlots / 2) : 0;
       const int U = J.nq * T * J.nr;
       if constexpr (kFold) {
         // the norm digits of the job's slots, expanded by the kNG MMA warps (HBM keeps only the column
         // terms W: 4 B per keypoint instead of 32 B of digits); both 16-byte halves of the constant
         // operand are equal, so the SWIZZLE_32B placement of a row's halves does not matter and rows
         // are written plainly, 32 B each
-        for (int sl = 0; sl < nslots; ++sl) mbar_wait(rfull(sl), slot_par >> sl & 1u);
+        for (int sl = 0; sl < nslots; ++sl) mbar_wait(rfull(b0 + sl), slot_par >> (b0 + sl) & 1u);
         for (int x = mw * 32 + lane; x < nslots * kBN; x += kNG * 32) {
           const int sl = x / kBN, col = x % kBN;
           int W;
-          asm volatile("ld.shared.s32 %0, [%1];" : "=r"(W) : "r"(sbase + SmemPlan::kCol + sl * kColBytes + col * 4));
+          asm volatile("ld.shared.s32 %0, [%1];" : "=r"(W) : "r"(sbase + SmemPlan::kCol + (b0 + sl) * kColBytes + col * 4));
           uint32_t w8[8];
           norm_digits(W, w8);
-          const uint32_t dst = sbase + SmemPlan::kX + sl * kXTileBytes + col * kXDim;
+          const uint32_t dst = sbase + SmemPlan::kX + (b0 + sl) * kXTileBytes + col * kXDim;
           asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst), "r"(w8[0]), "r"(w8[1]), "r"(w8[2]),
                        "r"(w8[3]) : "memory");
           asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst + 16), "r"(w8[4]), "r"(w8[5]), "r"(w8[6]),
@@ -678,7 +682,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> tensor-core reads
         __syncwarp();
         if (lane == 0)
-          for (int sl = 0; sl < nslots; ++sl) mbar_arrive(xready(sl));
+          for (int sl = 0; sl < nslots; ++sl) mbar_arrive(xready(b0 + sl));
       }
       uint32_t ready_mask = 0;
       int waited = 0, t = 0, s = 0, g = 0;
@@ -693,7 +697,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           }
           const uint32_t at = tmem_base + kTQBase + ((qctr + t) % kTQ) * kQCols;  // A (query tile) in TMEM
           for (int c = 0; c < cpr; ++c) {
-            const int sl = s * cpr + c;
+            const int sl = b0 + s * cpr + c;
             if (!(ready_mask >> sl & 1u)) {
               PROF_B(); mbar_wait(rfull(sl), (slot_par >> sl & 1u));
               // search: norm digits expanded; verify with m_r: rows beyond m_r zeroed
@@ -735,7 +739,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         if (++g == kNG) g = 0;
         if (++s == J.nr) { s = 0; ++t; }
       }
-      for (int sl = 0; sl < nslots; ++sl) {
+      for (int sl = b0; sl < b0 + nslots; ++sl) {
         if (!(ready_mask >> sl & 1u)) {  // keep rempty / xready phases ordered
           mbar_wait(rfull(sl), (slot_par >> sl & 1u));
           if (kFold || p.m_valid) mbar_wait(xready(sl), (slot_par >> sl & 1u));
@@ -762,14 +766,16 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     uint32_t ph_t = 0;                    // bit b: phase flip of TMEM buffer b (see the MMA warps)
     uint32_t v[64];
 
-    for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x) {
+    uint32_t jc = 0;
+    for (int32_t j = blockIdx.x; j < p.n_jobs; j += gridDim.x, ++jc) {
       const Job J = decode_job(p, j);
       const int nslots = J.nr * cpr;
+      const int b0 = p.slot_banks == 2 ? static_cast<int>(jc & 1u) * (kMaxSlots / 2) : 0;
       const int U = J.nq * T * J.nr;
       // column keys of every slot of the job (also orders this warp's rempty arrivals)
       const int mcap = (!kFold && p.m_valid) ? min(p.m_valid[J.ref_first], p.m) : p.m;  // issued before the wait
       PROF_B();
-      for (int sl = 0; sl < nslots; ++sl) mbar_wait(rfull(sl), slot_par >> sl & 1u);
+      for (int sl = 0; sl < nslots; ++sl) mbar_wait(rfull(b0 + sl), slot_par >> (b0 + sl) & 1u);
       if constexpr (!kFold) {
         // verify: the packed column keys N_R * 256 + i (Alg. 1 step 1) computed here from the
         // reference tile already in shared memory (no separate pass over the references in HBM).
@@ -822,7 +828,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         if constexpr (kFold) {
           int G1 = INT_MIN, G2 = INT_MIN;  // two largest folded values X over the reference
           for (int c = 0; c < cpr; ++c) {
-            const uint32_t ck = sbase + SmemPlan::kCol + (s * cpr + c) * kColBytes;
+            const uint32_t ck = sbase + SmemPlan::kCol + (b0 + s * cpr + c) * kColBytes;
             int kpc;  // real columns of this chunk: the last column term is -1 - kpc when padded
             asm volatile("ld.shared.s32 %0, [%1];" : "=r"(kpc) : "r"(ck + (kBN - 1) * 4));
             kpc = kpc < 0 ? -1 - kpc : kBN;
@@ -908,7 +914,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         } else {
         int g1d = INT_MAX, g1i = -1, g2d = INT_MAX, g2i = -1;  // running exact 2-NN over chunks
         for (int c = 0; c < cpr; ++c) {
-          const uint32_t ck = sbase + SmemPlan::kCol + (s * cpr + c) * kColBytes;
+          const uint32_t ck = sbase + SmemPlan::kCol + (b0 + s * cpr + c) * kColBytes;
           int R[16];
 #pragma unroll
           for (int b = 0; b < 16; ++b) R[b] = INT_MAX;
@@ -996,8 +1002,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
       }
       __syncwarp();
       if (lane == 0)
-        for (int sl = 0; sl < nslots; ++sl) mbar_arrive(rempty(sl));
-      slot_par ^= (1u << nslots) - 1u;
+        for (int sl = 0; sl < nslots; ++sl) mbar_arrive(rempty(b0 + sl));
+      slot_par ^= ((1u << nslots) - 1u) << b0;
     }
   }
 
