@@ -59,4 +59,15 @@ with tid.Index(ref_kp=256) as idx:
 _, onn = oracle.verify(Q, R)
 eg, ei, em = oracle.geometric(onn, qxy, rxy, iterations=64, inlier_px=5.0)
 assert np.array_equal(g.astype(np.int64), eg) and np.array_equal(inl.astype(np.int64), ei)
+# graph replay (device buffers, repeated shape) and a small batch (two slot banks)
+import torch  # noqa: E402
+with tid.Index(ref_kp=256, query_kp_max=1024) as idx:
+    idx.add_references(refs, kp)
+    dq = torch.from_numpy(qs).cuda()
+    did = torch.empty((3, 4), dtype=torch.int64, device="cuda")
+    dcn = torch.empty((3, 4), dtype=torch.int32, device="cuda")
+    for _ in range(3):
+        idx.search(dq, 4, out=(did, dcn))
+    torch.cuda.synchronize()
+assert np.array_equal(did.cpu().numpy(), e_ids)
 print("sanitize run ok")
