@@ -23,11 +23,19 @@ def tid():
     return t
 
 
+def host_rank(counts, k, id_base=0):
+    """(count desc, id asc) ranking of a count matrix the GPU produced, in plain NumPy (a property
+    check of the top-k kernel against its own counts; the oracle never sees GPU output)."""
+    counts = np.asarray(counts, np.int64)
+    ids = np.arange(counts.shape[1]) + id_base
+    order = np.lexsort((np.broadcast_to(ids, counts.shape), -counts), axis=1)[:, :k]
+    return ids[order], np.take_along_axis(counts, order, 1).astype(np.int32)
+
+
 def test_f16_index_rootsift_parity(tid):
     """RootSIFT fp16 index, 64 queries x 2,000 references: every count within +-1 of the float64
     oracle on the same fp16 values for >= 99.9 % of pairs; the planted target ranks first; the
-    returned top-k is the (count desc, id asc) ranking of the index's own count matrix; Eq. 2
-     of the GPU's own fp16 values is small."""
+    returned top-k is the (count desc, id asc) ranking of the index's own count matrix."""
     B, n, R, m, k = 64, 1000, 2000, 256, 5
     refs, _ = tidgen.refs(0, R, m)
     qs, tg = tidgen.queries(0, B, n, R_total=R, m=m)
@@ -35,20 +43,17 @@ def test_f16_index_rootsift_parity(tid):
         idx.add_references(refs)
         counts = idx.search_counts(qs).astype(np.int64)
         ids, cnt = idx.search(qs, k)
-        q16 = idx.f16_prepare(qs, True, 1.0)
-        r16 = idx.f16_prepare(refs, True, 1.0)
         info = idx.info()
     assert info["hbm_bytes_per_reference"] == m * 128 * 2 + 256 * 16 * 2
-    want = oracle.f16_search_counts_c(q16, r16).astype(np.int64)
+    # the oracle end to end on the same u8 inputs: its own RootSIFT -> fp16, its own float64 counts
+    want = oracle.f16_search_counts_c(oracle.to_fp16(oracle.rootsift(qs)), oracle.to_fp16(oracle.rootsift(refs)))
+    want = want.astype(np.int64)
     d = np.abs(counts - want)
     assert np.mean(d <= 1) >= 0.999 and d.max() <= 2, (np.mean(d <= 1), d.max())
     np.testing.assert_array_equal(ids[:, 0], tg)
-    e_ids, e_cnt = oracle.topk(counts, k)
+    e_ids, e_cnt = host_rank(counts, k)
     np.testing.assert_array_equal(ids, e_ids)
     np.testing.assert_array_equal(cnt, e_cnt)
-    rq, rr = oracle.rootsift(qs[0, :300]), oracle.rootsift(refs[0])
-    e = oracle.compression_error(rq, rr, q16[0, :300].astype(np.float64), r16[0].astype(np.float64))
-    assert 0 < e < 1e-3
 
 
 @pytest.mark.parametrize("host,m", [(False, 200), (True, 200), (False, 384), (True, 500)])
@@ -111,8 +116,8 @@ def test_f16_index_m384_rootsift_parity(tid):
         idx.add_references(refs)
         counts = idx.search_counts(qs).astype(np.int64)
         ids, _ = idx.search(qs, 3)
-        q16, r16 = idx.f16_prepare(qs, True, 1.0), idx.f16_prepare(refs, True, 1.0)
-    want = oracle.f16_search_counts_c(q16, r16).astype(np.int64)
+    want = oracle.f16_search_counts_c(oracle.to_fp16(oracle.rootsift(qs)), oracle.to_fp16(oracle.rootsift(refs)))
+    want = want.astype(np.int64)
     d = np.abs(counts - want)
     assert np.mean(d <= 1) >= 0.999 and d.max() <= 2
     np.testing.assert_array_equal(ids[:, 0], tg)
@@ -137,7 +142,7 @@ def test_f16_index_graph_replay(tid):
             idx.search(dq, k, out=(ids, cnt))
             torch.cuda.synchronize()
             outs.append((ids.cpu().numpy(), cnt.cpu().numpy()))
-    e_ids, e_cnt = oracle.topk(c, k)
+    e_ids, e_cnt = host_rank(c, k)
     for ids, cnt in outs:
         np.testing.assert_array_equal(ids, e_ids)
         np.testing.assert_array_equal(cnt, e_cnt)
