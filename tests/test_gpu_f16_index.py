@@ -146,3 +146,31 @@ def test_f16_index_graph_replay(tid):
     for ids, cnt in outs:
         np.testing.assert_array_equal(ids, e_ids)
         np.testing.assert_array_equal(cnt, e_cnt)
+
+
+def test_f16_index_lifecycle(tid, tmp_path):
+    """Float index lifecycle: delete / update in place and the FIFO hybrid cache behave like the u8
+    index (exact on u8 x 2^-7); save / load are refused (TID_EUNSUPPORTED: the persisted format is
+    the u8 one)."""
+    R, m, n, B, k = 24, 256, 200, 2, 5
+    s = 2.0 ** -7
+    refs, _ = tidgen.refs(0, R + 4, m)
+    qs, _ = tidgen.queries(0, B, n, R_total=R, m=m, n_planted=50)
+    rb = m * 256
+    with tid.Index(ref_kp=m, descriptor="f16", f16_rootsift=False, f16_scale=s, hbm_budget_bytes=8 * rb,
+                   host_budget_bytes=64 * rb, cache_policy="fifo") as idx:
+        for b0 in range(0, R, 6):  # FIFO: every batch enters HBM, the oldest move to the host tier
+            idx.add_references(refs[b0:b0 + 6])
+        info = idx.info()
+        assert info["hbm_references"] <= 8 and info["host_references"] >= R - 8
+        idx.delete([3])
+        idx.update([5, 20], refs[R:R + 2])  # one in the host tier, one in HBM
+        counts = idx.search_counts(qs).astype(np.int64)
+        with pytest.raises(tid.TidError) as e:
+            idx.save(str(tmp_path / "f.tidx"))
+        assert e.value.status == tid.TID_EUNSUPPORTED
+    cur = refs[:R].copy()
+    cur[5], cur[20] = refs[R], refs[R + 1]
+    want = oracle.search_counts(qs, cur)
+    want[:, 3] = 0
+    np.testing.assert_array_equal(counts, want)
