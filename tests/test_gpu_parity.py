@@ -638,3 +638,25 @@ def test_search_graph_replay_tracks_index_changes(tid):
             idx.search(dq, k, out=(ids, cnt))
             torch.cuda.synchronize()
             check(R + 10, dead=(0, 7))
+
+
+@pytest.mark.parametrize("n,m", [(2000, 700), (4100, 256)])
+def test_large_query_budgets(tid, n, m):
+    """Query keypoint budgets beyond the paper's (n = 2000, 4100: 16 / 33 query tiles) against
+    references of 3 chunks (m = 700) and 1 chunk: search counts, top-k and verify (d1, i1, d2, i2)
+    equal the oracle bit for bit."""
+    R, B, k = 7, 2, 3
+    refs, _ = tidgen.refs(0, R, m)
+    qs, _ = tidgen.queries(0, B, n, R_total=R, m=m, n_planted=min(200, m))
+    with tid.Index(ref_kp=m, query_kp_max=8192) as idx:
+        idx.add_references(refs)
+        counts = idx.search_counts(qs)
+        ids, cnt = idx.search(qs, k)
+        vc, nn = idx.verify(qs, refs[:B])
+    e_ids, e_cnt, e_counts = oracle.search(qs, refs, k)
+    np.testing.assert_array_equal(counts.astype(np.int64), e_counts)
+    np.testing.assert_array_equal(ids, e_ids)
+    np.testing.assert_array_equal(cnt, e_cnt)
+    ec, enn = oracle.verify(qs, refs[:B])
+    np.testing.assert_array_equal(vc.astype(np.int64), ec)
+    np.testing.assert_array_equal(nn.astype(np.int64), nn_from_oracle(enn))
