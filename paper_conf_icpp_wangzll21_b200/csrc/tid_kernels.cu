@@ -926,20 +926,21 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             const uint32_t buf = g * kNB + (pp & 1);
             PROF_B(); mbar_wait(tfull(buf), ((pp >> 1) ^ (ph_t >> (pp & 1))) & 1); PROF_E(0);
             tc_fence_after();
-            // x64 loads; the buffer is released as soon as its last load has landed
+            // x32 loads (32 registers live instead of 64: the verify epilogue also carries the running
+            // 2-NN with indices); the buffer is released as soon as its last load has landed
+            uint32_t (&h32)[32] = *reinterpret_cast<uint32_t(*)[32]>(v);
 #pragma unroll
-            for (int h = 0; h < kPiece / 64; ++h) {
-              tmem_ld64(taddr_q + buf * kPiece + h * 64, v);
+            for (int h = 0; h < kPiece / 32; ++h) {
+              tmem_ld32(taddr_q + buf * kPiece + h * 32, h32);
               tmem_wait_ld();
-              reg_fence64(v);
-              if (h == kPiece / 64 - 1) {
+              reg_fence(h32);
+              if (h == kPiece / 32 - 1) {
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(tempty(buf));
               }
               PROF_B();
-              scan32_regs(v, ck + (pp * kPiece + h * 64) * 4, R, T1, T2);
-              scan32_regs(v + 32, ck + (pp * kPiece + h * 64 + 32) * 4, R, T1, T2);
+              scan32_regs(h32, ck + (pp * kPiece + h * 32) * 4, R, T1, T2);
               PROF_E(1);
             }
           }
