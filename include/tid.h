@@ -182,6 +182,8 @@ tid_status tid_search_counts(tid_index* idx, const uint8_t* queries, const int32
  *            squared distances and reference-keypoint indices of the two nearest
  *            neighbours (Alg. 1 step 8's 2 x n output); a missing
  *            neighbour (m_r < 2) is (-1, -1).  Rows >= n_q[p] are not written.
+ * Without nn_out the counts come from the search path's folded kernel run on the pairs (same exact
+ * results).
  */
 tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t* r, int32_t m,
                       int64_t P, const int32_t* n_q, const int32_t* m_r,

@@ -1552,8 +1552,17 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
     TRY(copy_in(idx, idx->ws_mr.p, m_r, static_cast<size_t>(P) * 4, s));
     dmr = idx->ws_mr.as<int32_t>();
   }
+  // counts only: the search path's folded kernel in pair mode (s8 x u8 + the norm K-step, no per-element
+  // key arithmetic; column terms and digits computed on chip) — exact like the packed-key kernel, which
+  // remains the path that also returns (d1, i1, d2, i2).  TID_VERIFY_FOLD=0 disables it (A/B).
+  static const bool fold_ok = [] {
+    const char* e = getenv("TID_VERIFY_FOLD");
+    return !(e && e[0] == '0');
+  }();
+  const bool fold = fold_ok && nn_out == nullptr;
   TRY(idx->ws_nq.ensure(static_cast<size_t>(P) * T * kBM * 4, "query norms"));
-  launch_query_prep(dq, P, n, T, idx->ws_nq.as<int32_t>(), nullptr, s);
+  if (fold) TRY(idx->ws_qs.ensure(static_cast<size_t>(P) * n * kDim, "shifted queries"));
+  launch_query_prep(dq, P, n, T, idx->ws_nq.as<int32_t>(), fold ? idx->ws_qs.as<uint8_t>() : nullptr, s);
   count_kernel(idx);
   const bool dev_counts = is_device_ptr(counts_out);
   TRY(idx->ws_counts.ensure(static_cast<size_t>(P) * 4, "pair counts"));
@@ -1570,7 +1579,7 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
     }
   }
   CUtensorMap qmap, rmap;
-  TRY(make_map(&qmap, dq, P, n, kBM));
+  TRY(make_map(&qmap, fold ? idx->ws_qs.p : dq, P, n, kBM));
   TRY(make_map(&rmap, dr, P, m, kBN));
   MatchParams p{};
   p.mode = kModeVerify;
@@ -1610,7 +1619,12 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
     ++idx->prof_used;
     CU(cudaEventRecord(e0, s));
   }
-  cudaError_t e = launch_match(p, qmap, rmap, false, grid, s);
+  if (fold) {
+    p.qs = idx->ws_qs.as<uint8_t>();  // exact recompute of the rare +-1-undecided rows
+    p.rdesc = dr;
+    p.slot_banks = 1;
+  }
+  cudaError_t e = launch_match(p, qmap, rmap, fold, grid, s);
   if (e != cudaSuccess) return fail(TID_ECUDA, "match kernel launch: %s", cudaGetErrorString(e));
   if (idx->prof) {
     CU(cudaEventRecord(e1, s));

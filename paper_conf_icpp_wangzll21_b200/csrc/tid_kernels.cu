@@ -441,15 +441,19 @@ __device__ __forceinline__ uint32_t dp4a_su(uint32_t a_s8, uint32_t b_u8, uint32
 // Exact 2-NN distances (d1 <= d2) of one query row against one reference, straight from global
 // memory (the rare rows whose ratio decision the folded +-1 leaves open).  Whole warp; the
 // result is valid in every lane.  d = N_Q - 2 q'.r - W (column term W, < 0 marks padding).
+// W comes from the reference's column terms in shared memory (ck0 = its first chunk's 1 KiB; the
+// chunks of one reference occupy consecutive slots): the copy of the stored W (search) or the terms
+// the kernel computed from the tile (folded verification).
 __device__ __forceinline__ void exact_row_global(const MatchParams& p, int qi, int row, int64_t ref, int32_t nqv,
-                                                 int lane, int cpr, int& d1, int& d2) {
+                                                 int lane, int cpr, uint32_t ck0, int& d1, int& d2) {
   const uint4* qrow = reinterpret_cast<const uint4*>(p.qs + (static_cast<int64_t>(qi) * p.n_rows + row) * kDim);
   uint4 q[8];
 #pragma unroll
   for (int w = 0; w < 8; ++w) q[w] = qrow[w];
   int a1 = INT_MAX, a2 = INT_MAX;
   for (int col = lane; col < cpr * kBN; col += 32) {
-    const int32_t W = p.colkey[ref * cpr * kColInts + col];
+    int32_t W;
+    asm volatile("ld.shared.s32 %0, [%1];" : "=r"(W) : "r"(ck0 + col * 4));
     if (col >= p.m || W < 0) continue;
     const uint4* rr = reinterpret_cast<const uint4*>(p.rdesc + ((p.ref_map_base + ref) * p.m + col) * kDim);
     uint32_t dot = 0;
@@ -515,6 +519,54 @@ __device__ __forceinline__ void norm_digits(int32_t W, uint32_t (&w8)[8]) {
   w8[7] = __byte_perm(rk[6], rk[7], 0x6543) & 0x00FFFFFFu;  // ranks 27..29, position 31 = 0
 }
 
+// Per job: the fifth MMA K-step's digits of every slot column (see norm_digits) — and, for the folded
+// verification (no stored column terms, p.colkey == nullptr), first the column terms themselves,
+// W = 256 sum r - N_R from the tile row in shared memory (the order of its 16-byte chunks is
+// irrelevant under SWIZZLE_128B), -1 - (real columns of the chunk) for padding.  Columns x = first,
+// first + stride, ... of the job's nslots slots starting at slot b0.
+__device__ __forceinline__ void expand_slot_terms(const MatchParams& p, uint32_t sbase, int b0, int nslots, int cpr,
+                                                  int mcap, int first, int stride) {
+  for (int x = first; x < nslots * kBN; x += stride) {
+    const int sl = x / kBN, col = x % kBN;
+    int W;
+    const uint32_t wa = sbase + SmemPlan::kCol + (b0 + sl) * kColBytes + col * 4;
+    if (p.colkey) {
+      asm volatile("ld.shared.s32 %0, [%1];" : "=r"(W) : "r"(wa));
+    } else {
+      // folded verification: W = 256 sum r - N_R of the tile row (order of its 16-byte chunks
+      // irrelevant under SWIZZLE_128B), -1 - (real columns of the chunk) for padding
+      const int gcol = (sl % cpr) * kBN + col;
+      if (gcol < mcap) {
+        const uint32_t row = sbase + SmemPlan::kR + (b0 + sl) * kRTileBytes + col * kDim;
+        uint32_t nr = 0, sr = 0;
+#pragma unroll
+        for (int w = 0; w < kDim / 16; ++w) {
+          const int4 x4 = lds128(row + 16 * w);
+          nr = __dp4a(static_cast<uint32_t>(x4.x), static_cast<uint32_t>(x4.x), nr);
+          nr = __dp4a(static_cast<uint32_t>(x4.y), static_cast<uint32_t>(x4.y), nr);
+          nr = __dp4a(static_cast<uint32_t>(x4.z), static_cast<uint32_t>(x4.z), nr);
+          nr = __dp4a(static_cast<uint32_t>(x4.w), static_cast<uint32_t>(x4.w), nr);
+          sr = __dp4a(static_cast<uint32_t>(x4.x), 0x01010101u, sr);
+          sr = __dp4a(static_cast<uint32_t>(x4.y), 0x01010101u, sr);
+          sr = __dp4a(static_cast<uint32_t>(x4.z), 0x01010101u, sr);
+          sr = __dp4a(static_cast<uint32_t>(x4.w), 0x01010101u, sr);
+        }
+        W = 256 * static_cast<int>(sr) - static_cast<int>(nr);
+      } else {
+        W = -1 - max(0, min(mcap - (sl % cpr) * kBN, kBN));
+      }
+      asm volatile("st.shared.s32 [%0], %1;" ::"r"(wa), "r"(W) : "memory");
+    }
+    uint32_t w8[8];
+    norm_digits(W, w8);
+    const uint32_t dst = sbase + SmemPlan::kX + (b0 + sl) * kXTileBytes + col * kXDim;
+    asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst), "r"(w8[0]), "r"(w8[1]), "r"(w8[2]),
+                 "r"(w8[3]) : "memory");
+    asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst + 16), "r"(w8[4]), "r"(w8[5]), "r"(w8[6]),
+                 "r"(w8[7]) : "memory");
+  }
+}
+
 // ------------------------------------------------------------------ fused match kernel
 // One persistent CTA per SM.  A job = (up to kNG = 3 references resident in SMEM, fewer chunks'
 // worth for m > 256) x (range of query tiles streamed through a kQStages ring; search: copied
@@ -569,7 +621,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
       mbar_init(rempty(i), kNG + kEpiWarps);
       // search: the kNG MMA warps expanded the slot's norm digits; verify: the epilogue computed the
       // keys and masked rows beyond m_r (one arrival)
-      mbar_init(xready(i), kFold ? kNG : 1);
+      mbar_init(xready(i), kFold ? (p.colkey ? kNG : kNG + kEpiWarps) : 1);
     }
     for (int i = 0; i < kTmemBufs; ++i) { mbar_init(tfull(i), 1); mbar_init(tempty(i), 4); }
     fence_barrier_init();
@@ -604,12 +656,13 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         if (lane == 0) {
           for (int sl = 0; sl < nslots; ++sl) {
             PROF_B(); mbar_wait_sleep(rempty(b0 + sl), (slot_par >> (b0 + sl) & 1u) ^ 1); PROF_E(0);
-            mbar_expect_tx(rfull(b0 + sl), kRTileBytes + (kFold ? kColBytes : 0u));
+            const bool ck_global = kFold && p.colkey != nullptr;  // else computed on chip (folded verify)
+            mbar_expect_tx(rfull(b0 + sl), kRTileBytes + (ck_global ? kColBytes : 0u));
             const int s = sl / cpr, c = sl % cpr;
             const int64_t ref = J.ref_first + s;
             tma_load_3d(sbase + SmemPlan::kR + (b0 + sl) * kRTileBytes, &rmap, rfull(b0 + sl), 0, c * kBN,
                         static_cast<int>(p.ref_map_base + ref));
-            if (kFold)  // search: the stored column terms W (verify computes its keys on chip)
+            if (ck_global)  // search: the stored column terms W (verify computes them on chip)
               bulk_load(sbase + SmemPlan::kCol + (b0 + sl) * kColBytes, p.colkey + (ref * cpr + c) * kColInts, kColBytes,
                         rfull(b0 + sl));
           }
@@ -667,18 +720,10 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         // operand are equal, so the SWIZZLE_32B placement of a row's halves does not matter and rows
         // are written plainly, 32 B each
         for (int sl = 0; sl < nslots; ++sl) mbar_wait(rfull(b0 + sl), slot_par >> (b0 + sl) & 1u);
-        for (int x = mw * 32 + lane; x < nslots * kBN; x += kNG * 32) {
-          const int sl = x / kBN, col = x % kBN;
-          int W;
-          asm volatile("ld.shared.s32 %0, [%1];" : "=r"(W) : "r"(sbase + SmemPlan::kCol + (b0 + sl) * kColBytes + col * 4));
-          uint32_t w8[8];
-          norm_digits(W, w8);
-          const uint32_t dst = sbase + SmemPlan::kX + (b0 + sl) * kXTileBytes + col * kXDim;
-          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst), "r"(w8[0]), "r"(w8[1]), "r"(w8[2]),
-                       "r"(w8[3]) : "memory");
-          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst + 16), "r"(w8[4]), "r"(w8[5]), "r"(w8[6]),
-                       "r"(w8[7]) : "memory");
-        }
+        const int mcap = p.colkey ? p.m : (p.m_valid ? min(p.m_valid[J.ref_first], p.m) : p.m);
+        // folded verification: the 3 MMA warps and the 12 epilogue warps share the work (job start)
+        if (p.colkey) expand_slot_terms(p, sbase, b0, nslots, cpr, mcap, mw * 32 + lane, kNG * 32);
+        else expand_slot_terms(p, sbase, b0, nslots, cpr, mcap, mw * 32 + lane, (kNG + kEpiWarps) * 32);
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> tensor-core reads
         __syncwarp();
         if (lane == 0)
@@ -776,6 +821,15 @@ __global__ void __launch_bounds__(kNumThreads, 1)
       const int mcap = (!kFold && p.m_valid) ? min(p.m_valid[J.ref_first], p.m) : p.m;  // issued before the wait
       PROF_B();
       for (int sl = 0; sl < nslots; ++sl) mbar_wait(rfull(b0 + sl), slot_par >> (b0 + sl) & 1u);
+      if (kFold && p.colkey == nullptr) {  // folded verification: column terms + digits, shared with the MMA warps
+        const int mcap = p.m_valid ? min(p.m_valid[J.ref_first], p.m) : p.m;
+        expand_slot_terms(p, sbase, b0, nslots, cpr, mcap, (kNG + ew) * 32 + lane, (kNG + kEpiWarps) * 32);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        __syncwarp();
+        if (lane == 0)
+          for (int sl = 0; sl < nslots; ++sl) mbar_arrive(xready(b0 + sl));
+        for (int sl = 0; sl < nslots; ++sl) mbar_wait(xready(b0 + sl), slot_par >> (b0 + sl) & 1u);
+      }
       if constexpr (!kFold) {
         // verify: the packed column keys N_R * 256 + i (Alg. 1 step 1) computed here from the
         // reference tile already in shared memory (no separate pass over the references in HBM).
@@ -907,7 +961,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             const int rl = __shfl_sync(0xffffffffu, row, l);
             const int nl = __shfl_sync(0xffffffffu, nqv, l);
             int d1, d2;
-            exact_row_global(p, qi, rl, J.ref_first + s, nl, lane, cpr, d1, d2);
+            exact_row_global(p, qi, rl, J.ref_first + s, nl, lane, cpr,
+                             sbase + SmemPlan::kCol + (b0 + s * cpr) * kColBytes, d1, d2);
             if (lane == l)
               pass = d2 != INT_MAX && uint64_t(p.den2) * uint64_t(d1) < uint64_t(p.num2) * uint64_t(d2);
           }

@@ -660,3 +660,21 @@ def test_large_query_budgets(tid, n, m):
     ec, enn = oracle.verify(qs, refs[:B])
     np.testing.assert_array_equal(vc.astype(np.int64), ec)
     np.testing.assert_array_equal(nn.astype(np.int64), nn_from_oracle(enn))
+
+
+@pytest.mark.parametrize("n,m,P", [(1000, 1000, 6), (300, 600, 5), (129, 257, 3), (200, 256, 4), (5, 2, 3)])
+def test_verify_counts_only_folded(tid, rng, n, m, P):
+    """Counts-only verification runs the folded kernel (s8 x u8 + norm K-step, column terms computed
+    on chip, the +-1-undecided rows recomputed exactly): counts equal the oracle bit for bit, also
+    with ragged n_q / m_r and adversarial pairs (ties in {0, 1, 2}, duplicates, identical rows)."""
+    Q, Rr, _ = tidgen.pairs(P, n, m, n_planted=min(200, n, m))
+    Q[1 % P, : n // 2] = rng.integers(0, 3, (n // 2, 128))
+    Rr[1 % P] = rng.integers(0, 3, (m, 128))
+    Rr[2 % P, : m // 2] = Rr[2 % P, m // 2: 2 * (m // 2)]
+    n_q = rng.integers(1, n + 1, P).astype(np.int32)
+    m_r = rng.integers(1, m + 1, P).astype(np.int32)
+    with tid.Index(ref_kp=256, query_kp_max=1024) as idx:
+        c_full, _ = idx.verify(Q, Rr, want_nn=False)
+        c_mask, _ = idx.verify(Q, Rr, n_q=n_q, m_r=m_r, want_nn=False)
+    np.testing.assert_array_equal(c_full.astype(np.int64), oracle.verify(Q, Rr, want_nn=False)[0])
+    np.testing.assert_array_equal(c_mask.astype(np.int64), oracle.verify(Q, Rr, n_q=n_q, m_r=m_r, want_nn=False)[0])
