@@ -253,32 +253,46 @@ def relaunch(n: int) -> int:
 
 def dry_run(args):
     """The multi-rank host logic of the bench on CPU (gloo): shard plan, per-rank local top-k,
-    all-gather + merge in the shared total order, max over ranks.  The per-rank matching is the
-    oracle on a tiny shard (this is a plumbing check, not a measurement)."""
+    all-gather + merge in the shared total order, max over ranks.  No matching runs here (no GPU,
+    and no CPU stand-in for the product path): each rank ranks a synthetic count row per query — a
+    fixed function of (query, global id) with the planted target on top — so the merged top-k must
+    equal the global ranking of the same function and put every planted target first."""
     import torch
     import torch.distributed as dist
 
-    import oracle
-    import tidgen
     from paper_conf_icpp_wangzll21_b200.dist import shard_plan
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     if world > 1:
         dist.init_process_group("gloo")
-    Rg, m, n, B, k = 6, 64, 80, 3, 4
-    start, end = shard_plan(Rg * world, world, rank)
-    refs, _ = tidgen.refs(start, end - start, m, seed=SEED)
-    qs, targets = tidgen.queries(0, B, n, R_total=Rg * world, m=m, n_planted=30, seed=SEED)
+    Rg, B, k = 6, 3, 4
+    R_total = Rg * world
+    start, end = shard_plan(R_total, world, rank)
+    targets = (np.arange(B) * 5 + 1) % R_total
+
+    def counts_of(ids):  # synthetic counts with many ties (id tie-break exercised), target on top
+        c = (np.arange(B)[:, None] * 7919 + ids[None, :] * 104729) % 5
+        c = c + 100 * (ids[None, :] == targets[:, None])
+        return c.astype(np.int64)
+
+    def rank_top(c, ids):  # (count desc, id asc)
+        order = np.lexsort((np.broadcast_to(ids, c.shape), -c), axis=1)[:, :k]
+        return ids[order], np.take_along_axis(c, order, 1)
+
     t0 = time.perf_counter()
-    ids, cnt = oracle.topk(oracle.search_counts(qs, refs), k, id_base=start)
+    lids = np.arange(start, end)
+    ids, cnt = rank_top(counts_of(lids), lids)
     dt = time.perf_counter() - t0
     spans = [(start, end)]
     if world > 1:
         gi = [torch.zeros((B, k), dtype=torch.int64) for _ in range(world)]
-        gc = [torch.zeros((B, k), dtype=torch.int32) for _ in range(world)]
+        gc = [torch.zeros((B, k), dtype=torch.int64) for _ in range(world)]
         dist.all_gather(gi, torch.from_numpy(ids))
         dist.all_gather(gc, torch.from_numpy(cnt))
-        ids, cnt = oracle.merge_topk(np.stack([t.numpy() for t in gi]), np.stack([t.numpy() for t in gc]))
+        all_ids = np.concatenate([t.numpy() for t in gi], 1)
+        all_cnt = np.concatenate([t.numpy() for t in gc], 1)
+        order = np.lexsort((all_ids, -all_cnt), axis=1)[:, :k]
+        ids, cnt = np.take_along_axis(all_ids, order, 1), np.take_along_axis(all_cnt, order, 1)
         sp = [None] * world
         dist.all_gather_object(sp, (start, end))
         spans = sp
@@ -286,8 +300,11 @@ def dry_run(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         dt = float(t.item())
     if rank == 0:
-        print(json.dumps({"dry_run": True, "n_gpus": world, "shards": spans, "refs_total": Rg * world,
-                          "planted_top1": float(np.mean(ids[:, 0] == targets)), "max_rank_s": dt,
+        gids = np.arange(R_total)
+        e_ids, _ = rank_top(counts_of(gids), gids)
+        print(json.dumps({"dry_run": True, "n_gpus": world, "shards": spans, "refs_total": R_total,
+                          "planted_top1": float(np.mean(ids[:, 0] == targets)),
+                          "merge_equals_global": bool(np.array_equal(ids, e_ids)), "max_rank_s": dt,
                           "top_ids": ids.tolist()}), flush=True)
     if world > 1:
         dist.destroy_process_group()
