@@ -396,6 +396,7 @@ tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const ui
   plan_search(idx, n_refs, B, T, &G, &qpj, &banks);
   p.refs_per_job = G;
   p.slot_banks = banks;
+  p.scan_one = idx->tune.scan == 2;  // automatic: the exact two-partition scan (the one-partition experiment was slower)
   p.cpr = idx->cpr;
   p.tiles_per_q = T;
   p.num_q = static_cast<int32_t>(B);
@@ -1386,9 +1387,11 @@ tid_status search_graph(tid_index* idx, const void* q, const void* nq, int32_t n
     e = &idx->graphs.back();
   }
   if (e->uses < 0 || ++e->uses < 2) return enqueue(s);  // first occurrence (or not capturable): direct
-  CU(cudaEventRecord(idx->ev_gin, s));
-  CU(cudaStreamWaitEvent(idx->graph_stream, idx->ev_gin, 0));
   if (!e->exec) {
+    // capture on the index's own stream (the caller's may be the legacy default stream, which cannot
+    // be captured), ordered after the caller's prior work
+    CU(cudaEventRecord(idx->ev_gin, s));
+    CU(cudaStreamWaitEvent(idx->graph_stream, idx->ev_gin, 0));
     CU(cudaStreamBeginCapture(idx->graph_stream, cudaStreamCaptureModeThreadLocal));
     const tid_status st = enqueue(idx->graph_stream);
     cudaGraph_t g = nullptr;
@@ -1405,10 +1408,10 @@ tid_status search_graph(tid_index* idx, const void* q, const void* nq, int32_t n
       return enqueue(s);
     }
     e->exec = exec;
+    CU(cudaEventRecord(idx->ev_gout, idx->graph_stream));  // the caller's stream waits for the capture point
+    CU(cudaStreamWaitEvent(s, idx->ev_gout, 0));
   }
-  CU(cudaGraphLaunch(e->exec, idx->graph_stream));
-  CU(cudaEventRecord(idx->ev_gout, idx->graph_stream));
-  CU(cudaStreamWaitEvent(s, idx->ev_gout, 0));
+  CU(cudaGraphLaunch(e->exec, s));  // replay straight on the caller's stream (any stream may launch a graph)
   return TID_OK;
 }
 }  // namespace
@@ -1623,6 +1626,7 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
     p.qs = idx->ws_qs.as<uint8_t>();  // exact recompute of the rare +-1-undecided rows
     p.rdesc = dr;
     p.slot_banks = 1;
+    p.scan_one = idx->tune.scan == 2;  // automatic: the exact two-partition scan (matching pairs pass often)
   }
   cudaError_t e = launch_match(p, qmap, rmap, fold, grid, s);
   if (e != cudaSuccess) return fail(TID_ECUDA, "match kernel launch: %s", cudaGetErrorString(e));
@@ -1870,6 +1874,8 @@ tid_status tid_set_tuning(tid_index* idx, const tid_tuning* t) {
   if (t->grid < 0) return fail(TID_EINVAL, "grid < 0");
   if (t->host_chunk_refs < 0) return fail(TID_EINVAL, "host_chunk_refs < 0");
   if (t->window_refs < 0) return fail(TID_EINVAL, "window_refs < 0");
+  if (t->scan < 0 || t->scan > 2) return fail(TID_EINVAL, "scan outside 0..2");
+  if (t->reserved != 0) return fail(TID_EINVAL, "reserved must be 0");
   idx->tune = *t;
   ++idx->gen;
   if (t->host_chunk_refs > 0) idx->host_chunk = t->host_chunk_refs;
