@@ -301,19 +301,12 @@ tid_status tid_get_stats(tid_index* idx, tid_stats* out); /* synchronises record
  * host-tier staging buffer; window_refs: references per count window of tid_search
  * (automatic: the whole local set while its B x R u32 count matrix fits 512 MiB, else
  * 512 MiB / (4 B) references; each window's counts are reduced into a running top-k, so the
- * search workspace does not grow with R).  scan: the epilogue of the folded (search / counts-only
- * verification) kernel — 1 = exact two-partition top-2 of every row; 2 = only the maxima of each
- * 32-column half, which prove that the ratio test fails, with the rows they cannot decide
- * recomputed exactly (about half the ALU work per element; the better choice when few rows pass,
- * as in a search over mostly unrelated references); 0 = automatic (2 for tid_search, 1 for
- * tid_verify).  reserved: must be 0.  Results never depend on these knobs. */
+ * search workspace does not grow with R).  Results never depend on these knobs. */
 typedef struct {
   int32_t refs_per_job;
   int32_t grid;
   int64_t host_chunk_refs;
   int64_t window_refs;
-  int32_t scan;
-  int32_t reserved;
 } tid_tuning;
 
 tid_status tid_set_tuning(tid_index* idx, const tid_tuning* t);

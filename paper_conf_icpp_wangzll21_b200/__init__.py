@@ -66,7 +66,7 @@ class GeomParams(ctypes.Structure):
 
 class Tuning(ctypes.Structure):
     _fields_ = [("refs_per_job", ctypes.c_int32), ("grid", ctypes.c_int32), ("host_chunk_refs", ctypes.c_int64),
-                ("window_refs", ctypes.c_int64), ("scan", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("window_refs", ctypes.c_int64)]
 
 
 _lib = None
@@ -385,9 +385,8 @@ class Index:
         _check(self._lib.tid_get_stats(self._h, ctypes.byref(s)))
         return {f: getattr(s, f) for f, _ in Stats._fields_}
 
-    def set_tuning(self, refs_per_job: int = 0, grid: int = 0, host_chunk_refs: int = 0, window_refs: int = 0,
-                   scan: int = 0):
-        t = Tuning(refs_per_job, grid, host_chunk_refs, window_refs, scan, 0)
+    def set_tuning(self, refs_per_job: int = 0, grid: int = 0, host_chunk_refs: int = 0, window_refs: int = 0):
+        t = Tuning(refs_per_job, grid, host_chunk_refs, window_refs)
         _check(self._lib.tid_set_tuning(self._h, ctypes.byref(t)))
 
 

@@ -396,7 +396,6 @@ tid_status launch_search_range(tid_index* idx, const CUtensorMap& qmap, const ui
   plan_search(idx, n_refs, B, T, &G, &qpj, &banks);
   p.refs_per_job = G;
   p.slot_banks = banks;
-  p.scan_one = idx->tune.scan == 2;  // automatic: the exact two-partition scan (the one-partition experiment was slower)
   p.cpr = idx->cpr;
   p.tiles_per_q = T;
   p.num_q = static_cast<int32_t>(B);
@@ -1626,7 +1625,6 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
     p.qs = idx->ws_qs.as<uint8_t>();  // exact recompute of the rare +-1-undecided rows
     p.rdesc = dr;
     p.slot_banks = 1;
-    p.scan_one = idx->tune.scan == 2;  // automatic: the exact two-partition scan (matching pairs pass often)
   }
   cudaError_t e = launch_match(p, qmap, rmap, fold, grid, s);
   if (e != cudaSuccess) return fail(TID_ECUDA, "match kernel launch: %s", cudaGetErrorString(e));
@@ -1874,8 +1872,6 @@ tid_status tid_set_tuning(tid_index* idx, const tid_tuning* t) {
   if (t->grid < 0) return fail(TID_EINVAL, "grid < 0");
   if (t->host_chunk_refs < 0) return fail(TID_EINVAL, "host_chunk_refs < 0");
   if (t->window_refs < 0) return fail(TID_EINVAL, "window_refs < 0");
-  if (t->scan < 0 || t->scan > 2) return fail(TID_EINVAL, "scan outside 0..2");
-  if (t->reserved != 0) return fail(TID_EINVAL, "reserved must be 0");
   idx->tune = *t;
   ++idx->gen;
   if (t->host_chunk_refs > 0) idx->host_chunk = t->host_chunk_refs;

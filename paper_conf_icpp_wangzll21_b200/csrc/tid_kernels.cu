@@ -6,7 +6,7 @@
 
 // Timing-experiment switches that skip work and give WRONG results (skeleton timings in DESIGN.md):
 // refused unless the build says it is an experiment.
-#if (defined(TID_NOSCAN) || defined(TID_NOMMA) || defined(TID_NOLOAD) || defined(TID_NOFB)) && !defined(TID_EXPERIMENT)
+#if (defined(TID_NOSCAN) || defined(TID_NOMMA) || defined(TID_NOLOAD)) && !defined(TID_EXPERIMENT)
 #error "TID_NOSCAN / TID_NOMMA / TID_NOLOAD skip work (wrong results): timing experiments only, add -DTID_EXPERIMENT"
 #endif
 
@@ -25,29 +25,6 @@ __device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
 __device__ __forceinline__ void mbar_arrive(uint32_t bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }
-#ifdef TID_WATCHDOG
-__device__ unsigned long long g_watch[64] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 42};
-__device__ __forceinline__ void mbar_wait_wd(uint32_t bar, uint32_t parity, int tag, int a, int b) {
-  for (long long it = 0;; ++it) {
-    uint32_t done;
-    asm volatile("{\n\t.reg .pred P1;\n\tmbarrier.test_wait.parity.shared::cta.b64 P1, [%1], %2;\n\tselp.u32 %0, 1, 0, P1;\n\t}"
-                 : "=r"(done) : "r"(bar), "r"(parity) : "memory");
-    if (done) return;
-    if (it == (1ll << 24) && (threadIdx.x & 31) == 0 && blockIdx.x == g_watch[63]) {
-      const unsigned long long k = atomicAdd(&g_watch[0], 1ull);
-      if (k < 15) {
-        g_watch[1 + 4 * k] = tag; g_watch[2 + 4 * k] = blockIdx.x * 1000 + (threadIdx.x >> 5);
-        g_watch[3 + 4 * k] = a; g_watch[4 + 4 * k] = b;
-      }
-    }
-    if (it > (1ll << 25)) return;  // give up (debug only): the kernel finishes, the record is readable
-  }
-}
-extern "C" int tid_debug_read_watch(void* host) { return (int)cudaMemcpyFromSymbol(host, g_watch, sizeof(g_watch)); }
-#define WAITD(bar, par, tag, a, b) mbar_wait_wd(bar, par, tag, a, b)
-#else
-#define WAITD(bar, par, tag, a, b) mbar_wait(bar, par)
-#endif
 __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
   asm volatile(
       "{\n\t.reg .pred P1;\n\t"
@@ -322,19 +299,13 @@ constexpr int kFirstEpiWarp = 1 + kNG;         // then 4 warps per group; lane q
 static_assert(kNumThreads <= 512, "at most 16 warps: >= 128 registers per thread");
 
 // ------------------------------------------------------------------ shared memory plan
-// kOne: rows whose ratio test the piece maxima cannot decide are settled during the warp's next unit
-// (overlapping its MMAs); per deferred row the scratch holds the query row q' (128 B, by cp.async),
-// then {G1, max(G2, WL), winning half, row} and N_Q.
-constexpr int kFbRows = 4;
-constexpr uint32_t kFbBytes = kDim + 32;
 struct SmemPlan {
   static constexpr uint32_t kR = 0;                                        // kMaxSlots x 32 KiB
   static constexpr uint32_t kQ = kR + kMaxSlots * kRTileBytes;             // kQStages x 16 KiB
   static constexpr uint32_t kX = kQ + kQStages * kQTileBytes;              // kMaxSlots x 8 KiB norm-term tiles
   static constexpr uint32_t kAx = kX + kMaxSlots * kXTileBytes;            // 4 KiB constant norm-term operand
   static constexpr uint32_t kCol = kAx + kBM * kXDim;                      // kMaxSlots x 1 KiB
-  static constexpr uint32_t kFb = kCol + kMaxSlots * kColBytes;            // deferred-row scratch per epilogue warp
-  static constexpr uint32_t kBar = kFb + kEpiWarps * kFbRows * kFbBytes;   // mbarriers
+  static constexpr uint32_t kBar = kCol + kMaxSlots * kColBytes;           // mbarriers
   static constexpr uint32_t kQFull = kBar;
   static constexpr uint32_t kQEmpty = kQFull + 8 * kQStages;
   static constexpr uint32_t kRFull = kQEmpty + 8 * kQStages;
@@ -448,36 +419,6 @@ __device__ __forceinline__ void scan32_fold(const uint32_t* v, int lim, int (&R)
   T2 = max3i(T2, min(T1, hi), lo);
   T1 = max(T1, hi);
 }
-// One-partition scan (search): only the maxima of the two 32-column halves of each piece.  Over the
-// whole reference the epilogue keeps T1 = the largest X (exact), the piece wp holding it, WL = the
-// other half's maximum of that piece and T2 = the largest piece maximum outside it.  The second
-// largest X is >= max(T2, WL), so d2 <= N_Q - 2 max(T2, WL): enough to prove that the ratio test
-// fails, which is the outcome for almost every (row, reference).  The rows it cannot prove
-// (those that pass, or nearly) are settled by recomputing piece wp exactly from the reference tile
-// in shared memory (half_exact).  0.63 ALU ops per element instead of 1.16.
-template <bool kMask>
-__device__ __forceinline__ int max32_fold(const uint32_t* v, int lim) {
-  int k[32];
-#pragma unroll
-  for (int i = 0; i < 32; ++i) k[i] = (!kMask || i < lim) ? static_cast<int>(v[i]) : INT_MIN;
-  int a[10];
-#pragma unroll
-  for (int i = 0; i < 10; ++i) a[i] = max3i(k[3 * i], k[3 * i + 1], k[3 * i + 2]);
-  const int b0 = max3i(a[0], a[1], a[2]), b1 = max3i(a[3], a[4], a[5]), b2 = max3i(a[6], a[7], a[8]);
-  const int b3 = max3i(a[9], k[30], k[31]);
-  return max(max3i(b0, b1, b2), b3);
-}
-template <bool kMask>
-__device__ __forceinline__ void scan64_one(const uint32_t* v, int lim, int piece, int& T1, int& T2, int& WL, int& wp) {
-  const int x = max32_fold<kMask>(v, lim), y = max32_fold<kMask>(v + 32, lim - 32);
-  const int hi = max(x, y), lo = min(x, y);
-  const bool up = hi > T1;
-  WL = up ? lo : WL;
-  wp = up ? 2 * piece + (y > x) : wp;  // the winning 32-column half
-  T2 = max(T2, min(T1, hi));  // the previous winner piece becomes an outside piece
-  T1 = max(T1, hi);
-}
-
 __device__ __forceinline__ void finish_fold(const int (&R)[16], int T1, int T2, int& x1, int& x2) {
   int rm[4], cm[4];
 #pragma unroll
@@ -535,50 +476,6 @@ __device__ __forceinline__ void exact_row_global(const MatchParams& p, int qi, i
   }
   d1 = a1;
   d2 = a2;
-}
-
-// Exact distances of one query row (q: its shifted copy q' = q ^ 0x80) to the 32 columns of half h
-// (0..7) of the reference chunk whose tile sits at `rtile` in shared memory (SWIZZLE_128B: 16-byte
-// chunk j of tile row i is stored at chunk position j ^ (i & 7)); column terms W at `ck` (< 0 =
-// padding).  Whole warp, one column per lane; the two smallest d (INT_MAX: none) in every lane.
-__device__ __forceinline__ void half_exact(const uint4 (&q)[8], uint32_t rtile, uint32_t ck, int h, int32_t nqv,
-                                           int lane, int& d1, int& d2) {
-  const int i = h * 32 + lane;
-  int32_t W;
-  asm volatile("ld.shared.s32 %0, [%1];" : "=r"(W) : "r"(ck + i * 4));
-  const uint32_t rrow = rtile + i * kDim;
-  uint32_t acc[4] = {0, 0, 0, 0};  // four independent dp4a chains
-#pragma unroll
-  for (int j = 0; j < 8; ++j) {
-    const int4 x = lds128(rrow + ((j ^ (i & 7)) << 4));
-    acc[0] = dp4a_su(q[j].x, static_cast<uint32_t>(x.x), acc[0]);
-    acc[1] = dp4a_su(q[j].y, static_cast<uint32_t>(x.y), acc[1]);
-    acc[2] = dp4a_su(q[j].z, static_cast<uint32_t>(x.z), acc[2]);
-    acc[3] = dp4a_su(q[j].w, static_cast<uint32_t>(x.w), acc[3]);
-  }
-  const int dot = static_cast<int>(acc[0] + acc[1] + acc[2] + acc[3]);
-  const int d = W < 0 ? INT_MAX : nqv - 2 * dot - W;
-  d1 = __reduce_min_sync(0xffffffffu, d);
-  const uint32_t eq = __ballot_sync(0xffffffffu, d == d1);
-  d2 = __reduce_min_sync(0xffffffffu, lane == __ffs(eq) - 1 ? INT_MAX : d);
-}
-
-// Settle one row of the one-partition scan from its winning half h of slot sl (whole warp): t1 = its
-// largest X, o = the largest X outside the half (o < t1: d1 lies in the half).  Returns 1 = the
-// ratio test passes, 0 = fails, 2 = still undecided (the whole reference must be recomputed).
-__device__ __forceinline__ int settle_half(const MatchParams& p, const uint4 (&q)[8], uint32_t sbase, int sl, int h,
-                                           int32_t nl, int t1, int o, int lane) {
-  if (!(o < t1)) return 2;
-  int d1, d2in;
-  half_exact(q, sbase + SmemPlan::kR + sl * kRTileBytes, sbase + SmemPlan::kCol + sl * kColBytes, h, nl, lane, d1, d2in);
-  // outside the half the best X is o: d there in [N_Q - 2 o - 1, N_Q - 2 o]
-  const int64_t o_lo = o > INT_MIN ? max(nl - 2 * o - 1, 0) : int64_t(INT_MAX);
-  const int64_t o_hi = o > INT_MIN ? nl - 2 * o : int64_t(INT_MAX);
-  const int64_t d2lo = d2in < o_lo ? int64_t(d2in) : o_lo, d2hi = d2in < o_hi ? int64_t(d2in) : o_hi;
-  if (d2hi == INT_MAX) return 0;  // a single real column: no second neighbour, no match
-  if (uint64_t(p.den2) * uint64_t(d1) < uint64_t(p.num2) * uint64_t(d2lo)) return 1;
-  if (uint64_t(p.den2) * uint64_t(d1) >= uint64_t(p.num2) * uint64_t(d2hi)) return 0;
-  return 2;
 }
 
 // Pieces of kPiece columns in a reference's last 256-column chunk that can hold real keypoints:
@@ -684,7 +581,7 @@ __device__ __forceinline__ void expand_slot_terms(const MatchParams& p, uint32_t
 // kSkip: the last chunk of every reference has fewer than 4 pieces that can hold keypoints
 // (m mod 256 in 1..192): those pieces are skipped, with the buffer phases tracked at run time;
 // otherwise every chunk is 4 pieces and the schedule is fully static.
-template <bool kFold, bool kSkip, bool kOne>
+template <bool kFold, bool kSkip>
 __global__ void __launch_bounds__(kNumThreads, 1)
     match_kernel(const __grid_constant__ CUtensorMap qmap, const __grid_constant__ CUtensorMap rmap,
                  const MatchParams p) {
@@ -778,13 +675,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           // from TMEM, so each query tile crosses the shared-memory port once, not once per piece)
           auto issue = [&](int t) {
             const uint32_t gq = qctr + t, st = gq % kQStages;
-            PROF_B();
-#ifdef TID_WATCHDOG
-            WAITD(qempty(st), ((gq / kQStages) & 1) ^ 1, 2, gq, 0);
-#else
-            mbar_wait_sleep(qempty(st), ((gq / kQStages) & 1) ^ 1);
-#endif
-            PROF_E(1);
+            PROF_B(); mbar_wait_sleep(qempty(st), ((gq / kQStages) & 1) ^ 1); PROF_E(1);
             mbar_expect_tx(qfull(st), kQTileBytes);
             tma_load_3d(sbase + SmemPlan::kQ + st * kQTileBytes, &qmap, qfull(st), 0, (t % T) * kBM, J.q_first + t / T);
           };
@@ -792,7 +683,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           for (int t = 0; t < ntiles; ++t) {
             if (t + 1 < ntiles) issue(t + 1);
             const uint32_t gq = qctr + t, st = gq % kQStages, sl = gq % kTQ;
-            WAITD(qfull(st), (gq / kQStages) & 1, 1, gq, 0);
+            mbar_wait(qfull(st), (gq / kQStages) & 1);
             mbar_wait_sleep(tqempty(sl), ((gq / kTQ) & 1) ^ 1);
             tc_fence_after();
             const uint64_t sd = smem_desc_sw128(sbase + SmemPlan::kQ + st * kQTileBytes);
@@ -845,7 +736,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           while (waited <= t) {
             const uint32_t gq = qctr + waited;
             PROF_B();
-            WAITD(tqfull(gq % kTQ), (gq / kTQ) & 1, 4, gq, u);
+            mbar_wait(tqfull(gq % kTQ), (gq / kTQ) & 1);
             PROF_E(1);
             ++waited;
           }
@@ -865,7 +756,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             for (int pp = 0; pp < kPiecesPerChunk; ++pp) {  // static buffer / phase (see the epilogue)
               if (kSkip && pp >= np) break;  // all-padding pieces of the last chunk are never computed
               const uint32_t buf = mw * kNB + (pp & 1);
-              PROF_B(); WAITD(tempty(buf), (((pp >> 1) ^ (ph_t >> (pp & 1))) & 1) ^ 1, 5, u, pp); PROF_E(0);
+              PROF_B(); mbar_wait(tempty(buf), (((pp >> 1) ^ (ph_t >> (pp & 1))) & 1) ^ 1); PROF_E(0);
               tc_fence_after();
               // rows kPiece*pp.. of the chunk: SWIZZLE_128B core groups of 8 rows x 128 B
               const uint64_t bd = bd0 + pp * (kPiece * kDim >> 4);
@@ -885,7 +776,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         if (s == J.nr - 1) {  // this warp's release of query tile t (covers all its prior MMAs)
           const uint32_t gq = qctr + t;
           if (waited <= t) {  // never touched tile t: still wait for it so the phase order holds
-            WAITD(tqfull(gq % kTQ), (gq / kTQ) & 1, 6, gq, u);
+            mbar_wait(tqfull(gq % kTQ), (gq / kTQ) & 1);
             waited = t + 1;
           }
           mma_commit(tqempty(gq % kTQ));
@@ -913,7 +804,6 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     const int quarter = warp & 3;         // TMEM lanes 32*quarter .. +31 (hardware restriction)
     const uint32_t taddr_q = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16);
     const int row_in_tile = quarter * 32 + lane;
-    const uint32_t fbuf = sbase + SmemPlan::kFb + ew * kFbRows * kFbBytes;  // kOne: deferred-row scratch
     const int nq_ld = T * kBM;
     const bool ratio32 = p.num2 <= 511u && p.den2 <= 511u;  // den^2 * d fits 32 bits (d <= 8,323,200)
     uint32_t slot_par = 0;                // bit sl = phase parity of reference slot sl
@@ -983,72 +873,6 @@ __global__ void __launch_bounds__(kNumThreads, 1)
       int nvalid = u < U ? min(p.n_valid ? p.n_valid[qi] : p.n_rows, p.n_rows) : 0;
       const int32_t* nq_row = p.nq + static_cast<int64_t>(qi) * nq_ld + row_in_tile;
       uint32_t cnt = 0;
-      // kOne: rows of this warp's previous unit awaiting their exact recompute (deferred_rows) in the
-      // warp's scratch; settled by run_deferred, their passes added to that unit's (query, reference)
-      uint32_t dmask = 0, dall = 0, dpass = 0;  // pending / deferred lanes, passes found so far
-      int d_qi = 0, d_s = 0;
-      // settle the lowest pending deferred row (whole warp); when the last one is done, add the passes
-      // to (d_qi, d_s): to the running count if that is still the current pair, else atomically
-      auto run_one = [&](int cur_qi, int cur_s, uint32_t& c_cur) {
-        if constexpr (kOne) {
-          const int l = __ffs(dmask) - 1;
-          const uint32_t slot = fbuf + __popc(dall & ((1u << l) - 1)) * kFbBytes;
-          asm volatile("cp.async.wait_all;" ::: "memory");
-          __syncwarp();
-          const int4 meta = lds128(slot + kDim);  // G1, max(G2, WL), winning half, row
-          int32_t nl;
-          asm volatile("ld.shared.s32 %0, [%1];" : "=r"(nl) : "r"(slot + kDim + 16));
-          uint4 q[8];
-#pragma unroll
-          for (int w = 0; w < 8; ++w) {
-            const int4 x = lds128(slot + 16 * w);
-            q[w] = make_uint4(x.x, x.y, x.z, x.w);
-          }
-          int r = settle_half(p, q, sbase, b0 + d_s * cpr + meta.z / (2 * kPiecesPerChunk), meta.z % (2 * kPiecesPerChunk),
-                              nl, meta.x, meta.y, lane);
-          if (r == 2) {
-#ifdef TID_PROF
-            if (lane == 0) atomicAdd(&g_prof[148 * 32 * 8 - 3], 1ull);
-#endif
-            int d1, d2;
-            exact_row_global(p, d_qi, meta.w, J.ref_first + d_s, nl, lane, cpr,
-                             sbase + SmemPlan::kCol + (b0 + d_s * cpr) * kColBytes, d1, d2);
-            r = d2 != INT_MAX && uint64_t(p.den2) * uint64_t(d1) < uint64_t(p.num2) * uint64_t(d2);
-          }
-          dpass += r == 1;
-          dmask &= dmask - 1;
-          if (dmask == 0) {
-            __syncwarp();  // the scratch may be refilled after this
-            if (dpass) {
-              if (d_qi == cur_qi && d_s == cur_s) {
-                c_cur += dpass;  // same (query, reference) as the running count: not flushed yet
-              } else if (lane == 0) {
-                const int64_t ci = (p.mode == kModeVerify) ? d_qi
-                                                           : static_cast<int64_t>(d_qi) * p.ldc + p.col0 + J.ref_first + d_s;
-                atomicAdd(p.counts + ci, dpass);
-              }
-            }
-            dpass = 0;
-          }
-        }
-      };
-      auto run_deferred = [&](int cur_qi, int cur_s, uint32_t& c_cur) {
-        while (dmask) run_one(cur_qi, cur_s, c_cur);
-      };
-      // kOne: wait for an accumulator, settling deferred rows while it is not ready (their recompute
-      // fills the time the warp would spend waiting, off the group's buffer round trip)
-      auto wait_or_work = [&](uint32_t bar, uint32_t par) {
-        if constexpr (kOne) {
-          while (dmask) {
-            uint32_t ready;
-            asm volatile("{\n\t.reg .pred P1;\n\tmbarrier.test_wait.parity.shared::cta.b64 P1, [%1], %2;\n\t"
-                         "selp.u32 %0, 1, 0, P1;\n\t}" : "=r"(ready) : "r"(bar), "r"(par) : "memory");
-            if (__all_sync(0xffffffffu, ready)) return;
-            run_one(qi, s, cnt);
-          }
-        }
-        mbar_wait(bar, par);
-      };
       while (u < U) {
         const int row = tq * kBM + row_in_tile;
         const bool valid = row < nvalid;
@@ -1057,7 +881,6 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         bool pass = false;
         if constexpr (kFold) {
           int G1 = INT_MIN, G2 = INT_MIN;  // two largest folded values X over the reference
-          int WL = INT_MIN, wp = 0;        // kOne: the winner piece's other-half maximum, the winning half
           for (int c = 0; c < cpr; ++c) {
             const uint32_t ck = sbase + SmemPlan::kCol + (b0 + s * cpr + c) * kColBytes;
             int kpc;  // real columns of this chunk: the last column term is -1 - kpc when padded
@@ -1075,10 +898,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
               if (kSkip && pp >= np) break;  // all-padding pieces (m not a multiple of 64 x 4) are not computed
               const uint32_t buf = g * kNB + (pp & 1);
-              PROF_B();
-              if constexpr (kOne) wait_or_work(tfull(buf), ((pp >> 1) ^ (ph_t >> (pp & 1))) & 1);
-              else WAITD(tfull(buf), ((pp >> 1) ^ (ph_t >> (pp & 1))) & 1, 8, u, pp);
-              PROF_E(0);
+              PROF_B(); mbar_wait(tfull(buf), ((pp >> 1) ^ (ph_t >> (pp & 1))) & 1); PROF_E(0);
               PROF_B();
               tc_fence_after();
 #ifndef TID_NOLOAD  // timing experiment only: scan stale registers (wrong results)
@@ -1091,10 +911,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               if (lane == 0) mbar_arrive(tempty(buf));
               PROF_E(3);
               PROF_B();
-              if constexpr (kOne) {  // piece maxima only, tracked over the whole reference
-                if (kpc >= (pp + 1) * kPiece) scan64_one<false>(v, kPiece, c * kPiecesPerChunk + pp, G1, G2, WL, wp);
-                else scan64_one<true>(v, kpc - pp * kPiece, c * kPiecesPerChunk + pp, G1, G2, WL, wp);
-              } else if (kpc >= (pp + 1) * kPiece) {  // every column of the piece is real (the common case)
+              if (kpc >= (pp + 1) * kPiece) {  // every column of the piece is real (the common case)
 #ifndef TID_NOSCAN
                 scan32_fold<false>(v, 32, R, T1, T2);
                 scan32_fold<false>(v + 32, 32, R, T1, T2);
@@ -1106,32 +923,18 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               PROF_E(1);
             }
             if (kSkip) ph_t ^= use_parity(np);
-            if constexpr (!kOne) {
-              PROF_B();
-              int x1, x2;
-              finish_fold(R, T1, T2, x1, x2);
-              G2 = max3i(min(G1, x1), G2, x2);
-              G1 = max(G1, x1);
-              PROF_E(2);
-            }
+            PROF_B();
+            int x1, x2;
+            finish_fold(R, T1, T2, x1, x2);
+            G2 = max3i(min(G1, x1), G2, x2);
+            G1 = max(G1, x1);
+            PROF_E(2);
           }
           PROF_B();
           // d = N_Q - 2X - p, p in {0, 1}: decide the ratio test from the bounds
+          const bool real2 = G2 > INT_MIN;
           bool undecided = false;
-          if constexpr (kOne) {
-            // the second largest X is >= L2 (a column other than G1's), so d2 <= N_Q - 2 L2 and
-            // d1 >= N_Q - 2 G1 - 1: proves the failures; every other row is settled exactly below
-            const int L2 = max(G2, WL);
-            if (valid && G1 > INT_MIN) {
-              bool fail_sure = false;
-              if (L2 > INT_MIN) {
-                const int lo1 = max(nqv - 2 * G1 - 1, 0), hi2 = nqv - 2 * L2;
-                fail_sure = ratio32 ? p.den2 * static_cast<uint32_t>(lo1) >= p.num2 * static_cast<uint32_t>(hi2)
-                                    : uint64_t(p.den2) * uint64_t(lo1) >= uint64_t(p.num2) * uint64_t(hi2);
-              }
-              undecided = !fail_sure;
-            }
-          } else if (valid && G2 > INT_MIN) {
+          if (valid && real2) {
             const int hi1 = nqv - 2 * G1, hi2 = nqv - 2 * G2;
             const int lo1 = max(hi1 - 1, 0), lo2 = max(hi2 - 1, 0);
             bool pass_sure, fail_sure;
@@ -1152,59 +955,16 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             if (und) atomicAdd(&g_prof[148 * 32 * 8 - 1], 1ull);
           }
 #endif
-#ifdef TID_NOFB  // timing experiment only: no exact recompute (wrong results)
-          und = 0;
-#endif
-          if constexpr (kOne) {
-            run_deferred(qi, s, cnt);  // rows of the previous unit not settled while waiting
-            // defer up to kFbRows rows to this warp's next unit of the job: their exact recompute then
-            // overlaps that unit's MMAs.  The query row goes to the warp's scratch by cp.async now.
-            if (has_next && und) {
-              const int rank = __popc(und & ((1u << lane) - 1));
-              const bool dfr = undecided && rank < kFbRows;
-              if (dfr) {
-                const uint32_t slot = fbuf + rank * kFbBytes;
-                const uint8_t* src = p.qs + (static_cast<int64_t>(qi) * p.n_rows + row) * kDim;
-#pragma unroll
-                for (int w = 0; w < 8; ++w)
-                  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(slot + 16 * w), "l"(src + 16 * w) : "memory");
-                asm volatile("st.shared.v4.s32 [%0], {%1, %2, %3, %4};" ::"r"(slot + kDim), "r"(G1), "r"(max(G2, WL)),
-                             "r"(wp), "r"(row) : "memory");
-                asm volatile("st.shared.s32 [%0], %1;" ::"r"(slot + kDim + 16), "r"(nqv) : "memory");
-              }
-              asm volatile("cp.async.commit_group;" ::: "memory");
-              dmask = dall = __ballot_sync(0xffffffffu, dfr);
-              d_qi = qi;
-              d_s = s;
-              und &= ~dmask;
-            }
-          }
-          while (und) {  // recompute the row exactly now (kOne: from its winning half first)
+          while (und) {  // rare: recompute the row exactly
             const int l = __ffs(und) - 1;
             und &= und - 1;
             const int rl = __shfl_sync(0xffffffffu, row, l);
             const int nl = __shfl_sync(0xffffffffu, nqv, l);
-            int r = 2;
-            if constexpr (kOne) {
-              const int t1 = __shfl_sync(0xffffffffu, G1, l), o = __shfl_sync(0xffffffffu, max(G2, WL), l);
-              const int wpl = __shfl_sync(0xffffffffu, wp, l);
-              const uint4* qg = reinterpret_cast<const uint4*>(p.qs + (static_cast<int64_t>(qi) * p.n_rows + rl) * kDim);
-              uint4 q[8];
-#pragma unroll
-              for (int w = 0; w < 8; ++w) q[w] = qg[w];
-              r = settle_half(p, q, sbase, b0 + s * cpr + wpl / (2 * kPiecesPerChunk), wpl % (2 * kPiecesPerChunk), nl, t1,
-                              o, lane);
-            }
-            if (r == 2) {  // the whole reference from global memory
-#ifdef TID_PROF
-              if (kOne && lane == 0) atomicAdd(&g_prof[148 * 32 * 8 - 3], 1ull);
-#endif
-              int d1, d2;
-              exact_row_global(p, qi, rl, J.ref_first + s, nl, lane, cpr,
-                               sbase + SmemPlan::kCol + (b0 + s * cpr) * kColBytes, d1, d2);
-              r = d2 != INT_MAX && uint64_t(p.den2) * uint64_t(d1) < uint64_t(p.num2) * uint64_t(d2);
-            }
-            if (lane == l) pass = r == 1;
+            int d1, d2;
+            exact_row_global(p, qi, rl, J.ref_first + s, nl, lane, cpr,
+                             sbase + SmemPlan::kCol + (b0 + s * cpr) * kColBytes, d1, d2);
+            if (lane == l)
+              pass = d2 != INT_MAX && uint64_t(p.den2) * uint64_t(d1) < uint64_t(p.num2) * uint64_t(d2);
           }
         } else {
         int g1d = INT_MAX, g1i = -1, g2d = INT_MAX, g2i = -1;  // running exact 2-NN over chunks
@@ -1326,8 +1086,8 @@ cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CU
   int dev = 0;
   cudaGetDevice(&dev);
   if (dev >= 64 || !(attr_set >> dev & 1)) {
-    for (auto k : {match_kernel<true, false, false>, match_kernel<true, true, false>, match_kernel<true, false, true>,
-                   match_kernel<true, true, true>, match_kernel<false, false, false>, match_kernel<false, true, false>}) {
+    for (auto k : {match_kernel<true, false>, match_kernel<true, true>, match_kernel<false, false>,
+                   match_kernel<false, true>}) {
       cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                            static_cast<int>(SmemPlan::kAlloc));
       if (e != cudaSuccess) return e;
@@ -1335,10 +1095,8 @@ cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CU
     if (dev < 64) attr_set |= uint64_t(1) << dev;
   }
   const bool skip = piece_count_last(p.m, p.cpr) < kPiecesPerChunk;
-  const bool one = fold && p.scan_one;
-  auto kern = one ? (skip ? match_kernel<true, true, true> : match_kernel<true, false, true>)
-            : fold ? (skip ? match_kernel<true, true, false> : match_kernel<true, false, false>)
-                   : (skip ? match_kernel<false, true, false> : match_kernel<false, false, false>);
+  auto kern = fold ? (skip ? match_kernel<true, true> : match_kernel<true, false>)
+                   : (skip ? match_kernel<false, true> : match_kernel<false, false>);
   kern<<<grid, kNumThreads, SmemPlan::kAlloc, s>>>(qmap, rmap, p);
   return cudaGetLastError();
 }

@@ -90,8 +90,6 @@ struct MatchParams {
   const uint8_t* qs;         // [num_q][n_rows][128] shifted queries q' = q ^ 0x80
   const uint8_t* rdesc;      // reference descriptors of the tensor map, [*][m][128] raw u8
   int32_t m;                 // stored rows per reference
-  int32_t scan_one;          // search epilogue: 1 = piece maxima only + exact recompute of the rows that
-                             //    the bound cannot decide; 0 = exact two-partition top-2 (folded verify)
   int32_t slot_banks;        // 2: jobs alternate between slots {0, 1} and {2, 3} (small batches: the next
                              //    job's references load while this one runs); else 1
 };

@@ -21,8 +21,6 @@ else:
     refs, _ = tidgen.refs(0, R, m)
     qs, _ = tidgen.queries(0, B, n, R_total=R, m=m)
     idx = tid.Index(ref_kp=m)
-    if os.environ.get("TID_SCAN"):
-        idx.set_tuning(scan=int(os.environ["TID_SCAN"]))
     idx.add_references(refs)
     idx.search(qs, 5)
     idx.profile(True)

@@ -20,8 +20,6 @@ qs, tg = tidgen.queries(0, B, n, R_total=R, m=m)
 import torch  # noqa: E402
 dq = torch.from_numpy(qs).cuda()
 with tid.Index(ref_kp=m) as idx:
-    if os.environ.get("TID_SCAN"):  # epilogue scan mode (tid_tuning.scan) for A/B runs
-        idx.set_tuning(scan=int(os.environ["TID_SCAN"]))
     idx.add_references(refs)
     ids, cnt = idx.search(dq, k)
     torch.cuda.synchronize()

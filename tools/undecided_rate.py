@@ -1,7 +1,5 @@
-"""Rate of rows the folded search leaves undecided, from a -DTID_PROF build:
-python tools/undecided_rate.py [R] [scan]; scan 1 = two-partition (undecided = ratio within the +-1
-bound -> exact recompute from global memory), 2 = piece maxima (undecided = not provably failing ->
-winner piece recomputed from shared memory; "full" = rows that still needed the global recompute)."""
+"""Rate of rows the folded search leaves undecided (ratio within the +-1 bound -> exact global
+recompute), from a -DTID_PROF build: python tools/undecided_rate.py [R]"""
 import ctypes
 import os
 import sys
@@ -15,9 +13,7 @@ import paper_conf_icpp_wangzll21_b200 as tid  # noqa: E402
 R, B, n, m = int(sys.argv[1]) if len(sys.argv) > 1 else 20000, 256, 1000, 256
 refs, _ = tidgen.refs(0, R, m)
 qs, _ = tidgen.queries(0, B, n, R_total=R, m=m)
-scan = int(sys.argv[2]) if len(sys.argv) > 2 else 0
 with tid.Index(ref_kp=m) as idx:
-    idx.set_tuning(scan=scan)
     idx.add_references(refs)
     idx.search(qs, 5)
 lib = tid.load_library()
@@ -26,4 +22,4 @@ lib.tid_debug_read_prof(buf.ctypes.data, ctypes.c_size_t(buf.nbytes))
 rows = B * 1024 * R  # padded rows x references, one search
 units = B * 8 * R * 4  # warp-units (4 lane-quarter warps per 128-row unit)
 print(f"undecided rows {int(buf[-2])} of {rows} ({buf[-2] / rows:.2e}); warp-units with any: {int(buf[-1])} "
-      f"of {units} ({buf[-1] / units:.2e}); full recomputes {int(buf[-3])} ({buf[-3] / rows:.2e}); scan={scan}")
+      f"of {units} ({buf[-1] / units:.2e})")
