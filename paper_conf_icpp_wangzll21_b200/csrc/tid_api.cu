@@ -1626,7 +1626,14 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
     p.rdesc = dr;
     p.slot_banks = 1;
   }
-  cudaError_t e = launch_match(p, qmap, rmap, fold, grid, s);
+  // pairs streamed through per-chunk reference slots (TID_VERIFY_STREAM=0: the job kernel, for A/B).
+  // The stream kernel's parity waits assume every group runs a tile of every pair (T >= 3 = kNG); with
+  // fewer tiles per query a group skips pairs, so n <= 256 takes the job kernel.
+  static const bool stream_ok = [] {
+    const char* e = getenv("TID_VERIFY_STREAM");
+    return !(e && e[0] == '0');
+  }();
+  cudaError_t e = (stream_ok && T >= kNG) ? launch_verify_stream(p, qmap, rmap, fold, grid, s) : launch_match(p, qmap, rmap, fold, grid, s);
   if (e != cudaSuccess) return fail(TID_ECUDA, "match kernel launch: %s", cudaGetErrorString(e));
   if (idx->prof) {
     CU(cudaEventRecord(e1, s));

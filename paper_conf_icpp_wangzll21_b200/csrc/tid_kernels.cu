@@ -1101,6 +1101,442 @@ cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CU
   return cudaGetLastError();
 }
 
+// ------------------------------------------------------------------ one-to-one verification, streamed
+// Pair-streaming verification (one query image against one reference image; counts, and for
+// the packed-key variant (d1, i1, d2, i2), exactly as the job kernel above).  The job kernel loads a
+// pair's whole reference (up to 4 chunks = all 4 slots), runs its T query tiles on the 3 groups
+// (T = 8: 3 / 3 / 2) and only then releases the slots, so every pair boundary drains the pipeline on
+// every group.  Here a CTA's pairs form one sequence of query tiles gt = lp * T + t (lp = the CTA's
+// pair count), tile gt runs on group gt % 3 (its TMEM query slot and its SMEM stage are gt % 3 too),
+// and reference slot c is released as soon as all T tiles of pair lp have finished chunk c (one MMA
+// commit per tile): the next pair's chunk c loads while the last tiles of this pair still run on
+// chunks > c, and no group idles at a pair boundary unless the next pair's chunk is still in flight.
+// The column terms (folded: W and the norm digits; packed-key: N_R * 256 + i and the zeroing of rows
+// >= m_r) are computed on chip by the 4 warps of the group that runs the pair's first tile, chunk by
+// chunk ahead of its MMAs, into a per-pair column buffer double-buffered by pair parity (released by
+// the 4 * T epilogue warp-tiles that read it).
+// Every wait below is a parity wait on a barrier whose phase advances once per pair (slots) or once per
+// two pairs (column buffers); it is unambiguous because each group runs at least one tile of every pair,
+// so no waiter can be two phases behind: the kernel requires T >= 3 (tid_verify routes n <= 256 to the
+// job kernel).
+struct VSmem {
+  static constexpr uint32_t kR = 0;                                        // 4 x 32 KiB reference chunks
+  static constexpr uint32_t kQ = kR + kMaxSlots * kRTileBytes;             // 3 x 16 KiB query stages
+  static constexpr uint32_t kX = kQ + kQStages * kQTileBytes;              // 4 x 8 KiB norm digits (folded)
+  static constexpr uint32_t kAx = kX + kMaxSlots * kXTileBytes;            // constant norm-term operand
+  static constexpr uint32_t kCol = kAx + kBM * kXDim;                      // 2 pair buffers x 4 x 1 KiB
+  static constexpr uint32_t kColPair = kMaxSlots * kColBytes;
+  static constexpr uint32_t kBar = kCol + 2 * kColPair;
+  static constexpr uint32_t kQFull = kBar;
+  static constexpr uint32_t kQEmpty = kQFull + 8 * kQStages;
+  static constexpr uint32_t kRFull = kQEmpty + 8 * kQStages;
+  static constexpr uint32_t kREmpty = kRFull + 8 * kMaxSlots;
+  static constexpr uint32_t kXReady = kREmpty + 8 * kMaxSlots;
+  static constexpr uint32_t kTFull = kXReady + 8 * kMaxSlots;
+  static constexpr uint32_t kTEmpty = kTFull + 8 * kTmemBufs;
+  static constexpr uint32_t kTQFull = kTEmpty + 8 * kTmemBufs;
+  static constexpr uint32_t kTQEmpty = kTQFull + 8 * kTQ;
+  static constexpr uint32_t kColEmpty = kTQEmpty + 8 * kTQ;                // per pair buffer: all readers done
+  static constexpr uint32_t kColReady = kColEmpty + 8 * 2;               // per (pair buffer, chunk): terms written
+  static constexpr uint32_t kAxFull = kColReady + 8 * 2 * kMaxSlots;
+  static constexpr uint32_t kTmemPtr = kAxFull + 8;
+  static constexpr uint32_t kEnd = kTmemPtr + 16;
+  static constexpr uint32_t kAlloc = kEnd + 1024;
+};
+static_assert(VSmem::kAlloc <= 232448, "227 KiB of shared memory per CTA");
+static_assert(kNG == 3 && kQStages == 3 && kTQ == 3, "tile gt -> group, stage and TMEM slot gt % 3");
+
+// Column terms of chunk c of the current pair, columns col = tig, tig + 128 (the group's 128 threads):
+// folded: W = 256 sum r - N_R (-1 - kpc for padding) into the pair's column buffer and the norm digits
+// into X slot c; packed-key: N_R * 256 + i (sentinel for padding) and rows in [mcap, m) zeroed.
+template <bool kFold>
+__device__ __forceinline__ void vstream_terms(uint32_t sbase, uint32_t colbuf, int c, int mcap, int m, int tig) {
+#pragma unroll 1
+  for (int col = tig; col < kBN; col += 128) {
+    const int gcol = c * kBN + col;
+    const uint32_t row = sbase + VSmem::kR + c * kRTileBytes + col * kDim;
+    uint32_t nr = 0, sr = 0;
+    if (gcol < mcap) {
+#pragma unroll
+      for (int w = 0; w < kDim / 16; ++w) {
+        const int4 x4 = lds128(row + 16 * w);
+        nr = __dp4a(static_cast<uint32_t>(x4.x), static_cast<uint32_t>(x4.x), nr);
+        nr = __dp4a(static_cast<uint32_t>(x4.y), static_cast<uint32_t>(x4.y), nr);
+        nr = __dp4a(static_cast<uint32_t>(x4.z), static_cast<uint32_t>(x4.z), nr);
+        nr = __dp4a(static_cast<uint32_t>(x4.w), static_cast<uint32_t>(x4.w), nr);
+        if (kFold) {
+          sr = __dp4a(static_cast<uint32_t>(x4.x), 0x01010101u, sr);
+          sr = __dp4a(static_cast<uint32_t>(x4.y), 0x01010101u, sr);
+          sr = __dp4a(static_cast<uint32_t>(x4.z), 0x01010101u, sr);
+          sr = __dp4a(static_cast<uint32_t>(x4.w), 0x01010101u, sr);
+        }
+      }
+    } else if (!kFold && gcol < m) {
+      // a row beyond this pair's m_r holds the caller's bytes: zeroed, so its product is 0 and the
+      // sentinel key never wins (rows >= m are zero-filled by TMA).  The folded path masks by W < 0.
+#pragma unroll
+      for (int w = 0; w < kDim / 16; ++w)
+        asm volatile("st.shared.v4.b32 [%0], {%1, %1, %1, %1};" ::"r"(row + 16 * w), "r"(0) : "memory");
+    }
+    int32_t term;
+    if (kFold) {
+      term = gcol < mcap ? 256 * static_cast<int>(sr) - static_cast<int>(nr) : -1 - max(0, min(mcap - c * kBN, kBN));
+      uint32_t w8[8];
+      norm_digits(term, w8);
+      const uint32_t dst = sbase + VSmem::kX + c * kXTileBytes + col * kXDim;
+      asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst), "r"(w8[0]), "r"(w8[1]), "r"(w8[2]),
+                   "r"(w8[3]) : "memory");
+      asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst + 16), "r"(w8[4]), "r"(w8[5]), "r"(w8[6]),
+                   "r"(w8[7]) : "memory");
+    } else {
+      term = (gcol < mcap ? static_cast<int32_t>(nr) : kSentinelNorm) * 256 + col;
+    }
+    asm volatile("st.shared.s32 [%0], %1;" ::"r"(colbuf + c * kColBytes + col * 4), "r"(term) : "memory");
+  }
+}
+
+template <bool kFold, bool kSkip>
+__global__ void __launch_bounds__(kNumThreads, 1)
+    verify_stream_kernel(const __grid_constant__ CUtensorMap qmap, const __grid_constant__ CUtensorMap rmap,
+                         const MatchParams p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const uint32_t sbase = smem_u32(smem);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int T = p.tiles_per_q, cpr = p.cpr;
+  const int npairs = static_cast<int>(blockIdx.x) < p.num_q
+                         ? (p.num_q - static_cast<int>(blockIdx.x) + static_cast<int>(gridDim.x) - 1) /
+                               static_cast<int>(gridDim.x)
+                         : 0;
+  const int ntiles = npairs * T;  // this CTA's tile sequence gt = lp * T + t, pair = blockIdx.x + lp * gridDim.x
+
+  auto bar = [&](uint32_t base, int i) { return sbase + base + 8 * i; };
+  uint32_t* tmem_ptr_smem = reinterpret_cast<uint32_t*>(smem + VSmem::kTmemPtr);
+  const uint32_t axfull = sbase + VSmem::kAxFull;
+
+  if (kFold) {  // constant norm-term operand (see the job kernel)
+    uint32_t* ax = reinterpret_cast<uint32_t*>(smem + VSmem::kAx);
+    for (int i = threadIdx.x; i < kBM * kXDim / 4; i += blockDim.x) ax[i] = (i & 3) == 3 ? 0x01FFFFFFu : 0xFFFFFFFFu;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
+  if (threadIdx.x == 0) {
+    prefetch_tmap(&qmap);
+    prefetch_tmap(&rmap);
+    for (int i = 0; i < kQStages; ++i) { mbar_init(bar(VSmem::kQFull, i), 1); mbar_init(bar(VSmem::kQEmpty, i), 1); }
+    for (int i = 0; i < kTQ; ++i) { mbar_init(bar(VSmem::kTQFull, i), 1); mbar_init(bar(VSmem::kTQEmpty, i), 1); }
+    for (int c = 0; c < kMaxSlots; ++c) {
+      mbar_init(bar(VSmem::kRFull, c), 1);
+      mbar_init(bar(VSmem::kREmpty, c), T);   // one MMA commit per tile of the pair
+      mbar_init(bar(VSmem::kXReady, c), 4);   // the 4 warps of the first tile's group
+    }
+    for (int i = 0; i < kTmemBufs; ++i) { mbar_init(bar(VSmem::kTFull, i), 1); mbar_init(bar(VSmem::kTEmpty, i), 4); }
+    for (int b = 0; b < 2; ++b) mbar_init(bar(VSmem::kColEmpty, b), 4 * T);  // every warp-tile of the pair
+    for (int i = 0; i < 2 * kMaxSlots; ++i) mbar_init(bar(VSmem::kColReady, i), 4);
+    mbar_init(axfull, 1);
+    fence_barrier_init();
+  }
+  if (warp == kFirstMmaWarp) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(tmem_ptr_smem))
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_ptr_smem;
+
+  if (warp == kProducerWarp) {
+    if (lane == 0) {
+      // ---- query tiles: TMA into stage gt % 3, then SMEM -> TMEM slot gt % 3 (the group's)
+      if (kFold) {
+        tc_fence_after();
+        tmem_cp_128x256b(tmem_base + kAxCol, smem_desc_sw32(sbase + VSmem::kAx));
+        commit_one(axfull);
+      }
+      auto issue = [&](int gt) {
+        const int st = gt % kQStages, k = gt / kQStages;
+        mbar_wait_sleep(bar(VSmem::kQEmpty, st), (k & 1) ^ 1);
+        mbar_expect_tx(bar(VSmem::kQFull, st), kQTileBytes);
+        const int lp = gt / T, t = gt - lp * T;
+        tma_load_3d(sbase + VSmem::kQ + st * kQTileBytes, &qmap, bar(VSmem::kQFull, st), 0, t * kBM,
+                    static_cast<int>(blockIdx.x) + lp * static_cast<int>(gridDim.x));
+      };
+      if (ntiles > 0) issue(0);
+      for (int gt = 0; gt < ntiles; ++gt) {
+        if (gt + 1 < ntiles) issue(gt + 1);
+        const int sl = gt % kTQ, k = gt / kTQ;
+        mbar_wait(bar(VSmem::kQFull, sl), k & 1);
+        mbar_wait_sleep(bar(VSmem::kTQEmpty, sl), (k & 1) ^ 1);
+        tc_fence_after();
+        const uint64_t sd = smem_desc_sw128(sbase + VSmem::kQ + sl * kQTileBytes);
+#pragma unroll
+        for (int kk = 0; kk < kDim / kXDim; ++kk)
+          tmem_cp_128x256b(tmem_base + kTQBase + sl * kQCols + 8 * kk, sd + 2 * kk);
+        commit_one(bar(VSmem::kTQFull, sl));
+        commit_one(bar(VSmem::kQEmpty, sl));
+      }
+    } else if (lane == 1) {
+      // ---- reference chunks: chunk c of pair lp as soon as pair lp - 1 has finished with slot c
+      for (int lp = 0; lp < npairs; ++lp) {
+        const int pair = static_cast<int>(blockIdx.x) + lp * static_cast<int>(gridDim.x);
+        for (int c = 0; c < cpr; ++c) {
+          mbar_wait_sleep(bar(VSmem::kREmpty, c), (lp & 1) ^ 1);
+          mbar_expect_tx(bar(VSmem::kRFull, c), kRTileBytes);
+          tma_load_3d(sbase + VSmem::kR + c * kRTileBytes, &rmap, bar(VSmem::kRFull, c), 0, c * kBN, pair);
+        }
+      }
+    }
+  } else if (warp < kFirstEpiWarp) {
+    // ---- MMA issuer of group g: tiles gt = g, g + 3, ...
+    const int g = warp - kFirstMmaWarp;
+    const int np_last = kSkip ? piece_count_last(p.m, cpr) : kPiecesPerChunk;
+    uint32_t ph_t = 0;
+    if (kFold) mbar_wait(axfull, 0);
+    const uint32_t at = tmem_base + kTQBase + g * kQCols;
+    for (int gt = g, k = 0; gt < ntiles; gt += kNG, ++k) {
+      const int lp = gt / T;
+      mbar_wait(bar(VSmem::kTQFull, g), k & 1);
+      for (int c = 0; c < cpr; ++c) {
+        mbar_wait(bar(VSmem::kRFull, c), lp & 1);
+        mbar_wait(bar(VSmem::kXReady, c), lp & 1);
+        const uint64_t bd0 = smem_desc_sw128(sbase + VSmem::kR + c * kRTileBytes);
+        const int np = c == cpr - 1 ? np_last : kPiecesPerChunk;
+#pragma unroll
+        for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
+          if (kSkip && pp >= np) break;
+          const uint32_t buf = g * kNB + (pp & 1);
+          mbar_wait(bar(VSmem::kTEmpty, buf), (((pp >> 1) ^ (ph_t >> (pp & 1))) & 1) ^ 1);
+          tc_fence_after();
+          const uint64_t bd = bd0 + pp * (kPiece * kDim >> 4);
+          if (kFold)
+            mma_piece_fold_ts(tmem_base + buf * kPiece, at, bd, tmem_base + kAxCol,
+                              smem_desc_sw32(sbase + VSmem::kX + c * kXTileBytes) + pp * (kPiece * kXDim >> 4),
+                              bar(VSmem::kTFull, buf));
+          else
+            mma_piece_ts(tmem_base + buf * kPiece, at, bd, bar(VSmem::kTFull, buf));
+        }
+        if (kSkip) ph_t ^= use_parity(np);
+        mma_commit(bar(VSmem::kREmpty, c));  // this tile's MMAs on chunk c done: slot c may be refilled
+      }
+      mma_commit(bar(VSmem::kTQEmpty, g));
+    }
+  } else {
+    // ---- epilogue group g: TMEM -> registers -> top-2 -> ratio -> count (and (d1, i1, d2, i2))
+    const int ew = warp - kFirstEpiWarp;
+    const int g = ew >> 2;
+    const int quarter = warp & 3;
+    const int tig = (ew & 3) * 32 + lane;  // thread in group (column-term work)
+    const uint32_t taddr_q = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16);
+    const int row_in_tile = quarter * 32 + lane;
+    const int nq_ld = T * kBM;
+    const bool ratio32 = p.num2 <= 511u && p.den2 <= 511u;
+    const int np_last = kSkip ? piece_count_last(p.m, cpr) : kPiecesPerChunk;
+    uint32_t ph_t = 0;
+    uint32_t v[64];
+    for (int gt = g; gt < ntiles; gt += kNG) {
+      const int lp = gt / T, t = gt - lp * T;
+      const int pair = static_cast<int>(blockIdx.x) + lp * static_cast<int>(gridDim.x);
+      const uint32_t colbuf = sbase + VSmem::kCol + (lp & 1) * VSmem::kColPair;
+      const int mcap = p.m_valid ? min(p.m_valid[pair], p.m) : p.m;
+      const int nvalid = min(p.n_valid ? p.n_valid[pair] : p.n_rows, p.n_rows);
+      const int row = t * kBM + row_in_tile;
+      const bool valid = row < nvalid;
+      const int32_t nqv = valid ? p.nq[static_cast<int64_t>(pair) * nq_ld + row] : 0;
+      int done_terms = cpr;  // chunks whose column terms this warp has written (first tile of a pair only)
+      auto terms = [&](int c) {
+        mbar_wait(bar(VSmem::kRFull, c), lp & 1);
+        vstream_terms<kFold>(sbase, colbuf, c, mcap, p.m, tig);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // digits / zeroed rows -> tensor core
+        __syncwarp();
+        if (lane == 0) {
+          mbar_arrive(bar(VSmem::kXReady, c));                    // for the MMA warps (slot phase = pair)
+          mbar_arrive(bar(VSmem::kColReady, (lp & 1) * kMaxSlots + c));  // for the epilogue (buffer phase)
+        }
+      };
+      if (t == 0) {  // this group computes the pair's column terms, one chunk ahead of its MMAs
+        mbar_wait(bar(VSmem::kColEmpty, lp & 1), ((lp >> 1) & 1) ^ 1);
+        terms(0);
+        done_terms = 1;
+      }
+      bool pass = false;
+      int G1 = INT_MIN, G2 = INT_MIN;                                      // folded: two largest X
+      int g1d = INT_MAX, g1i = -1, g2d = INT_MAX, g2i = -1;                // packed keys: running 2-NN
+      for (int c = 0; c < cpr; ++c) {
+        if (done_terms < cpr) {
+          while (done_terms <= c) { terms(done_terms); ++done_terms; }
+          // the next chunk's terms now if its tile has landed (the MMAs of chunk c run meanwhile)
+          if (done_terms == c + 1 && done_terms < cpr) {
+            uint32_t ready;
+            asm volatile(
+                "{\n\t.reg .pred P1;\n\tmbarrier.test_wait.parity.shared::cta.b64 P1, [%1], %2;\n\t"
+                "selp.u32 %0, 1, 0, P1;\n\t}"
+                : "=r"(ready)
+                : "r"(bar(VSmem::kRFull, c + 1)), "r"(static_cast<uint32_t>(lp & 1))
+                : "memory");
+            if (__shfl_sync(0xffffffffu, ready, 0)) { terms(done_terms); ++done_terms; }
+          }
+        }
+        // this chunk's column buffer is written (a per-pair-buffer barrier: the slot's xready may already
+        // be in the next pair's phase once every tile's MMAs have left chunk c)
+        mbar_wait(bar(VSmem::kColReady, (lp & 1) * kMaxSlots + c), (lp >> 1) & 1);
+        const uint32_t ck = colbuf + c * kColBytes;
+        const int np = c == cpr - 1 ? np_last : kPiecesPerChunk;
+        if constexpr (kFold) {
+          int kpc;
+          asm volatile("ld.shared.s32 %0, [%1];" : "=r"(kpc) : "r"(ck + (kBN - 1) * 4));
+          kpc = kpc < 0 ? -1 - kpc : kBN;
+          int R[16];
+#pragma unroll
+          for (int b = 0; b < 16; ++b) R[b] = INT_MIN;
+          int T1 = INT_MIN, T2 = INT_MIN;
+#pragma unroll
+          for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
+            if (kSkip && pp >= np) break;
+            const uint32_t buf = g * kNB + (pp & 1);
+            mbar_wait(bar(VSmem::kTFull, buf), ((pp >> 1) ^ (ph_t >> (pp & 1))) & 1);
+            tc_fence_after();
+            tmem_ld64(taddr_q + buf * kPiece, v);
+            tmem_wait_ld();
+            reg_fence64(v);
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(bar(VSmem::kTEmpty, buf));
+            if (kpc >= (pp + 1) * kPiece) {
+              scan32_fold<false>(v, 32, R, T1, T2);
+              scan32_fold<false>(v + 32, 32, R, T1, T2);
+            } else {
+              scan32_fold<true>(v, kpc - pp * kPiece, R, T1, T2);
+              scan32_fold<true>(v + 32, kpc - pp * kPiece - 32, R, T1, T2);
+            }
+          }
+          int x1, x2;
+          finish_fold(R, T1, T2, x1, x2);
+          G2 = max3i(min(G1, x1), G2, x2);
+          G1 = max(G1, x1);
+        } else {
+          int R[16];
+#pragma unroll
+          for (int b = 0; b < 16; ++b) R[b] = INT_MAX;
+          int T1 = INT_MAX, T2 = INT_MAX;
+#pragma unroll
+          for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
+            if (kSkip && pp >= np) break;
+            const uint32_t buf = g * kNB + (pp & 1);
+            mbar_wait(bar(VSmem::kTFull, buf), ((pp >> 1) ^ (ph_t >> (pp & 1))) & 1);
+            tc_fence_after();
+            uint32_t (&h32)[32] = *reinterpret_cast<uint32_t(*)[32]>(v);
+#pragma unroll
+            for (int h = 0; h < kPiece / 32; ++h) {
+              tmem_ld32(taddr_q + buf * kPiece + h * 32, h32);
+              tmem_wait_ld();
+              reg_fence(h32);
+              if (h == kPiece / 32 - 1) {
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(bar(VSmem::kTEmpty, buf));
+              }
+              scan32_regs(h32, ck + (pp * kPiece + h * 32) * 4, R, T1, T2);
+            }
+          }
+          int k1, k2;
+          finish_partition(R, T1, T2, k1, k2);
+          const int c1d = k1 >> 8, c1i = (k1 & 255) + c * kBN;
+          const int c2d = k2 >> 8, c2i = (k2 & 255) + c * kBN;
+          if (c == 0) {
+            g1d = c1d; g1i = c1i; g2d = c2d; g2i = c2i;
+          } else if (c1d < g1d) {  // earlier chunks win ties (lower index)
+            if (c2d < g1d) { g2d = c2d; g2i = c2i; } else { g2d = g1d; g2i = g1i; }
+            g1d = c1d; g1i = c1i;
+          } else if (c1d < g2d) {
+            g2d = c1d; g2i = c1i;
+          }
+        }
+        if (kSkip) ph_t ^= use_parity(np);
+      }
+      if constexpr (kFold) {
+        // d = N_Q - 2X - p, p in {0, 1}: the ratio test from the bounds, exact recompute if open
+        const bool real2 = G2 > INT_MIN;
+        bool undecided = false;
+        if (valid && real2) {
+          const int hi1 = nqv - 2 * G1, hi2 = nqv - 2 * G2;
+          const int lo1 = max(hi1 - 1, 0), lo2 = max(hi2 - 1, 0);
+          bool pass_sure, fail_sure;
+          if (ratio32) {
+            pass_sure = p.den2 * static_cast<uint32_t>(hi1) < p.num2 * static_cast<uint32_t>(lo2);
+            fail_sure = p.den2 * static_cast<uint32_t>(lo1) >= p.num2 * static_cast<uint32_t>(hi2);
+          } else {
+            pass_sure = uint64_t(p.den2) * uint64_t(hi1) < uint64_t(p.num2) * uint64_t(lo2);
+            fail_sure = uint64_t(p.den2) * uint64_t(lo1) >= uint64_t(p.num2) * uint64_t(hi2);
+          }
+          pass = pass_sure;
+          undecided = !pass_sure && !fail_sure;
+        }
+        uint32_t und = __ballot_sync(0xffffffffu, undecided);
+        while (und) {
+          const int l = __ffs(und) - 1;
+          und &= und - 1;
+          const int rl = __shfl_sync(0xffffffffu, row, l);
+          const int nl = __shfl_sync(0xffffffffu, nqv, l);
+          int d1, d2;
+          exact_row_global(p, pair, rl, pair, nl, lane, cpr, colbuf, d1, d2);
+          if (lane == l) pass = d2 != INT_MAX && uint64_t(p.den2) * uint64_t(d1) < uint64_t(p.num2) * uint64_t(d2);
+        }
+      } else {
+        const bool real1 = g1d < kSentinelNorm, real2 = g2d < kSentinelNorm;
+        if (ratio32) {
+          const uint32_t d1 = static_cast<uint32_t>(nqv + g1d), d2 = static_cast<uint32_t>(nqv + g2d);
+          pass = p.den2 * d1 < p.num2 * d2;
+        } else {
+          const uint64_t d1 = static_cast<uint64_t>(static_cast<int64_t>(nqv) + g1d);
+          const uint64_t d2 = static_cast<uint64_t>(static_cast<int64_t>(nqv) + g2d);
+          pass = static_cast<uint64_t>(p.den2) * d1 < static_cast<uint64_t>(p.num2) * d2;
+        }
+        pass = pass && valid && real2;
+        if (p.nn_out != nullptr && row < p.n_rows) {
+          int4 o;
+          o.x = (valid && real1) ? nqv + g1d : -1; o.y = (valid && real1) ? g1i : -1;
+          o.z = (valid && real2) ? nqv + g2d : -1; o.w = (valid && real2) ? g2i : -1;
+          reinterpret_cast<int4*>(p.nn_out)[static_cast<int64_t>(pair) * p.n_rows + row] = o;
+        }
+      }
+      const uint32_t cnt = __popc(__ballot_sync(0xffffffffu, pass));
+      if (lane == 0) {
+        if (cnt) atomicAdd(p.counts + pair, cnt);
+        mbar_arrive(bar(VSmem::kColEmpty, lp & 1));  // this warp-tile's last read of the pair's column buffer
+      }
+      __syncwarp();
+    }
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  if (warp == kFirstMmaWarp) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem_base) : "memory");
+  }
+}
+
+cudaError_t launch_verify_stream(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap, bool fold,
+                                 int grid, cudaStream_t s) {
+  static thread_local uint64_t attr_set = 0;  // bit d = device d configured (the opt-in is per device)
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev >= 64 || !(attr_set >> dev & 1)) {
+    for (auto k : {verify_stream_kernel<true, false>, verify_stream_kernel<true, true>,
+                   verify_stream_kernel<false, false>, verify_stream_kernel<false, true>}) {
+      cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                           static_cast<int>(VSmem::kAlloc));
+      if (e != cudaSuccess) return e;
+    }
+    if (dev < 64) attr_set |= uint64_t(1) << dev;
+  }
+  const bool skip = piece_count_last(p.m, p.cpr) < kPiecesPerChunk;
+  auto kern = fold ? (skip ? verify_stream_kernel<true, true> : verify_stream_kernel<true, false>)
+                   : (skip ? verify_stream_kernel<false, true> : verify_stream_kernel<false, false>);
+  kern<<<grid, kNumThreads, VSmem::kAlloc, s>>>(qmap, rmap, p);
+  return cudaGetLastError();
+}
+
 // ------------------------------------------------------------------ a1: reference prep
 // One thread per (reference, column) row: N_R = sum r^2 (dp4a) -> packed column key.
 // Modes: desc != null && src == null : in place (rows >= kp zeroed);

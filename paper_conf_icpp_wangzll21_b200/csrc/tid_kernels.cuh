@@ -112,6 +112,10 @@ void launch_query_prep(const uint8_t* q, int64_t B, int32_t n, int32_t tiles_per
 // fold = search path (s8 x u8 + on-chip norm-term K-step, counts); otherwise verify (exact 2-NN)
 cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap, bool fold, int grid,
                          cudaStream_t s);
+// one-to-one verification with pairs streamed through per-chunk reference slots (p.mode == kModeVerify,
+// p.colkey == nullptr; fold = counts only through the folded norms)
+cudaError_t launch_verify_stream(const MatchParams& p, const CUtensorMap& qmap, const CUtensorMap& rmap, bool fold,
+                                 int grid, cudaStream_t s);
 // ids_out / counts_out (optional): with segs == 1 the final ranking is written directly
 // Candidate lists: cand_out holds lists_per_b lists of k keys per query; the launch's segments
 // fill lists list0 .. list0 + segs - 1.

@@ -678,3 +678,32 @@ def test_verify_counts_only_folded(tid, rng, n, m, P):
         c_mask, _ = idx.verify(Q, Rr, n_q=n_q, m_r=m_r, want_nn=False)
     np.testing.assert_array_equal(c_full.astype(np.int64), oracle.verify(Q, Rr, want_nn=False)[0])
     np.testing.assert_array_equal(c_mask.astype(np.int64), oracle.verify(Q, Rr, n_q=n_q, m_r=m_r, want_nn=False)[0])
+
+
+@pytest.mark.parametrize("n,m,grid", [(1000, 1000, 3), (300, 600, 2), (129, 257, 5), (100, 2, 4), (250, 384, 1),
+                                      (700, 900, 7)])
+def test_verify_streamed_pairs(tid, rng, n, m, grid):
+    """Many pairs per CTA (a forced small grid): the pair-streaming verification kernel refills each
+    reference slot as soon as the previous pair's tiles have left it, runs tile gt of its pair sequence
+    on group gt % 3 and double-buffers the column terms by pair parity.  Every T (1 .. 8 query tiles),
+    chunk count (1 .. 4), last-chunk piece skip and ragged n_q / m_r, with (d1, i1, d2, i2) and with the
+    counts-only folded variant, equal the oracle."""
+    P = 3 * grid + 4  # several pairs per CTA, uneven
+    Q, Rr, _ = tidgen.pairs(P, n, m, n_planted=min(200, n, m))
+    Q[1, : n // 2] = rng.integers(0, 3, (n // 2, 128))
+    Rr[1] = rng.integers(0, 3, (m, 128))
+    n_q = rng.integers(1, n + 1, P).astype(np.int32)
+    m_r = rng.integers(1, m + 1, P).astype(np.int32)
+    n_q[0], m_r[0] = n, m
+    with tid.Index(ref_kp=256, query_kp_max=1024) as idx:
+        idx.set_tuning(grid=grid)
+        c, nn = idx.verify(Q, Rr, n_q=n_q, m_r=m_r)
+        c_fold, _ = idx.verify(Q, Rr, n_q=n_q, m_r=m_r, want_nn=False)
+        c_full, _ = idx.verify(Q, Rr, want_nn=False)
+    ec, enn = oracle.verify(Q, Rr, n_q=n_q, m_r=m_r)
+    np.testing.assert_array_equal(c.astype(np.int64), ec)
+    np.testing.assert_array_equal(c_fold.astype(np.int64), ec)
+    np.testing.assert_array_equal(c_full.astype(np.int64), oracle.verify(Q, Rr, want_nn=False)[0])
+    for p in range(P):
+        np.testing.assert_array_equal(nn[p, :n_q[p]].astype(np.int64), nn_from_oracle(enn[p, :n_q[p]]))
+        assert (nn[p, n_q[p]:] == -1).all()
