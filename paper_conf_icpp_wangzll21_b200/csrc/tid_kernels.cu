@@ -209,6 +209,27 @@ __device__ __forceinline__ void mma_piece_ts(uint32_t tmem_d, uint32_t a_tmem, u
       : "memory");
 }
 
+// Search piece variant for the streamed verification: the four q'.r K-steps read A from TMEM, the norm-term
+// K-step reads the constant operand from shared memory (its TMEM columns hold a fourth query-tile slot).
+__device__ __forceinline__ void mma_piece_fold_ts_sx(uint32_t tmem_d, uint32_t a_tmem, uint64_t bdesc, uint64_t axdesc,
+                                                     uint64_t bxdesc, uint32_t bar) {
+  asm volatile(
+      "{\n\t.reg .pred e, f, t;\n\t.reg .b32 a1, a2, a3;\n\t.reg .b64 b1, b2, b3;\n\t"
+      "setp.ne.b32 f, 0, 0;\n\t"
+      "setp.eq.b32 t, 0, 0;\n\t"
+      "add.u32 a1, %1, 8;\n\tadd.u32 a2, %1, 16;\n\tadd.u32 a3, %1, 24;\n\t"
+      "add.s64 b1, %2, 2;\n\tadd.s64 b2, %2, 4;\n\tadd.s64 b3, %2, 6;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %5, f;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [a1], b1, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [a2], b2, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], [a3], b3, %5, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::i8 [%0], %3, %4, %6, t;\n\t"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%7];\n\t}" ::"r"(tmem_d),
+      "r"(a_tmem), "l"(bdesc), "l"(axdesc), "l"(bxdesc), "r"(kIdescFold), "r"(kIdescI8), "r"(bar)
+      : "memory");
+}
+
 __device__ __forceinline__ void mma_commit(uint32_t bar) {
   asm volatile(
       "{\n\t.reg .pred e;\n\t"
@@ -1107,7 +1128,7 @@ cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CU
 // pair's whole reference (up to 4 chunks = all 4 slots), runs its T query tiles on the 3 groups
 // (T = 8: 3 / 3 / 2) and only then releases the slots, so every pair boundary drains the pipeline on
 // every group.  Here a CTA's pairs form one sequence of query tiles gt = lp * T + t (lp = the CTA's
-// pair count), tile gt runs on group gt % 3 (its TMEM query slot and its SMEM stage are gt % 3 too),
+// pair count), tile gt runs on group gt % 3 (SMEM stage gt % 3, TMEM query slot gt % 4: see kVTQ),
 // and reference slot c is released as soon as all T tiles of pair lp have finished chunk c (one MMA
 // commit per tile): the next pair's chunk c loads while the last tiles of this pair still run on
 // chunks > c, and no group idles at a pair boundary unless the next pair's chunk is still in flight.
@@ -1119,6 +1140,13 @@ cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CU
 // two pairs (column buffers); it is unambiguous because each group runs at least one tile of every pair,
 // so no waiter can be two phases behind: the kernel requires T >= 3 (tid_verify routes n <= 256 to the
 // job kernel).
+// TMEM: the 6 x 64 accumulator columns and FOUR 32-column query-tile slots (tile gt in slot gt % 4): the
+// producer fills a group's next tile into the spare slot while the group still runs its current one (the
+// norm-term K-step's constant operand is read from shared memory instead of TMEM to make room).  A slot's
+// parity wait cannot alias: group g reaches tile gt only after tile gt - 3, whose copy followed those of
+// tiles gt - 4 and earlier (one thread, in order).
+constexpr int kVTQ = 4;
+static_assert(kTQBase + kVTQ * kQCols <= 512, "TMEM budget of the streamed verification");
 struct VSmem {
   static constexpr uint32_t kR = 0;                                        // 4 x 32 KiB reference chunks
   static constexpr uint32_t kQ = kR + kMaxSlots * kRTileBytes;             // 3 x 16 KiB query stages
@@ -1135,8 +1163,8 @@ struct VSmem {
   static constexpr uint32_t kTFull = kXReady + 8 * kMaxSlots;
   static constexpr uint32_t kTEmpty = kTFull + 8 * kTmemBufs;
   static constexpr uint32_t kTQFull = kTEmpty + 8 * kTmemBufs;
-  static constexpr uint32_t kTQEmpty = kTQFull + 8 * kTQ;
-  static constexpr uint32_t kColEmpty = kTQEmpty + 8 * kTQ;                // per pair buffer: all readers done
+  static constexpr uint32_t kTQEmpty = kTQFull + 8 * kVTQ;
+  static constexpr uint32_t kColEmpty = kTQEmpty + 8 * kVTQ;                // per pair buffer: all readers done
   static constexpr uint32_t kColReady = kColEmpty + 8 * 2;               // per (pair buffer, chunk): terms written
   static constexpr uint32_t kAxFull = kColReady + 8 * 2 * kMaxSlots;
   static constexpr uint32_t kTmemPtr = kAxFull + 8;
@@ -1144,7 +1172,7 @@ struct VSmem {
   static constexpr uint32_t kAlloc = kEnd + 1024;
 };
 static_assert(VSmem::kAlloc <= 232448, "227 KiB of shared memory per CTA");
-static_assert(kNG == 3 && kQStages == 3 && kTQ == 3, "tile gt -> group, stage and TMEM slot gt % 3");
+static_assert(kNG == 3 && kQStages == 3, "tile gt -> group gt % 3 and SMEM stage gt % 3");
 
 // Column terms of chunk c of the current pair, columns col = tig, tig + 128 (the group's 128 threads):
 // folded: W = 256 sum r - N_R (-1 - kpc for padding) into the pair's column buffer and the norm digits
@@ -1212,7 +1240,6 @@ __global__ void __launch_bounds__(kNumThreads, 1)
 
   auto bar = [&](uint32_t base, int i) { return sbase + base + 8 * i; };
   uint32_t* tmem_ptr_smem = reinterpret_cast<uint32_t*>(smem + VSmem::kTmemPtr);
-  const uint32_t axfull = sbase + VSmem::kAxFull;
 
   if (kFold) {  // constant norm-term operand (see the job kernel)
     uint32_t* ax = reinterpret_cast<uint32_t*>(smem + VSmem::kAx);
@@ -1223,7 +1250,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     prefetch_tmap(&qmap);
     prefetch_tmap(&rmap);
     for (int i = 0; i < kQStages; ++i) { mbar_init(bar(VSmem::kQFull, i), 1); mbar_init(bar(VSmem::kQEmpty, i), 1); }
-    for (int i = 0; i < kTQ; ++i) { mbar_init(bar(VSmem::kTQFull, i), 1); mbar_init(bar(VSmem::kTQEmpty, i), 1); }
+    for (int i = 0; i < kVTQ; ++i) { mbar_init(bar(VSmem::kTQFull, i), 1); mbar_init(bar(VSmem::kTQEmpty, i), 1); }
     for (int c = 0; c < kMaxSlots; ++c) {
       mbar_init(bar(VSmem::kRFull, c), 1);
       mbar_init(bar(VSmem::kREmpty, c), T);   // one MMA commit per tile of the pair
@@ -1232,7 +1259,6 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     for (int i = 0; i < kTmemBufs; ++i) { mbar_init(bar(VSmem::kTFull, i), 1); mbar_init(bar(VSmem::kTEmpty, i), 4); }
     for (int b = 0; b < 2; ++b) mbar_init(bar(VSmem::kColEmpty, b), 4 * T);  // every warp-tile of the pair
     for (int i = 0; i < 2 * kMaxSlots; ++i) mbar_init(bar(VSmem::kColReady, i), 4);
-    mbar_init(axfull, 1);
     fence_barrier_init();
   }
   if (warp == kFirstMmaWarp) {
@@ -1245,17 +1271,16 @@ __global__ void __launch_bounds__(kNumThreads, 1)
   tc_fence_after();
   const uint32_t tmem_base = *tmem_ptr_smem;
 
+  // -DTID_PROF buckets: epilogue 0 wait-accumulator 1 scan + chunk finish 2 wait for a chunk (terms)
+  // 3 TMEM load + release 4 column terms 5 wait column buffer 6 tile tail; MMA 0 wait-free-accumulator
+  // 1 wait-query 2 wait-ref; producer (lane 0) 0 wait-stage 1 wait-TMA 2 wait-TMEM-slot
+  PROF_DECL
   if (warp == kProducerWarp) {
     if (lane == 0) {
       // ---- query tiles: TMA into stage gt % 3, then SMEM -> TMEM slot gt % 3 (the group's)
-      if (kFold) {
-        tc_fence_after();
-        tmem_cp_128x256b(tmem_base + kAxCol, smem_desc_sw32(sbase + VSmem::kAx));
-        commit_one(axfull);
-      }
       auto issue = [&](int gt) {
         const int st = gt % kQStages, k = gt / kQStages;
-        mbar_wait_sleep(bar(VSmem::kQEmpty, st), (k & 1) ^ 1);
+        PROF_B(); mbar_wait_sleep(bar(VSmem::kQEmpty, st), (k & 1) ^ 1); PROF_E(0);
         mbar_expect_tx(bar(VSmem::kQFull, st), kQTileBytes);
         const int lp = gt / T, t = gt - lp * T;
         tma_load_3d(sbase + VSmem::kQ + st * kQTileBytes, &qmap, bar(VSmem::kQFull, st), 0, t * kBM,
@@ -1264,16 +1289,16 @@ __global__ void __launch_bounds__(kNumThreads, 1)
       if (ntiles > 0) issue(0);
       for (int gt = 0; gt < ntiles; ++gt) {
         if (gt + 1 < ntiles) issue(gt + 1);
-        const int sl = gt % kTQ, k = gt / kTQ;
-        mbar_wait(bar(VSmem::kQFull, sl), k & 1);
-        mbar_wait_sleep(bar(VSmem::kTQEmpty, sl), (k & 1) ^ 1);
+        const int st = gt % kQStages, sl = gt % kVTQ, k = gt / kVTQ;
+        PROF_B(); mbar_wait(bar(VSmem::kQFull, st), (gt / kQStages) & 1); PROF_E(1);
+        PROF_B(); mbar_wait_sleep(bar(VSmem::kTQEmpty, sl), (k & 1) ^ 1); PROF_E(2);
         tc_fence_after();
-        const uint64_t sd = smem_desc_sw128(sbase + VSmem::kQ + sl * kQTileBytes);
+        const uint64_t sd = smem_desc_sw128(sbase + VSmem::kQ + st * kQTileBytes);
 #pragma unroll
         for (int kk = 0; kk < kDim / kXDim; ++kk)
           tmem_cp_128x256b(tmem_base + kTQBase + sl * kQCols + 8 * kk, sd + 2 * kk);
         commit_one(bar(VSmem::kTQFull, sl));
-        commit_one(bar(VSmem::kQEmpty, sl));
+        commit_one(bar(VSmem::kQEmpty, st));
       }
     } else if (lane == 1) {
       // ---- reference chunks: chunk c of pair lp as soon as pair lp - 1 has finished with slot c
@@ -1291,34 +1316,35 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     const int g = warp - kFirstMmaWarp;
     const int np_last = kSkip ? piece_count_last(p.m, cpr) : kPiecesPerChunk;
     uint32_t ph_t = 0;
-    if (kFold) mbar_wait(axfull, 0);
-    const uint32_t at = tmem_base + kTQBase + g * kQCols;
-    for (int gt = g, k = 0; gt < ntiles; gt += kNG, ++k) {
-      const int lp = gt / T;
-      mbar_wait(bar(VSmem::kTQFull, g), k & 1);
+    for (int gt = g; gt < ntiles; gt += kNG) {
+      const int lp = gt / T, sl = gt % kVTQ;
+      const uint32_t at = tmem_base + kTQBase + sl * kQCols;
+      PROF_B(); mbar_wait(bar(VSmem::kTQFull, sl), (gt / kVTQ) & 1); PROF_E(1);
       for (int c = 0; c < cpr; ++c) {
+        PROF_B();
         mbar_wait(bar(VSmem::kRFull, c), lp & 1);
         mbar_wait(bar(VSmem::kXReady, c), lp & 1);
+        PROF_E(2);
         const uint64_t bd0 = smem_desc_sw128(sbase + VSmem::kR + c * kRTileBytes);
         const int np = c == cpr - 1 ? np_last : kPiecesPerChunk;
 #pragma unroll
         for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
           if (kSkip && pp >= np) break;
           const uint32_t buf = g * kNB + (pp & 1);
-          mbar_wait(bar(VSmem::kTEmpty, buf), (((pp >> 1) ^ (ph_t >> (pp & 1))) & 1) ^ 1);
+          PROF_B(); mbar_wait(bar(VSmem::kTEmpty, buf), (((pp >> 1) ^ (ph_t >> (pp & 1))) & 1) ^ 1); PROF_E(0);
           tc_fence_after();
           const uint64_t bd = bd0 + pp * (kPiece * kDim >> 4);
           if (kFold)
-            mma_piece_fold_ts(tmem_base + buf * kPiece, at, bd, tmem_base + kAxCol,
-                              smem_desc_sw32(sbase + VSmem::kX + c * kXTileBytes) + pp * (kPiece * kXDim >> 4),
-                              bar(VSmem::kTFull, buf));
+            mma_piece_fold_ts_sx(tmem_base + buf * kPiece, at, bd, smem_desc_sw32(sbase + VSmem::kAx),
+                                 smem_desc_sw32(sbase + VSmem::kX + c * kXTileBytes) + pp * (kPiece * kXDim >> 4),
+                                 bar(VSmem::kTFull, buf));
           else
             mma_piece_ts(tmem_base + buf * kPiece, at, bd, bar(VSmem::kTFull, buf));
         }
         if (kSkip) ph_t ^= use_parity(np);
         mma_commit(bar(VSmem::kREmpty, c));  // this tile's MMAs on chunk c done: slot c may be refilled
       }
-      mma_commit(bar(VSmem::kTQEmpty, g));
+      mma_commit(bar(VSmem::kTQEmpty, sl));
     }
   } else {
     // ---- epilogue group g: TMEM -> registers -> top-2 -> ratio -> count (and (d1, i1, d2, i2))
@@ -1344,7 +1370,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
       const int32_t nqv = valid ? p.nq[static_cast<int64_t>(pair) * nq_ld + row] : 0;
       int done_terms = cpr;  // chunks whose column terms this warp has written (first tile of a pair only)
       auto terms = [&](int c) {
-        mbar_wait(bar(VSmem::kRFull, c), lp & 1);
+        PROF_B(); mbar_wait(bar(VSmem::kRFull, c), lp & 1); PROF_E(2);
+        PROF_B();
         vstream_terms<kFold>(sbase, colbuf, c, mcap, p.m, tig);
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // digits / zeroed rows -> tensor core
         __syncwarp();
@@ -1352,9 +1379,10 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           mbar_arrive(bar(VSmem::kXReady, c));                    // for the MMA warps (slot phase = pair)
           mbar_arrive(bar(VSmem::kColReady, (lp & 1) * kMaxSlots + c));  // for the epilogue (buffer phase)
         }
+        PROF_E(4);
       };
       if (t == 0) {  // this group computes the pair's column terms, one chunk ahead of its MMAs
-        mbar_wait(bar(VSmem::kColEmpty, lp & 1), ((lp >> 1) & 1) ^ 1);
+        PROF_B(); mbar_wait(bar(VSmem::kColEmpty, lp & 1), ((lp >> 1) & 1) ^ 1); PROF_E(5);
         terms(0);
         done_terms = 1;
       }
@@ -1378,7 +1406,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         }
         // this chunk's column buffer is written (a per-pair-buffer barrier: the slot's xready may already
         // be in the next pair's phase once every tile's MMAs have left chunk c)
-        mbar_wait(bar(VSmem::kColReady, (lp & 1) * kMaxSlots + c), (lp >> 1) & 1);
+        PROF_B(); mbar_wait(bar(VSmem::kColReady, (lp & 1) * kMaxSlots + c), (lp >> 1) & 1); PROF_E(5);
         const uint32_t ck = colbuf + c * kColBytes;
         const int np = c == cpr - 1 ? np_last : kPiecesPerChunk;
         if constexpr (kFold) {
@@ -1393,7 +1421,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           for (int pp = 0; pp < kPiecesPerChunk; ++pp) {
             if (kSkip && pp >= np) break;
             const uint32_t buf = g * kNB + (pp & 1);
-            mbar_wait(bar(VSmem::kTFull, buf), ((pp >> 1) ^ (ph_t >> (pp & 1))) & 1);
+            PROF_B(); mbar_wait(bar(VSmem::kTFull, buf), ((pp >> 1) ^ (ph_t >> (pp & 1))) & 1); PROF_E(0);
+            PROF_B();
             tc_fence_after();
             tmem_ld64(taddr_q + buf * kPiece, v);
             tmem_wait_ld();
@@ -1401,6 +1430,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(bar(VSmem::kTEmpty, buf));
+            PROF_E(3);
+            PROF_B();
             if (kpc >= (pp + 1) * kPiece) {
               scan32_fold<false>(v, 32, R, T1, T2);
               scan32_fold<false>(v + 32, 32, R, T1, T2);
@@ -1408,11 +1439,14 @@ __global__ void __launch_bounds__(kNumThreads, 1)
               scan32_fold<true>(v, kpc - pp * kPiece, R, T1, T2);
               scan32_fold<true>(v + 32, kpc - pp * kPiece - 32, R, T1, T2);
             }
+            PROF_E(1);
           }
+          PROF_B();
           int x1, x2;
           finish_fold(R, T1, T2, x1, x2);
           G2 = max3i(min(G1, x1), G2, x2);
           G1 = max(G1, x1);
+          PROF_E(1);
         } else {
           int R[16];
 #pragma unroll
@@ -1453,6 +1487,7 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         }
         if (kSkip) ph_t ^= use_parity(np);
       }
+      PROF_B();
       if constexpr (kFold) {
         // d = N_Q - 2X - p, p in {0, 1}: the ratio test from the bounds, exact recompute if open
         const bool real2 = G2 > INT_MIN;
@@ -1505,9 +1540,11 @@ __global__ void __launch_bounds__(kNumThreads, 1)
         mbar_arrive(bar(VSmem::kColEmpty, lp & 1));  // this warp-tile's last read of the pair's column buffer
       }
       __syncwarp();
+      PROF_E(6);
     }
   }
 
+  PROF_FLUSH();
   tc_fence_before();
   __syncthreads();
   if (warp == kFirstMmaWarp) {
