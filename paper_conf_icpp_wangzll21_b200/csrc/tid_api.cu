@@ -1562,10 +1562,21 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
     return !(e && e[0] == '0');
   }();
   const bool fold = fold_ok && nn_out == nullptr;
-  TRY(idx->ws_nq.ensure(static_cast<size_t>(P) * T * kBM * 4, "query norms"));
-  if (fold) TRY(idx->ws_qs.ensure(static_cast<size_t>(P) * n * kDim, "shifted queries"));
-  launch_query_prep(dq, P, n, T, idx->ws_nq.as<int32_t>(), fold ? idx->ws_qs.as<uint8_t>() : nullptr, s);
-  count_kernel(idx);
+  // pairs streamed through per-chunk reference slots, queries shifted / normed on chip (TID_VERIFY_STREAM=0:
+  // the job kernel after a query-prep pass, for A/B).  The stream kernel's parity waits assume every
+  // group runs a tile of every pair (T >= 3 = kNG); with fewer tiles per query a group skips pairs, so
+  // n <= 256 takes the job kernel.
+  static const bool stream_ok = [] {
+    const char* e = getenv("TID_VERIFY_STREAM");
+    return !(e && e[0] == '0');
+  }();
+  const bool streamed = stream_ok && T >= kNG;
+  if (!streamed) {
+    TRY(idx->ws_nq.ensure(static_cast<size_t>(P) * T * kBM * 4, "query norms"));
+    if (fold) TRY(idx->ws_qs.ensure(static_cast<size_t>(P) * n * kDim, "shifted queries"));
+    launch_query_prep(dq, P, n, T, idx->ws_nq.as<int32_t>(), fold ? idx->ws_qs.as<uint8_t>() : nullptr, s);
+    count_kernel(idx);
+  }
   const bool dev_counts = is_device_ptr(counts_out);
   TRY(idx->ws_counts.ensure(static_cast<size_t>(P) * 4, "pair counts"));
   uint32_t* counts = dev_counts ? counts_out : idx->ws_counts.as<uint32_t>();
@@ -1581,7 +1592,7 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
     }
   }
   CUtensorMap qmap, rmap;
-  TRY(make_map(&qmap, fold ? idx->ws_qs.p : dq, P, n, kBM));
+  TRY(make_map(&qmap, (fold && !streamed) ? idx->ws_qs.p : dq, P, n, kBM));
   TRY(make_map(&rmap, dr, P, m, kBN));
   MatchParams p{};
   p.mode = kModeVerify;
@@ -1597,7 +1608,7 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
   p.ref_map_base = 0;
   p.colkey = nullptr;  // computed in the kernel
   p.m_valid = dmr;
-  p.nq = idx->ws_nq.as<int32_t>();
+  p.nq = streamed ? nullptr : idx->ws_nq.as<int32_t>();
   p.n_valid = dnv;
   p.n_rows = n;
   p.counts = counts;
@@ -1622,18 +1633,12 @@ tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t
     CU(cudaEventRecord(e0, s));
   }
   if (fold) {
-    p.qs = idx->ws_qs.as<uint8_t>();  // exact recompute of the rare +-1-undecided rows
+    // exact recompute of the rare +-1-undecided rows (the stream kernel reads the raw queries)
+    p.qs = streamed ? dq : idx->ws_qs.as<uint8_t>();
     p.rdesc = dr;
     p.slot_banks = 1;
   }
-  // pairs streamed through per-chunk reference slots (TID_VERIFY_STREAM=0: the job kernel, for A/B).
-  // The stream kernel's parity waits assume every group runs a tile of every pair (T >= 3 = kNG); with
-  // fewer tiles per query a group skips pairs, so n <= 256 takes the job kernel.
-  static const bool stream_ok = [] {
-    const char* e = getenv("TID_VERIFY_STREAM");
-    return !(e && e[0] == '0');
-  }();
-  cudaError_t e = (stream_ok && T >= kNG) ? launch_verify_stream(p, qmap, rmap, fold, grid, s) : launch_match(p, qmap, rmap, fold, grid, s);
+  cudaError_t e = streamed ? launch_verify_stream(p, qmap, rmap, fold, grid, s) : launch_match(p, qmap, rmap, fold, grid, s);
   if (e != cudaSuccess) return fail(TID_ECUDA, "match kernel launch: %s", cudaGetErrorString(e));
   if (idx->prof) {
     CU(cudaEventRecord(e1, s));
