@@ -1152,16 +1152,15 @@ cudaError_t launch_match(const MatchParams& p, const CUtensorMap& qmap, const CU
 // tiles gt - 4 and earlier (one thread, in order).
 constexpr int kVTQ = 4;
 static_assert(kTQBase + kVTQ * kQCols <= 512, "TMEM budget of the streamed verification");
-constexpr int kVQStages = 2;  // query tiles land here (TMA), are shifted / normed by the producer warp, copied to TMEM
+constexpr int kVQStages = kNG;  // query stage g holds group g's next tile (TMA), prepared by the group, copied to TMEM
 struct VSmem {
   static constexpr uint32_t kR = 0;                                        // 4 x 32 KiB reference chunks
-  static constexpr uint32_t kQ = kR + kMaxSlots * kRTileBytes;             // 2 x 16 KiB query stages
+  static constexpr uint32_t kQ = kR + kMaxSlots * kRTileBytes;             // 3 x 16 KiB query stages
   static constexpr uint32_t kX = kQ + kVQStages * kQTileBytes;             // 4 x 8 KiB norm digits (folded)
   static constexpr uint32_t kAx = kX + kMaxSlots * kXTileBytes;            // constant norm-term operand
   static constexpr uint32_t kCol = kAx + kBM * kXDim;                      // 2 pair buffers x 4 x 1 KiB
   static constexpr uint32_t kColPair = kMaxSlots * kColBytes;
-  static constexpr uint32_t kNQ = kCol + 2 * kColPair;                     // N_Q of the rows of each TMEM tile slot
-  static constexpr uint32_t kBar = kNQ + kVTQ * kBM * 4;
+  static constexpr uint32_t kBar = kCol + 2 * kColPair;
   static constexpr uint32_t kQFull = kBar;
   static constexpr uint32_t kQEmpty = kQFull + 8 * kVQStages;
   static constexpr uint32_t kRFull = kQEmpty + 8 * kVQStages;
@@ -1173,8 +1172,8 @@ struct VSmem {
   static constexpr uint32_t kTQEmpty = kTQFull + 8 * kVTQ;
   static constexpr uint32_t kColEmpty = kTQEmpty + 8 * kVTQ;                // per pair buffer: all readers done
   static constexpr uint32_t kColReady = kColEmpty + 8 * 2;               // per (pair buffer, chunk): terms written
-  static constexpr uint32_t kNQReady = kColReady + 8 * 2 * kMaxSlots;      // per TMEM tile slot: N_Q written
-  static constexpr uint32_t kTmemPtr = kNQReady + 8 * kVTQ;
+  static constexpr uint32_t kPrepped = kColReady + 8 * 2 * kMaxSlots;      // per stage: tile shifted + normed
+  static constexpr uint32_t kTmemPtr = kPrepped + 8 * kVQStages;
   static constexpr uint32_t kEnd = kTmemPtr + 16;
   static constexpr uint32_t kAlloc = kEnd + 1024;
 };
@@ -1256,12 +1255,12 @@ __global__ void __launch_bounds__(kNumThreads, 1)
   if (threadIdx.x == 0) {
     prefetch_tmap(&qmap);
     prefetch_tmap(&rmap);
-    for (int i = 0; i < kVQStages; ++i) { mbar_init(bar(VSmem::kQFull, i), 1); mbar_init(bar(VSmem::kQEmpty, i), 1); }
-    for (int i = 0; i < kVTQ; ++i) {
-      mbar_init(bar(VSmem::kTQFull, i), 1);
-      mbar_init(bar(VSmem::kTQEmpty, i), 1);
-      mbar_init(bar(VSmem::kNQReady, i), 1);
+    for (int i = 0; i < kVQStages; ++i) {
+      mbar_init(bar(VSmem::kQFull, i), 1);
+      mbar_init(bar(VSmem::kQEmpty, i), 1);
+      mbar_init(bar(VSmem::kPrepped, i), 4);  // the group's 4 epilogue warps
     }
+    for (int i = 0; i < kVTQ; ++i) { mbar_init(bar(VSmem::kTQFull, i), 1); mbar_init(bar(VSmem::kTQEmpty, i), 1); }
     for (int c = 0; c < kMaxSlots; ++c) {
       mbar_init(bar(VSmem::kRFull, c), 1);
       mbar_init(bar(VSmem::kREmpty, c), T);   // one MMA commit per tile of the pair
@@ -1283,104 +1282,64 @@ __global__ void __launch_bounds__(kNumThreads, 1)
   const uint32_t tmem_base = *tmem_ptr_smem;
 
   // -DTID_PROF buckets: epilogue 0 wait-accumulator 1 scan + chunk finish 2 wait for a chunk (terms)
-  // 3 TMEM load + release 4 column terms 5 wait column buffer 6 tile tail; MMA 0 wait-free-accumulator
-  // 1 wait-query 2 wait-ref; producer 0 wait-stage 1 wait-TMA 2 wait-TMEM-slot 3 query prep (N_Q, shift)
+  // 3 TMEM load + release 4 column terms 5 wait column buffer 6 next tile's query prep + tile tail;
+  // MMA 0 wait-free-accumulator 1 wait-query 2 wait-ref; producer 0 wait-stage 1 wait-prep 2 wait-TMEM-slot
   PROF_DECL
   if (warp == kProducerWarp) {
-    // ---- query tiles (whole warp) + reference chunks (lane 0, serviced whenever lane 0 waits).
-    // Tile gt: TMA of the raw u8 rows into stage gt % 2; the warp computes N_Q of every row (Alg. 1
-    // step 2) into the slot's N_Q array and, for the folded path, shifts the rows in place
-    // (q' = q ^ 0x80 = q - 128 as s8; rows beyond n stay zero); then SMEM -> TMEM slot gt % 4.  No
-    // separate pass over the queries in HBM.  Reference chunk c of pair lp is loaded as soon as pair
-    // lp - 1 has finished with slot c.
-    int r_lp = 0, r_c = 0;  // next reference chunk (lane 0)
-    auto service_refs = [&]() {
-      while (r_lp < npairs) {
-        uint32_t free_;
-        asm volatile(
-            "{\n\t.reg .pred P1;\n\tmbarrier.test_wait.parity.shared::cta.b64 P1, [%1], %2;\n\t"
-            "selp.u32 %0, 1, 0, P1;\n\t}"
-            : "=r"(free_)
-            : "r"(bar(VSmem::kREmpty, r_c)), "r"(static_cast<uint32_t>((r_lp & 1) ^ 1))
-            : "memory");
-        if (!free_) return;
-        mbar_expect_tx(bar(VSmem::kRFull, r_c), kRTileBytes);
-        tma_load_3d(sbase + VSmem::kR + r_c * kRTileBytes, &rmap, bar(VSmem::kRFull, r_c), 0, r_c * kBN,
-                    static_cast<int>(blockIdx.x) + r_lp * static_cast<int>(gridDim.x));
-        if (++r_c == cpr) { r_c = 0; ++r_lp; }
-      }
-    };
-    auto wait_serving = [&](uint32_t b, uint32_t par) {  // lane 0: poll, issuing reference loads meanwhile
-      uint32_t ns = 32;
-      while (true) {
-        uint32_t done;
-        asm volatile(
-            "{\n\t.reg .pred P1;\n\tmbarrier.test_wait.parity.shared::cta.b64 P1, [%1], %2;\n\t"
-            "selp.u32 %0, 1, 0, P1;\n\t}"
-            : "=r"(done)
-            : "r"(b), "r"(par)
-            : "memory");
-        if (done) return;
-        service_refs();
-        __nanosleep(ns);
-        ns = ns < 256 ? ns * 2 : 256;
-      }
-    };
-    auto issue = [&](int gt) {
-      const int st = gt % kVQStages, k = gt / kVQStages;
-      PROF_B(); wait_serving(bar(VSmem::kQEmpty, st), (k & 1) ^ 1); PROF_E(0);
-      mbar_expect_tx(bar(VSmem::kQFull, st), kQTileBytes);
-      const int lp = gt / T, t = gt - lp * T;
-      tma_load_3d(sbase + VSmem::kQ + st * kQTileBytes, &qmap, bar(VSmem::kQFull, st), 0, t * kBM,
-                  static_cast<int>(blockIdx.x) + lp * static_cast<int>(gridDim.x));
-    };
+    // ---- lane 0: query tiles + reference chunks.  Tile gt (group g = gt % 3) lands raw in stage g by TMA;
+    // the group's epilogue warps compute N_Q of its rows and, for the folded path, shift them in place
+    // (during the group's previous tile, off its critical path); then SMEM -> TMEM slot gt % 4 here.
+    // Reference chunk c of pair lp is loaded as soon as pair lp - 1 has finished with slot c (serviced
+    // whenever lane 0 waits).
     if (lane == 0) {
-      service_refs();
-      if (ntiles > 0) issue(0);
-    }
-    for (int gt = 0; gt < ntiles; ++gt) {
-      const int st = gt % kVQStages, sl = gt % kVTQ, k = gt / kVTQ;
-      if (lane == 0) {
-        if (gt + 1 < ntiles) issue(gt + 1);
-        PROF_B(); wait_serving(bar(VSmem::kQFull, st), (gt / kVQStages) & 1); PROF_E(1);
-        // the slot's previous tile (gt - 4) has left TMEM; its epilogue read its N_Q at tile start
-        PROF_B(); wait_serving(bar(VSmem::kTQEmpty, sl), (k & 1) ^ 1); PROF_E(2);
-      }
-      __syncwarp();
-      PROF_B();
-      {
-        const uint32_t tile = sbase + VSmem::kQ + st * kQTileBytes;
-        const int lp = gt / T, t = gt - lp * T;
-        const int rows_real = min(kBM, p.n_rows - t * kBM);
-#pragma unroll
-        for (int i = 0; i < kBM / 32; ++i) {
-          const int row = lane + 32 * i;
-          const uint32_t ra = tile + row * kDim;
-          uint32_t acc = 0;
-#pragma unroll
-          for (int w = 0; w < kDim / 16; ++w) {
-            // a row's 16-byte chunks sit permuted within its 128-byte line (SWIZZLE_128B): visiting them
-            // in the order w ^ (row & 7) keeps the 8 lanes of a phase on distinct banks
-            const uint32_t ca = ra + 16 * (w ^ (row & 7));
-            const int4 x4 = lds128(ca);
-            acc = __dp4a(static_cast<uint32_t>(x4.x), static_cast<uint32_t>(x4.x), acc);
-            acc = __dp4a(static_cast<uint32_t>(x4.y), static_cast<uint32_t>(x4.y), acc);
-            acc = __dp4a(static_cast<uint32_t>(x4.z), static_cast<uint32_t>(x4.z), acc);
-            acc = __dp4a(static_cast<uint32_t>(x4.w), static_cast<uint32_t>(x4.w), acc);
-            if (kFold && row < rows_real)
-              asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(ca), "r"(x4.x ^ 0x80808080),
-                           "r"(x4.y ^ 0x80808080), "r"(x4.z ^ 0x80808080), "r"(x4.w ^ 0x80808080)
-                           : "memory");
-          }
-          asm volatile("st.shared.u32 [%0], %1;" ::"r"(sbase + VSmem::kNQ + (sl * kBM + row) * 4), "r"(acc)
-                       : "memory");
+      int r_lp = 0, r_c = 0;  // next reference chunk
+      auto service_refs = [&]() {
+        while (r_lp < npairs) {
+          uint32_t free_;
+          asm volatile(
+              "{\n\t.reg .pred P1;\n\tmbarrier.test_wait.parity.shared::cta.b64 P1, [%1], %2;\n\t"
+              "selp.u32 %0, 1, 0, P1;\n\t}"
+              : "=r"(free_)
+              : "r"(bar(VSmem::kREmpty, r_c)), "r"(static_cast<uint32_t>((r_lp & 1) ^ 1))
+              : "memory");
+          if (!free_) return;
+          mbar_expect_tx(bar(VSmem::kRFull, r_c), kRTileBytes);
+          tma_load_3d(sbase + VSmem::kR + r_c * kRTileBytes, &rmap, bar(VSmem::kRFull, r_c), 0, r_c * kBN,
+                      static_cast<int>(blockIdx.x) + r_lp * static_cast<int>(gridDim.x));
+          if (++r_c == cpr) { r_c = 0; ++r_lp; }
         }
-      }
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // shifted rows -> tensor-core copy
-      __syncwarp();
-      PROF_E(3);
-      if (lane == 0) {
-        mbar_arrive(bar(VSmem::kNQReady, sl));
+      };
+      auto wait_serving = [&](uint32_t b, uint32_t par) {  // poll, issuing reference loads meanwhile
+        uint32_t ns = 32;
+        while (true) {
+          uint32_t done;
+          asm volatile(
+              "{\n\t.reg .pred P1;\n\tmbarrier.test_wait.parity.shared::cta.b64 P1, [%1], %2;\n\t"
+              "selp.u32 %0, 1, 0, P1;\n\t}"
+              : "=r"(done)
+              : "r"(b), "r"(par)
+              : "memory");
+          if (done) return;
+          service_refs();
+          __nanosleep(ns);
+          ns = ns < 256 ? ns * 2 : 256;
+        }
+      };
+      auto issue = [&](int gt) {  // tile gt -> stage gt % 3 (its previous occupant, tile gt - 3, is in TMEM)
+        const int st = gt % kVQStages, k = gt / kVQStages;
+        PROF_B(); wait_serving(bar(VSmem::kQEmpty, st), (k & 1) ^ 1); PROF_E(0);
+        mbar_expect_tx(bar(VSmem::kQFull, st), kQTileBytes);
+        const int lp = gt / T, t = gt - lp * T;
+        tma_load_3d(sbase + VSmem::kQ + st * kQTileBytes, &qmap, bar(VSmem::kQFull, st), 0, t * kBM,
+                    static_cast<int>(blockIdx.x) + lp * static_cast<int>(gridDim.x));
+      };
+      service_refs();
+      for (int gt = 0; gt < min(ntiles, kVQStages); ++gt) issue(gt);
+      for (int gt = 0; gt < ntiles; ++gt) {
+        const int st = gt % kVQStages, sl = gt % kVTQ;
+        PROF_B(); wait_serving(bar(VSmem::kPrepped, st), (gt / kVQStages) & 1); PROF_E(1);
+        // the slot's previous tile (gt - 4) has left TMEM
+        PROF_B(); wait_serving(bar(VSmem::kTQEmpty, sl), ((gt / kVTQ) & 1) ^ 1); PROF_E(2);
         tc_fence_after();
         const uint64_t sd = smem_desc_sw128(sbase + VSmem::kQ + st * kQTileBytes);
 #pragma unroll
@@ -1388,12 +1347,10 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           tmem_cp_128x256b(tmem_base + kTQBase + sl * kQCols + 8 * kk, sd + 2 * kk);
         commit_one(bar(VSmem::kTQFull, sl));
         commit_one(bar(VSmem::kQEmpty, st));
+        if (gt + kVQStages < ntiles) issue(gt + kVQStages);
         service_refs();
       }
-      __syncwarp();
-    }
-    if (lane == 0) {  // the remaining reference chunks
-      while (r_lp < npairs) {
+      while (r_lp < npairs) {  // the remaining reference chunks
         mbar_wait_sleep(bar(VSmem::kREmpty, r_c), (r_lp & 1) ^ 1);
         service_refs();
       }
@@ -1445,6 +1402,34 @@ __global__ void __launch_bounds__(kNumThreads, 1)
     const int np_last = kSkip ? piece_count_last(p.m, cpr) : kPiecesPerChunk;
     uint32_t ph_t = 0;
     uint32_t v[64];
+    // Query prep of tile gt (in stage g): this thread's row N_Q (Alg. 1 step 2) and, folded, the
+    // shifted row q' = q ^ 0x80 (= q - 128 as s8; rows beyond n stay zero).  A row's 16-byte chunks sit
+    // permuted within its 128-byte line (SWIZZLE_128B): neither the sum nor the XOR depends on the order.
+    auto prep_tile = [&](int gt) -> int32_t {
+      const int lp = gt / T, t = gt - lp * T;
+      mbar_wait(bar(VSmem::kQFull, g), (gt / kNG) & 1);
+      const uint32_t ra = sbase + VSmem::kQ + g * kQTileBytes + row_in_tile * kDim;
+      const bool shift = kFold && t * kBM + row_in_tile < p.n_rows;
+      uint32_t acc = 0;
+#pragma unroll
+      for (int w = 0; w < kDim / 16; ++w) {
+        const uint32_t ca = ra + 16 * (w ^ (row_in_tile & 7));  // 8 lanes of a phase on distinct banks
+        const int4 x4 = lds128(ca);
+        acc = __dp4a(static_cast<uint32_t>(x4.x), static_cast<uint32_t>(x4.x), acc);
+        acc = __dp4a(static_cast<uint32_t>(x4.y), static_cast<uint32_t>(x4.y), acc);
+        acc = __dp4a(static_cast<uint32_t>(x4.z), static_cast<uint32_t>(x4.z), acc);
+        acc = __dp4a(static_cast<uint32_t>(x4.w), static_cast<uint32_t>(x4.w), acc);
+        if (shift)
+          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(ca), "r"(x4.x ^ 0x80808080),
+                       "r"(x4.y ^ 0x80808080), "r"(x4.z ^ 0x80808080), "r"(x4.w ^ 0x80808080)
+                       : "memory");
+      }
+      if (kFold) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // shifted rows -> TMEM copy
+      __syncwarp();
+      if (lane == 0) mbar_arrive(bar(VSmem::kPrepped, g));
+      return static_cast<int32_t>(acc);
+    };
+    int32_t nq_next = 0;
     for (int gt = g; gt < ntiles; gt += kNG) {
       const int lp = gt / T, t = gt - lp * T;
       const int pair = static_cast<int>(blockIdx.x) + lp * static_cast<int>(gridDim.x);
@@ -1453,12 +1438,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
       const int nvalid = min(p.n_valid ? p.n_valid[pair] : p.n_rows, p.n_rows);
       const int row = t * kBM + row_in_tile;
       const bool valid = row < nvalid;
-      // N_Q of this row, computed by the producer warp from the tile (slot gt % 4)
-      const int qsl = gt % kVTQ;
-      mbar_wait(bar(VSmem::kNQReady, qsl), (gt / kVTQ) & 1);
-      int32_t nqv;
-      asm volatile("ld.shared.s32 %0, [%1];" : "=r"(nqv) : "r"(sbase + VSmem::kNQ + (qsl * kBM + row_in_tile) * 4));
-      if (!valid) nqv = 0;
+      if (gt == g) nq_next = prep_tile(gt);  // the group's first tile: nothing to overlap it with
+      const int32_t nqv = valid ? nq_next : 0;
       int done_terms = cpr;  // chunks whose column terms this warp has written (first tile of a pair only)
       auto terms = [&](int c) {
         PROF_B(); mbar_wait(bar(VSmem::kRFull, c), lp & 1); PROF_E(2);
@@ -1577,6 +1558,8 @@ __global__ void __launch_bounds__(kNumThreads, 1)
           }
         }
         if (kSkip) ph_t ^= use_parity(np);
+        // the group's next tile (already in stage g): prepared here, off the MMA's critical path
+        if (c == 0 && gt + kNG < ntiles) { PROF_B(); nq_next = prep_tile(gt + kNG); PROF_E(6); }
       }
       PROF_B();
       if constexpr (kFold) {
