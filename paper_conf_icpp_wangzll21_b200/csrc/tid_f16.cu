@@ -46,7 +46,12 @@ constexpr uint32_t kXTile = kBN * kXH * 2;          // 8 KiB: 256 reference rows
 // MMA pieces of kFN = 128 columns through kFNB = 4 TMEM buffers (512 columns): a reference chunk
 // of 256 keypoints is 2 pieces; global piece gp of the CTA uses buffer gp % 4 with phase
 // (gp / 4) & 1, so with one chunk per reference the MMA runs up to 1.5 units ahead of the epilogue.
-constexpr int kFN = 128;
+#ifndef TID_F16_N
+#define TID_F16_N 128
+#endif
+constexpr int kFN = TID_F16_N;  // 256: one MMA per chunk through 2 buffers (B / A operand bytes per
+                                // tensor cycle 96 instead of 128, the shared-memory port's width)
+static_assert(kFN == 128 || kFN == 256, "MMA N");
 constexpr int kFPieces = kBN / kFN;                 // pieces per 256-column chunk
 constexpr int kFNB = 512 / kFN;                     // TMEM buffers
 
@@ -310,18 +315,23 @@ __global__ void __launch_bounds__(kThreads, 1)
         // every chunk's pieces into one two-partition state: two columns of different loads are in
         // different P groups, two of one load differ in position mod 16, so the top-2 stays exact
 #pragma unroll
-        for (int pc = 0; pc < kCpr * kFPieces; ++pc, ++gp) {  // one x64 load (128 columns) per piece
+        for (int pc = 0; pc < kCpr * kFPieces; ++pc, ++gp) {  // one x64 load per 128 columns of a piece
           const int buf = gp % kFNB;
           bar_wait(tfull(buf), (gp / kFNB) & 1);
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-          ld16x64(tq + buf * kFN, v);
-          asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-          __syncwarp();
-          if (lane == 0) bar_arrive(tempty(buf));
+#pragma unroll
+          for (int l = 0; l < kFN / 128; ++l) {
+            ld16x64(tq + buf * kFN + l * 128, v);
+            if (l == kFN / 128 - 1) {  // the piece is in registers: buffer free
+              asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+              __syncwarp();
+              if (lane == 0) bar_arrive(tempty(buf));
+            }
 #ifndef TID_NOSCAN  // timing experiment only
-          scan32(v, Rm, T1, T2);
-          scan32(v + 32, Rm, T1, T2);
+            scan32(v, Rm, T1, T2);
+            scan32(v + 32, Rm, T1, T2);
 #endif
+          }
         }
         int x1, x2;
         finish(Rm, T1, T2, x1, x2);

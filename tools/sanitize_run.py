@@ -71,3 +71,14 @@ with tid.Index(ref_kp=256, query_kp_max=1024) as idx:
     torch.cuda.synchronize()
 assert np.array_equal(did.cpu().numpy(), e_ids)
 print("sanitize run ok")
+# streamed verification (n > 256): several pairs per CTA (grid 2), ragged n_q / m_r, nn and counts-only
+Qs, Rs, _ = tidgen.pairs(7, 500, 600, n_planted=150)
+n_q = np.array([500, 3, 257, 400, 129, 500, 1], np.int32)
+m_r = np.array([600, 2, 300, 599, 256, 257, 600], np.int32)
+with tid.Index(ref_kp=256, query_kp_max=1024) as idx:
+    idx.set_tuning(grid=2)
+    vc, nn = idx.verify(Qs, Rs, n_q=n_q, m_r=m_r)
+    vf, _ = idx.verify(Qs, Rs, n_q=n_q, m_r=m_r, want_nn=False)
+ec, _ = oracle.verify(Qs, Rs, n_q=n_q, m_r=m_r)
+assert np.array_equal(vc.astype(np.int64), ec) and np.array_equal(vf.astype(np.int64), ec)
+print("streamed verification ok")
