@@ -528,12 +528,18 @@ __device__ __forceinline__ void norm_digits(int32_t W, uint32_t (&w8)[8]) {
   const uint32_t E = W > 0 ? static_cast<uint32_t>(W) >> 1 : 0u;
   const uint32_t hi = E / 255u, lo = E - 255u * hi;
   const uint32_t q = hi / 255u, rem = hi - 255u * q;
+  // Rank word i (ranks 4i .. 4i+3) has t = q - 4i full bytes, then rem, then zeros: one byte permute of
+  // {0, b = rem | 0xFFFFFF00} whose selector (nibble 5 = 0xFF, 4 = rem, 0 = 0x00) is a 16-bit window
+  // of the nibble string 0x4_5555_5555 at 4 (8 - clamp(t, -1, 5)) bits (tools/digits_check.py checks
+  // every W against the greedy encoding).
+  const uint32_t b = 0xFFFFFF00u | rem;
+  const int s0 = 32 - 4 * static_cast<int>(q);
   uint32_t rk[8];  // rank words: byte b of rk[i] = digit of rank 4 i + b
 #pragma unroll
   for (int i = 0; i < 8; ++i) {
-    const int d = static_cast<int>(q) - 4 * i;  // full bytes in this word
-    rk[i] = d >= 4 ? 0xFFFFFFFFu
-                   : (d < 0 ? 0u : ((d == 0 ? 0u : (0xFFFFFFFFu >> (32 - 8 * d))) | (rem << (8 * d))));
+    const int sh = min(max(s0 + 16 * i, 12), 36);
+    const uint32_t sel = static_cast<uint32_t>(0x0000000455555555ull >> sh);
+    rk[i] = __byte_perm(0u, b, sel);
   }
   w8[0] = rk[0];
   w8[1] = rk[1];
