@@ -39,7 +39,10 @@ def timed(fn, reps, warm=3):
     torch.cuda.synchronize()
     ts = []
     with ClockSampler(torch.cuda.current_device()) as clk:
-        for _ in range(reps):
+        t_start = time.perf_counter()
+        # at least `reps` calls and at least 1.5 s, so that nvidia-smi (200 ms period, slow to start)
+        # samples the clocks during timed calls even for sub-millisecond ones (C1, C2)
+        while len(ts) < reps or (time.perf_counter() - t_start < 1.5 and len(ts) < 100000):
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
             fn()
@@ -82,7 +85,7 @@ def search_case(name, B, n, R, m, k, reps, hbm_budget=0, host_budget=0, chunk=0)
     out = {"case": name, "queries": B, "query_kp": n, "refs": R, "ref_kp": m, "top_k": k,
            "p50_ms": p50, "p99_ms": float(np.percentile(ts, 99)), "comparisons_per_s": B * R / (p50 / 1e3),
            "e2e_p50_ms": statistics.median(ts_e2e), "e2e_comparisons_per_s": B * R / (statistics.median(ts_e2e) / 1e3),
-           "match_kernel_ms_per_search": st["match_ms"] / reps if st["match_launches"] else None,
+           "match_kernel_ms_per_search": st["match_ms"] / len(ts) if st["match_launches"] else None,
            "h2d_GBps": (st["h2d_bytes"] / (sum(ts) / 1e3) / 1e9) if st["h2d_bytes"] else 0.0,
            "planted_top1": top1, "info": idx.info(), "clocks": dict(LAST_CLOCKS),
            "tensor_tops_int8": 2.0 * B * R * n * m * 128 / (p50 / 1e3) / 1e12}
