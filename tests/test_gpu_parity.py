@@ -707,3 +707,22 @@ def test_verify_streamed_pairs(tid, rng, n, m, grid):
     for p in range(P):
         np.testing.assert_array_equal(nn[p, :n_q[p]].astype(np.int64), nn_from_oracle(enn[p, :n_q[p]]))
         assert (nn[p, n_q[p]:] == -1).all()
+
+
+@pytest.mark.parametrize("B,n,grid", [(1, 1000, 2), (2, 1000, 3), (3, 600, 1), (16, 100, 4)])
+def test_search_small_batch_slot_banks(tid, B, n, grid):
+    """Small batches (B * T <= 16 query tiles) alternate two banks of reference slots, and the producer
+    warp expands the next job's norm digits while the current job runs; a forced small grid makes each
+    CTA run many such jobs back to back (ragged last group, planted targets), bit-exact vs the oracle."""
+    R, m = 301, 256
+    refs, kp = tidgen.refs(11, R, m, kp_min=180)
+    qs, tg = tidgen.queries(12, B, n, R_total=R, m=m, n_planted=min(120, n))
+    with tid.Index(ref_kp=m, query_kp_max=1024) as idx:
+        idx.add_references(refs, kp)
+        idx.set_tuning(grid=grid)
+        counts = idx.search_counts(qs)
+        ids, cnt = idx.search(qs, 5)
+    e_ids, e_cnt, e_counts = oracle.search(qs, refs, 5, kp=kp)
+    np.testing.assert_array_equal(counts.astype(np.int64), e_counts)
+    np.testing.assert_array_equal(ids, e_ids)
+    np.testing.assert_array_equal(cnt, e_cnt)
