@@ -681,7 +681,7 @@ def test_verify_counts_only_folded(tid, rng, n, m, P):
 
 
 @pytest.mark.parametrize("n,m,grid", [(1000, 1000, 3), (300, 600, 2), (129, 257, 5), (100, 2, 4), (250, 384, 1),
-                                      (700, 900, 7)])
+                                      (700, 900, 7), (500, 2, 3), (384, 1024, 2), (1024, 256, 2), (257, 64, 1)])
 def test_verify_streamed_pairs(tid, rng, n, m, grid):
     """Many pairs per CTA (a forced small grid): the pair-streaming verification kernel refills each
     reference slot as soon as the previous pair's tiles have left it, runs tile gt of its pair sequence
