@@ -181,9 +181,12 @@ tid_status tid_search_counts(tid_index* idx, const uint8_t* queries, const int32
  *   nn_out : nullable int32 [P][n][4] = (d1, i1, d2, i2) per query row, the exact
  *            squared distances and reference-keypoint indices of the two nearest
  *            neighbours (Alg. 1 step 8's 2 x n output); a missing
- *            neighbour (m_r < 2) is (-1, -1).  Rows >= n_q[p] are not written.
- * Without nn_out the counts come from the search path's folded kernel run on the pairs (same exact
- * results).
+ *            neighbour (m_r < 2) is (-1, -1).  Rows >= n_q[p] are written as (-1, -1, -1, -1).
+ * Without nn_out the counts come from the search path's folded arithmetic (s8 x u8 + norm K-step) run
+ * on the pairs (same exact results).  For n > 256 the pairs stream through one persistent kernel that
+ * also computes N_Q and the reference norms on chip (no preparation pass).
+ * Errors: TID_EINVAL for null pointers or sizes out of range (nothing launched); TID_ECUDA / TID_ENOMEM
+ * from the device.
  */
 tid_status tid_verify(tid_index* idx, const uint8_t* q, int32_t n, const uint8_t* r, int32_t m,
                       int64_t P, const int32_t* n_q, const int32_t* m_r,
