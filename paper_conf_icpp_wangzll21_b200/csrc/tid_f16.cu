@@ -295,6 +295,8 @@ __global__ void __launch_bounds__(kThreads, 1)
     const uint32_t tq = tmem + (static_cast<uint32_t>(quarter * 32 + 16 * half) << 16);
     const int row_in_tile = quarter * 32 + 16 * half + (lane >> 2) + 8 * (lane & 1);
     const double c2 = 2.0 * static_cast<double>(*cterm);
+    const float c2f = static_cast<float>(c2);  // 2C: a power of two, exact in fp32
+    const float den2f = static_cast<float>(den2), num2f = static_cast<float>(num2);  // small integers, exact
     uint32_t rc = 0, gp = 0;
     uint32_t v[64];
     for (int64_t j = blockIdx.x; j < n_jobs; j += gridDim.x, ++rc) {
@@ -340,11 +342,27 @@ __global__ void __launch_bounds__(kThreads, 1)
           x2 = mx3(min(x1, o1), x2, o2);
           x1 = max(x1, o1);
         }
-        // d = N_Q + 2C - 2X (fp64 from the fp32 values; clamped at 0); padded columns have X < 0
-        const double d1 = fmax(double(nqv) + c2 - 2.0 * double(__int_as_float(x1)), 0.0);
-        const double d2 = fmax(double(nqv) + c2 - 2.0 * double(__int_as_float(x2)), 0.0);
-        // ratio test in fp64
-        const bool pass = valid && x2 >= 0 && double(den2) * d1 < double(num2) * d2;
+        // d = N_Q + 2C - 2X (clamped at 0; padded columns have X < 0) and the ratio test
+        // den^2 d1 < num^2 d2, decided exactly as in fp64 from these fp32 values (R10).
+        // B200's fp64 pipe is narrow (fp64 here was ~30 % of the kernel's stall samples), so the sign of
+        // den^2 d1 - num^2 d2 is first taken in fp32: its error is below 2^-20 (den^2 + num^2)(N_Q + 2C)
+        // (d <= N_Q + 2C, a few roundings), so outside 8x that band the fp32 sign is the fp64 sign;
+        // inside it (rare) the fp64 computation decides.
+        bool pass = false;
+        if (valid && x2 >= 0) {
+          const float f1 = __int_as_float(x1), f2 = __int_as_float(x2);
+          const float base = nqv + c2f;
+          const float e1 = fmaxf(base - 2.0f * f1, 0.0f), e2 = fmaxf(base - 2.0f * f2, 0.0f);
+          const float diff = fmaf(den2f, e1, -(num2f * e2));
+          const float tol = 0x1p-17f * base * (den2f + num2f);
+          if (diff < -tol) {
+            pass = true;
+          } else if (diff <= tol) {
+            const double d1 = fmax(double(nqv) + c2 - 2.0 * double(f1), 0.0);
+            const double d2 = fmax(double(nqv) + c2 - 2.0 * double(f2), 0.0);
+            pass = double(den2) * d1 < double(num2) * d2;
+          }
+        }
         cnt += __popc(__ballot_sync(0xffffffffu, pass) & 0x33333333u);  // one thread per row
         if (++tt == T) {
           if (lane == 0 && cnt) atomicAdd(counts + static_cast<int64_t>(qi) * ldc + col0 + r, cnt);
