@@ -515,7 +515,7 @@ tid_status run_pass(tid_index* idx, const uint8_t* dq, const int32_t* nvalid, in
     }
     CU(launch_f16_match(qmap, rmap, xmap, idx->ws_f16c.as<float>(), idx->ws_f16nq.as<float>(), static_cast<int32_t>(B),
                         n, T, cnt, idx->cfg.ratio_num * idx->cfg.ratio_num, idx->cfg.ratio_den * idx->cfg.ratio_den,
-                        counts, idx->num_sms, s, W, col0, base, nvalid, idx->cpr));
+                        counts, idx->num_sms, s, W, col0, base, nvalid, idx->cpr, idx->cfg.ref_kp));
     if (idx->prof) {
       CU(cudaEventRecord(e1, s));
       idx->stats.match_launches++;
@@ -1828,7 +1828,7 @@ tid_status tid_f16_search_counts(tid_index* idx, const uint16_t* q, int32_t n, i
   TRY(make_xmap(&xmap, xop, R, static_cast<int64_t>(kBN) * fcpr));  // 32-B rows, SWIZZLE_32B
   CU(launch_f16_match(qmap, rmap, xmap, cterm, idx->ws_f16nq.as<float>(), static_cast<int32_t>(B), n, T, R,
                       idx->cfg.ratio_num * idx->cfg.ratio_num, idx->cfg.ratio_den * idx->cfg.ratio_den, counts,
-                      idx->num_sms, s, 0, 0, 0, nullptr, fcpr));
+                      idx->num_sms, s, 0, 0, 0, nullptr, fcpr, m));
   count_kernel(idx);
   if (!dev_counts) {
     bool host_out = false;

@@ -192,8 +192,11 @@ __global__ void __launch_bounds__(kThreads, 1)
                      const __grid_constant__ CUtensorMap xmap, const float* __restrict__ cterm,
                      const float* __restrict__ nq_all, int32_t B, int32_t n, int32_t T, int64_t R, int32_t q_per_job,
                      uint32_t num2, uint32_t den2, uint32_t* __restrict__ counts, int64_t ldc, int64_t col0,
-                     int64_t rbase, const int32_t* __restrict__ n_valid) {
+                     int64_t rbase, const int32_t* __restrict__ n_valid, int32_t m_rows) {
   using P = Plan<kCpr>;
+  // pieces of kFN columns that can hold reference keypoints (rows >= m_rows are padding for every
+  // reference: m = 384, the paper's operating point, computes 3 of the 4 pieces of its two chunks)
+  const int np_ref = min(kCpr * kFPieces, (m_rows + kFN - 1) / kFN);
   constexpr int kStages = P::kStages;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -272,7 +275,8 @@ __global__ void __launch_bounds__(kThreads, 1)
           const uint64_t b0 = desc128(sb + P::kR + c * 2 * kRHalf), b1 = desc128(sb + P::kR + c * 2 * kRHalf + kRHalf);
           const uint64_t bx = desc32(sb + P::kX + c * kXTile);
 #pragma unroll
-          for (int h = 0; h < kFPieces; ++h, ++gp) {
+          for (int h = 0; h < kFPieces; ++h) {
+            if (c * kFPieces + h >= np_ref) break;  // all-padding piece: neither computed nor scanned
             const int buf = gp % kFNB;
             bar_wait(tempty(buf), ((gp / kFNB) & 1) ^ 1);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
@@ -283,6 +287,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             mma_unit(tmem + buf * kFN, desc128(qa), desc128(qa + kQHalf), b0 + h * (kFN * 128 >> 4),
                      b1 + h * (kFN * 128 >> 4), ax, bx + h * (kFN * 32 >> 4), tfull(buf));
 #endif
+            ++gp;
           }
         }
         commit(qempty(st));
@@ -318,6 +323,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         // different P groups, two of one load differ in position mod 16, so the top-2 stays exact
 #pragma unroll
         for (int pc = 0; pc < kCpr * kFPieces; ++pc, ++gp) {  // one x64 load per 128 columns of a piece
+          if (pc >= np_ref) break;  // all-padding piece (not computed)
           const int buf = gp % kFNB;
           bar_wait(tfull(buf), (gp / kFNB) & 1);
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
@@ -553,8 +559,9 @@ cudaError_t launch_f16_xop_fixed(const void* r, int64_t R, int32_t m, const int3
 cudaError_t launch_f16_match(const CUtensorMap& qmap, const CUtensorMap& rmap, const CUtensorMap& xmap,
                              const float* cterm, const float* nq, int32_t B, int32_t n, int32_t T, int64_t R,
                              uint32_t num2, uint32_t den2, uint32_t* counts, int num_sms, cudaStream_t s, int64_t ldc,
-                             int64_t col0, int64_t rbase, const int32_t* n_valid, int32_t cpr) {
+                             int64_t col0, int64_t rbase, const int32_t* n_valid, int32_t cpr, int32_t m) {
   if (cpr < 1 || cpr > 2) return cudaErrorInvalidValue;
+  if (m <= 0 || m > cpr * kBN) m = cpr * kBN;
   auto kern = cpr == 1 ? f16::match_f16_kernel<1> : f16::match_f16_kernel<2>;
   const size_t smem = cpr == 1 ? f16::Plan<1>::kAlloc : f16::Plan<2>::kAlloc;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
@@ -565,7 +572,7 @@ cudaError_t launch_f16_match(const CUtensorMap& qmap, const CUtensorMap& rmap, c
   const int64_t jobs = R * ((B + qpj - 1) / qpj);
   const int grid = static_cast<int>(jobs < num_sms ? jobs : num_sms);
   kern<<<grid, f16::kThreads, smem, s>>>(qmap, rmap, xmap, cterm, nq, B, n, T, R, qpj, num2, den2, counts,
-                                       ldc > 0 ? ldc : R, col0, rbase, n_valid);
+                                       ldc > 0 ? ldc : R, col0, rbase, n_valid, m);
   return cudaGetLastError();
 }
 

@@ -158,7 +158,7 @@ cudaError_t launch_f16_match(const CUtensorMap& qmap, const CUtensorMap& rmap, c
                              const float* cterm, const float* nq, int32_t B, int32_t n, int32_t T, int64_t R,
                              uint32_t num2, uint32_t den2, uint32_t* counts, int num_sms, cudaStream_t s,
                              int64_t ldc = 0, int64_t col0 = 0, int64_t rbase = 0, const int32_t* n_valid = nullptr,
-                             int32_t cpr = 1);
+                             int32_t cpr = 1, int32_t m = 0);  // m: stored rows per reference (0 = cpr * 256)
 // index path: norm-term rows with the index's fixed constant C and per-reference keypoint counts
 cudaError_t launch_f16_xop_fixed(const void* r, int64_t R, int32_t m, const int32_t* kp, float C, float* nr, void* xop,
                                  cudaStream_t s);
