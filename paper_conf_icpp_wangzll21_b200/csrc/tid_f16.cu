@@ -186,7 +186,9 @@ __device__ __forceinline__ void finish(const int (&R)[16], int T1, int T2, int& 
   x2 = mx3(T2, sr, sc);
 }
 
-template <int kCpr>
+// kSkip: the stored m leaves all-padding 128-column pieces (m = 384: the fourth), which are neither computed
+// nor scanned; without it every loop keeps its static trip count (a run-time break cost 3 % at m = 256).
+template <int kCpr, bool kSkip>
 __global__ void __launch_bounds__(kThreads, 1)
     match_f16_kernel(const __grid_constant__ CUtensorMap qmap, const __grid_constant__ CUtensorMap rmap,
                      const __grid_constant__ CUtensorMap xmap, const float* __restrict__ cterm,
@@ -196,7 +198,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   using P = Plan<kCpr>;
   // pieces of kFN columns that can hold reference keypoints (rows >= m_rows are padding for every
   // reference: m = 384, the paper's operating point, computes 3 of the 4 pieces of its two chunks)
-  const int np_ref = min(kCpr * kFPieces, (m_rows + kFN - 1) / kFN);
+  const int np_ref = kSkip ? min(kCpr * kFPieces, (m_rows + kFN - 1) / kFN) : kCpr * kFPieces;
   constexpr int kStages = P::kStages;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -276,7 +278,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           const uint64_t bx = desc32(sb + P::kX + c * kXTile);
 #pragma unroll
           for (int h = 0; h < kFPieces; ++h) {
-            if (c * kFPieces + h >= np_ref) break;  // all-padding piece: neither computed nor scanned
+            if (kSkip && c * kFPieces + h >= np_ref) break;  // all-padding piece: neither computed nor scanned
             const int buf = gp % kFNB;
             bar_wait(tempty(buf), ((gp / kFNB) & 1) ^ 1);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
@@ -323,7 +325,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         // different P groups, two of one load differ in position mod 16, so the top-2 stays exact
 #pragma unroll
         for (int pc = 0; pc < kCpr * kFPieces; ++pc, ++gp) {  // one x64 load per 128 columns of a piece
-          if (pc >= np_ref) break;  // all-padding piece (not computed)
+          if (kSkip && pc >= np_ref) break;  // all-padding piece (not computed)
           const int buf = gp % kFNB;
           bar_wait(tfull(buf), (gp / kFNB) & 1);
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
@@ -562,7 +564,9 @@ cudaError_t launch_f16_match(const CUtensorMap& qmap, const CUtensorMap& rmap, c
                              int64_t col0, int64_t rbase, const int32_t* n_valid, int32_t cpr, int32_t m) {
   if (cpr < 1 || cpr > 2) return cudaErrorInvalidValue;
   if (m <= 0 || m > cpr * kBN) m = cpr * kBN;
-  auto kern = cpr == 1 ? f16::match_f16_kernel<1> : f16::match_f16_kernel<2>;
+  const bool skip = (m + f16::kFN - 1) / f16::kFN < cpr * f16::kFPieces;
+  auto kern = cpr == 1 ? (skip ? f16::match_f16_kernel<1, true> : f16::match_f16_kernel<1, false>)
+                       : (skip ? f16::match_f16_kernel<2, true> : f16::match_f16_kernel<2, false>);
   const size_t smem = cpr == 1 ? f16::Plan<1>::kAlloc : f16::Plan<2>::kAlloc;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
   if (e != cudaSuccess) return e;
